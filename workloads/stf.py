@@ -1,0 +1,72 @@
+"""Sequential-task-flow (STF) DAG recorder.
+
+Input generator only: it holds none of the MultiPrio arithmetic (scores,
+bottom-levels, queues).  It reproduces how the runtime infers the DAG from the
+data-access modes and the submission order (§I, l.91 §III-A:
+"the runtime system infers the DAG automatically by taking into account the
+data dependencies between tasks"), at handle granularity:
+
+* RAW / WAW: the last writer of a handle precedes every later reader/writer;
+* WAR: every reader since the last write precedes the next writer.
+
+Edges are emitted raw, duplicates included (a task reading two handles last
+written by the same predecessor produces two identical edges), exactly as a
+runtime would observe them; deduplication is step a1 of the hot path
+(SURVEY.md §8(c) reading c19).
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+class STFRecorder:
+    __slots__ = ("n", "kind", "_src", "_dst", "_last_writer", "_readers")
+
+    def __init__(self) -> None:
+        self.n = 0
+        self.kind: list[int] = []
+        self._src: list[int] = []
+        self._dst: list[int] = []
+        self._last_writer: dict = {}
+        self._readers: dict = {}
+
+    def submit(self, kind: int, reads=(), writes=()) -> int:
+        """Submit one task.  `reads` are R handles, `writes` are RW handles."""
+        t = self.n
+        self.n += 1
+        self.kind.append(kind)
+        lw_map = self._last_writer
+        rd_map = self._readers
+        src = self._src
+        dst = self._dst
+        for h in reads:
+            lw = lw_map.get(h)
+            if lw is not None:
+                src.append(lw)
+                dst.append(t)
+            lst = rd_map.get(h)
+            if lst is None:
+                rd_map[h] = [t]
+            else:
+                lst.append(t)
+        for h in writes:
+            lw = lw_map.get(h)
+            if lw is not None:
+                src.append(lw)
+                dst.append(t)
+            lst = rd_map.get(h)
+            if lst:
+                for r in lst:
+                    if r != t:
+                        src.append(r)
+                        dst.append(t)
+                rd_map[h] = []
+            lw_map[h] = t
+        return t
+
+    def edges(self) -> tuple[np.ndarray, np.ndarray]:
+        return (np.asarray(self._src, dtype=np.int32),
+                np.asarray(self._dst, dtype=np.int32))
+
+    def kinds(self) -> np.ndarray:
+        return np.asarray(self.kind, dtype=np.int32)
