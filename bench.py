@@ -1,0 +1,422 @@
+#!/usr/bin/env python
+"""bench.py -- MultiPrio scoring + queue build on B200.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config c5|c1..c4]
+
+A step is one pass of the whole hot path over one batch:
+  c5 (default): ingest the 64x64 tiled-Cholesky DAG (mp_dag_rebuild: a1+a2),
+      score + queue this rank's block of the 4096 duration-perturbed replicas
+      (mp_replicas_run: a3-a10, queues materialised in HBM), and allgather the
+      per-replica records (CP + queue summaries) over NCCL.  Total replicas
+      are fixed as N grows (strong scaling, BASELINE config 5).
+  c1..c4: one DAG per step (rebuild + bottom_level + affinity + score + queues).
+Rank 0 prints ONE JSON line.  Under torchrun every rank runs; the timed
+region is bracketed by barrier + synchronize and the per-rank device time is
+max-reduced.  `--impl reference` times the CPU oracle (the reference arm of
+this tier) on rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+import torch.distributed as dist  # noqa: E402
+
+import workloads  # noqa: E402
+
+METRIC = "DAG tasks scored+queued/sec and ms per DAG (1 GPU; replicas at 1/2/4/8 GPUs)"
+UNIT = "tasks/s"
+CONFIG_TEXT = {
+    "c1": "tiled Cholesky DAG 4x4 tiles (20 tasks), 2 resource types CPU/GPU, fixed durations",
+    "c2": "tiled dense Cholesky DAG 64x64 tiles (45,760 tasks) with StarPU-like per-kernel CPU/GPU duration model",
+    "c3": "tiled QR DAG 128x128 tiles (707,264 tasks), 3 resource types",
+    "c4": "sparse-QR-like elimination-tree DAG + FMM octree DAG (depth 8), 2,156,466 tasks, skewed fan-in",
+    "c5": "4096 duration-perturbed replicas of the 64x64 Cholesky DAG sharded across 1/2/4/8 B200",
+}
+L2_FLUSH_BYTES = 256 << 20
+KERNELS = ("k_rep_main", "k_rep_out", "k_sort_pass", "k_sort_hist", "k_sort_plan", "k_kahn", "k_pack_edges",
+           "k_dedup_flags", "k_compact_edges", "k_scan_excl", "k_iota_level_keys", "k_level_order", "k_qmaps",
+           "k_qcols", "k_bl_small", "k_bl_flow", "k_aff_hd", "k_aff_gain", "k_crit_max", "k_score",
+           "k_q_member", "k_q_scatter", "k_copy_len", "k_q_out", "k_blocked", "k_nod_indeg", "k_nod_sum",
+           "k_perturb")
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", choices=("ours", "reference"), default="ours")
+    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5"))
+    p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS)
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-budget-s", type=float, default=12.0)
+    return p.parse_args()
+
+
+def env_rank():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("LOCAL_RANK", 0)), int(os.environ.get("WORLD_SIZE", 1))
+
+
+# --------------------------------------------------------------------------------------------------
+# clocks during the timed region
+# --------------------------------------------------------------------------------------------------
+class Clocks:
+    FIELDS = ("clocks.sm", "clocks.max.sm", "clocks_event_reasons.hw_slowdown",
+              "clocks_event_reasons.hw_thermal_slowdown", "clocks_event_reasons.sw_thermal_slowdown",
+              "clocks_event_reasons.sw_power_cap")
+    NAMES = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
+
+    def __init__(self, device):
+        self.proc = None
+        self.path = None
+        sel = str(device.index or 0)
+        try:
+            uuid = str(torch.cuda.get_device_properties(device).uuid)
+            sel = uuid if uuid.startswith("GPU-") else "GPU-" + uuid
+        except Exception:
+            pass
+        self.sel = sel
+
+    def start(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", self.sel, "--query-gpu=" + ",".join(self.FIELDS), "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        time.sleep(0.15)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) != len(self.FIELDS):
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(self.NAMES, parts[2:]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        os.unlink(self.path)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# --------------------------------------------------------------------------------------------------
+# the oracle as a baseline (rank 0 only)
+# --------------------------------------------------------------------------------------------------
+def oracle_sample(cfg, w, budget_s, R):
+    import oracle
+    t0 = time.perf_counter()
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    if cfg == "c5":
+        k = 0
+        while True:
+            oracle.replica(od, w.dur, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, k, want_queue=True)
+            k += 1
+            if time.perf_counter() - t0 >= budget_s or k >= R:
+                break
+        dt = time.perf_counter() - t0
+        return k * w.n / dt, f"1 DAG build + {k} of {R} replicas of c2 (perturbation seed {workloads.C5_SEED})", dt
+    reps = 0
+    while True:
+        oracle.score_and_queue(od, w.dur, w.workers)
+        reps += 1
+        if time.perf_counter() - t0 >= budget_s:
+            break
+    dt = time.perf_counter() - t0
+    return reps * w.n / dt, f"1 DAG build + {reps} full score+queue passes of {cfg}", dt
+
+
+def run_reference(args):
+    rank, local, world = env_rank()
+    if rank != 0:
+        return
+    import oracle
+    oracle.build()
+    cfg = args.config
+    w = workloads.config("c2" if cfg == "c5" else cfg)
+    per_step_budget = 3.0 if cfg != "c4" else 10.0
+    times, tasks = [], []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        v, sample, dt = oracle_sample(cfg, w, per_step_budget, args.replicas)
+        if i >= args.warmup:
+            times.append(dt)
+            tasks.append(v * dt)
+    value = sum(tasks) / sum(times)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
+            "scaling": "none", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": CONFIG_TEXT[cfg], "name": cfg,
+                       "step": "bounded sample: " + sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------------------------------------------
+# our arm
+# --------------------------------------------------------------------------------------------------
+def kernel_alg_bytes(name, ctx):
+    """Algorithmic (compulsory) bytes per launch of the dominant kernel (DESIGN.md §6 table)."""
+    n, E, A = ctx["n"], ctx["E"], ctx["A"]
+    if name == "k_rep_main":
+        # per replica: read base durations 4nA, CSR 4(n+1)+4E once per launch; write sort input 12 B per (t,a)
+        rb = ctx["replicas_per_launch"]
+        return 4 * n * A + 4 * (n + 1) + 4 * E + rb * 12 * n * A
+    if name == "k_sort_pass":
+        return 24 * ctx["sort_entries_per_launch"]
+    if name == "k_rep_out":
+        return ctx["replicas_per_launch"] * (4 * n * A * 2)
+    if name == "k_bl_flow" or name == "k_bl_small":
+        return 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n
+    return None
+
+
+def run_ours(args):
+    import paper_conf_ipps_tayebbfg24_b200 as mp
+    from paper_conf_ipps_tayebbfg24_b200 import dist as mpd
+
+    rank, local, world = env_rank()
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE {world}")
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a CUDA device (there is no CPU path)")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    cfg = args.config
+    w = workloads.config("c2" if cfg == "c5" else cfg)
+    A = w.n_arch
+    n = w.n
+    src_h = torch.from_numpy(w.src).pin_memory()
+    dst_h = torch.from_numpy(w.dst).pin_memory()
+    dur_h = torch.from_numpy(w.dur).pin_memory()
+    src_d = src_h.to(dev)
+    dst_d = dst_h.to(dev)
+    dur_d = dur_h.to(dev)
+    dag = mp.build_dag(n, src_d, dst_d)
+    E = dag.n_edges
+    stream = torch.cuda.current_stream()
+
+    if cfg == "c5":
+        R = args.replicas
+        r0, cnt = mpd.shard_range(R, world, rank)
+        slots = mpd.shard_range(R, world, 0)[1]
+        rb = mpd.record_bytes(A)
+        out = dict(cp=torch.empty(max(cnt, 1), dtype=torch.float32, device=dev),
+                   summary=torch.empty(max(cnt, 1) * A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev),
+                   qtask=torch.empty((max(cnt, 1), n * A), dtype=torch.int32, device=dev))
+        local_rec = torch.zeros((slots, rb), dtype=torch.uint8, device=dev)
+        gathered = torch.empty((world * slots, rb), dtype=torch.uint8, device=dev)
+        result_h = torch.empty((world * slots, rb), dtype=torch.uint8).pin_memory()
+        tasks_per_step = R * n
+
+        def step():
+            mp.dag_rebuild(dag, n, src_d, dst_d)
+            mp.replicas_run(dag, dur_d, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out=out)
+            mpd.pack_records(out["cp"], out["summary"], cnt, A, slots, out=local_rec)
+            if world > 1:
+                mpd.gather_records(local_rec, out=gathered)
+            else:
+                gathered.copy_(local_rec)
+            return gathered
+    else:
+        R, cnt = 1, 1
+        outs = {}
+        tasks_per_step = n
+        result_h = torch.empty(A * mp.SUMMARY_BYTES + 4, dtype=torch.uint8).pin_memory()
+
+        def step():
+            mp.dag_rebuild(dag, n, src_d, dst_d)
+            bl, cp, _ = mp.bottom_level(dag, dur_d, w.workers, out=outs.setdefault("bl", dict(
+                bl=torch.empty(n, dtype=torch.float32, device=dev), cp=torch.empty(1, dtype=torch.float32, device=dev),
+                nod=None)))
+            gain, hd, flags = mp.affinity(dag, dur_d, w.workers, out=outs.setdefault("aff", dict(
+                gain=torch.empty((n, A), dtype=torch.float32, device=dev),
+                hd=torch.empty(A, dtype=torch.float32, device=dev),
+                flags=torch.empty((n, A), dtype=torch.uint8, device=dev))))
+            cn, key = mp.score(dag, 0, bl, gain, flags, out=outs.setdefault("sc", dict(
+                crit_norm=torch.empty(n, dtype=torch.float32, device=dev),
+                key=torch.empty((n, A), dtype=torch.int64, device=dev))))
+            qptr, qtask, summ = mp.build_queues(dag, key, flags, dur_d, out=outs.setdefault("q", dict(
+                qptr=torch.empty(A + 1, dtype=torch.int64, device=dev),
+                qtask=torch.empty(n * A, dtype=torch.int32, device=dev),
+                summary=torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev))))
+            res = outs.setdefault("res", torch.empty(A * mp.SUMMARY_BYTES + 4, dtype=torch.uint8, device=dev))
+            res[:4].copy_(cp.view(torch.uint8))
+            res[4:].copy_(summ)
+            return res
+
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    # ---- warm-up ----
+    for _ in range(max(args.warmup, 0)):
+        step()
+    mp.check(dag)
+    torch.cuda.synchronize()
+    barrier()
+
+    # ---- timed region (device time per step, L2 flushed between steps) ----
+    clocks = Clocks(dev)
+    clocks.start()
+    mp.prof_reset()
+    mp.prof_enable(True)
+    l0 = mp.launch_count()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    torch.cuda.synchronize()
+    barrier()
+    for i in range(args.steps):
+        flush.zero_()
+        evs[i][0].record(stream)
+        step()
+        evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    launches = mp.launch_count() - l0
+    mp.prof_enable(False)
+    ck = clocks.stop()
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    ms_per_step = float(tot.item()) / args.steps
+    value = tasks_per_step / (ms_per_step * 1e-3)
+    prof = {k: mp.prof_query(k) for k in KERNELS}
+    step_dev_ms = {k: v[0] / args.steps for k, v in prof.items() if v[1] > 0}
+    dom = max(step_dev_ms, key=step_dev_ms.get)
+    dom_ms, dom_launches = prof[dom]
+    mp.check(dag)
+
+    # ---- e2e: host buffers in, records out, through the public API ----
+    e2e = None
+    if not args.no_e2e:
+        eev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        torch.cuda.synchronize()
+        barrier()
+        for i in range(args.steps):
+            flush.zero_()
+            eev[i][0].record(stream)
+            src_d.copy_(src_h, non_blocking=True)
+            dst_d.copy_(dst_h, non_blocking=True)
+            dur_d.copy_(dur_h, non_blocking=True)
+            res = step()
+            result_h[: res.numel()].view(-1).copy_(res.view(-1), non_blocking=True)
+            eev[i][1].record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        et = torch.tensor([sum(a.elapsed_time(b) for a, b in eev)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        e2e_ms = float(et.item()) / args.steps
+        h2d = src_h.numel() * 4 + dst_h.numel() * 4 + dur_h.numel() * 4
+        d2h = res.numel() * res.element_size()
+        e2e = {"value": tasks_per_step / (e2e_ms * 1e-3), "unit": UNIT, "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+        peak, peak_src = float(peaks["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        peak, peak_src = 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+    ctx = dict(n=n, E=E, A=A)
+    if cfg == "c5":
+        per = (256 << 20) // (n * A * 24)
+        rpl = max(1, min(cnt, per, 1024))
+        ctx["replicas_per_launch"] = rpl
+        ctx["sort_entries_per_launch"] = rpl * A * n
+    else:
+        ctx["replicas_per_launch"] = 1
+        ctx["sort_entries_per_launch"] = n * A
+    alg = kernel_alg_bytes(dom, ctx)
+    avg_ms = dom_ms / max(dom_launches, 1)
+    achieved = (alg / (avg_ms * 1e-3) / 1e9) if alg else None
+    roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": (achieved / peak) if achieved else None, "traffic": None,
+            "alg_bytes_per_launch": alg, "avg_launch_ms": avg_ms, "launches": dom_launches,
+            "share_of_step": (dom_ms / args.steps) / ms_per_step, "peak_source": peak_src,
+            "per_kernel_ms_per_step": {k: round(v, 4) for k, v in sorted(step_dev_ms.items(), key=lambda x: -x[1])}}
+    # whole-step algorithmic bytes (SURVEY §8(d) B_alg) as context
+    if cfg == "c5":
+        b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + args.replicas * 4 * n * A / world  # CSR + dur + queues out
+    else:
+        b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 4 * n * A + 4 * n * A
+    roof["step_alg_bytes_per_gpu"] = b_alg
+    roof["step_hbm_frac"] = b_alg / (ms_per_step * 1e-3) / 1e9 / peak
+
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        import oracle
+        oracle.build()
+        v, sample, dt = oracle_sample(cfg, w, args.cpu_budget_s, args.replicas)
+        cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, "seconds": round(dt, 2)}
+
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "strong" if cfg == "c5" else "none", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
+            "config": {"workload": CONFIG_TEXT[cfg], "name": cfg, "tasks_per_dag": n, "edges": E,
+                       "levels": dag.n_levels, "archs": A,
+                       "replicas": R if cfg == "c5" else 1, "replicas_per_gpu": cnt,
+                       "ms_per_dag": ms_per_step / (R if cfg == "c5" else 1) * world if cfg == "c5" else ms_per_step,
+                       "l2": f"flushed between timed steps ({L2_FLUSH_BYTES >> 20} MiB write)",
+                       "queues": "materialised in HBM for every replica" if cfg == "c5" else "materialised",
+                       "step": "mp_dag_rebuild + mp_replicas_run + allgather(records)" if cfg == "c5"
+                       else "mp_dag_rebuild + bottom_level + affinity + score + build_queues",
+                       "parallelism": f"replica shards x{world}" if cfg == "c5" else "single DAG"},
+            "ms_per_dag": ms_per_step / (R / world) if cfg == "c5" else ms_per_step,
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
+            "gpu_launches_per_step": launches / args.steps, "clocks": ck,
+            "device": torch.cuda.get_device_name(dev)}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

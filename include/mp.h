@@ -1,0 +1,216 @@
+/*
+ * mp.h -- C-ABI of libmp, the B200 (sm_100a) implementation of MultiPrio's
+ * data-parallel scoring and queue-build path (Tayeb, Bramas, Faverge,
+ * Guermouche, "Dynamic Tasks Scheduling with Multiple Priorities on
+ * Heterogeneous Computing Systems", IPDPS'24, hal-04498634).
+ *
+ * Citations "P:l.N" refer to /root/reference/PAPER.md line N; readings cN
+ * refer to DESIGN.md §2 (= SURVEY.md §8(c)).
+ *
+ * Conventions (all entry points):
+ *  - d_* are DEVICE pointers on the current CUDA device, h_* HOST pointers.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  Every call is asynchronous on `stream` unless stated; inputs
+ *    are never modified; every output buffer is caller-owned except the
+ *    handle's internal arrays (exposed read-only by mp_dag_get_info).
+ *  - Argument errors are detected on the host and returned before any
+ *    launch.  Errors the device detects (MP_ERR_DOMAIN for durations) are
+ *    raised into a per-handle device flag and reported by mp_check(), which
+ *    synchronises `stream`; only mp_build_dag synchronises by itself.
+ *  - No C++ exception crosses the ABI.  mp_last_error() returns a thread-local
+ *    detail string for the last failing call.
+ *  - One handle is used by one stream at a time.
+ *  - Layouts: per-task-per-arch arrays are row-major [n][A] (task-major).
+ *  - Limits: 1 <= A <= 8, 0 <= n < 2^30, unique edges E < 2^31.
+ *  - Durations delta(t,a) are binary32 milliseconds in {+inf} U {0} U
+ *    [2^-41, 2^20); +inf = "t has no implementation on a" (can_exec false,
+ *    P:l.91, l.135); -0 is read as +0; anything else (NaN, negative, nonzero
+ *    below 2^-41, finite >= 2^20) or a task with no enabled arch is
+ *    MP_ERR_DOMAIN (reading c20).  An arch a is enabled iff h_workers[a] > 0
+ *    (get_worker_count(a) > 0, Alg. 1 P:l.135).
+ *  - All float results are bit-exact with the CPU oracle: every binary32 op
+ *    is an explicit round-to-nearest-even op, no FMA contraction, sums are
+ *    exact integers.
+ */
+#ifndef MP_H
+#define MP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct mp_dag mp_dag; /* opaque; owns the CSR, levels and workspaces */
+
+typedef enum {
+    MP_OK = 0,
+    MP_ERR_ARG = 1,    /* bad argument / id out of range / self-loop        */
+    MP_ERR_CYCLE = 2,  /* the edge set is not a DAG                         */
+    MP_ERR_DOMAIN = 3, /* duration outside the domain above                 */
+    MP_ERR_CUDA = 4,   /* a CUDA runtime error (detail in mp_last_error)     */
+    MP_ERR_NOMEM = 5   /* device allocation failed                          */
+} mp_status;
+
+typedef enum {
+    MP_CRIT_BOTTOM_LEVEL = 0, /* bl(t) / CP, arch-independent (north_star)    */
+    MP_CRIT_NOD = 1           /* NOD_a(t) / max_t NOD_a, eq. 2 P:l.193         */
+} mp_crit;
+
+/* Read-only views of the handle's device arrays (valid until mp_free). */
+typedef struct {
+    int32_t n_tasks;
+    int64_t n_edges;         /* unique edges                                  */
+    int32_t n_levels;        /* L = 1 + max level (0 when n = 0)              */
+    int32_t max_width;       /* max tasks in one level                        */
+    const int32_t* d_row_ptr;     /* [n+1] successor CSR offsets              */
+    const int32_t* d_col;         /* [E]   successor ids, ascending per row   */
+    const int32_t* d_indeg;       /* [n]   |lambda^-(t)|                       */
+    const int32_t* d_level;       /* [n]   0 if no predecessor else 1+max     */
+    const int32_t* d_level_ptr;   /* [L+1] offsets of each level in order     */
+    const int32_t* d_level_order; /* [n]   ids sorted by (level, id)          */
+} mp_dag_info;
+
+/* One priority queue's counters (Alg. 1, P:l.135). */
+typedef struct {
+    int32_t count;   /* ready_tasks_count: entries in the queue              */
+    int32_t head;    /* task id at the root of the heap (queue[0]) or -1     */
+    uint64_t brw_lo; /* best_remaining_work = sum of delta(t,a) over entries */
+    int64_t brw_hi;  /*   with delta(t,a) == min_a' delta(t,a'), as the exact */
+                     /*   128-bit integer hi:lo in units of 2^-64 ms          */
+    double brw;      /* that exact value rounded once to binary64            */
+} mp_queue_summary;  /* 32 bytes */
+
+/*
+ * a1 + a2: DAG ingest and topological levels.
+ * Builds G = (V, E) from n_edges (src -> dst) pairs: "for each edge
+ * (t_i, t_j), t_j cannot start before the completion of t_i" (P:l.89);
+ * lambda^+/- are sets (Table I, P:l.83-84) so duplicate pairs collapse
+ * (reading c19).  Levels: level(t) = 0 if lambda^-(t) is empty else
+ * 1 + max level(p), p in lambda^-(t); level_order lists ids by (level, id).
+ * d_src/d_dst: device int32[n_edges]; may be NULL when n_edges = 0.
+ * Errors: MP_ERR_ARG for n < 0, id outside [0, n) or a self-loop;
+ * MP_ERR_CYCLE when the pairs contain a cycle.  Synchronises `stream` once.
+ * On success *out owns its device buffers (release with mp_free).
+ */
+mp_status mp_build_dag(int32_t n_tasks, int64_t n_edges, const int32_t* d_src,
+                       const int32_t* d_dst, void* stream, mp_dag** out);
+
+/*
+ * Same as mp_build_dag, into an existing handle: the previous DAG is replaced
+ * and the handle's device buffers are reused (grow-only), so re-ingesting a
+ * DAG no larger than an earlier one performs no device allocation.  On error
+ * the handle holds an empty DAG (n = 0) and stays valid for mp_free.
+ */
+mp_status mp_dag_rebuild(mp_dag* dag, int32_t n_tasks, int64_t n_edges, const int32_t* d_src,
+                         const int32_t* d_dst, void* stream);
+
+mp_status mp_dag_get_info(const mp_dag* dag, mp_dag_info* out);
+
+/*
+ * a3 + a4 (+ a5): bottom-level criticality (north_star) and, optionally, the
+ * paper's NOD criticality (eq. 2, P:l.191-193).
+ *   w(t)  = min over enabled a of delta(t,a)            (reading c2, P:l.265)
+ *   bl(t) = w(t) + max_{s in lambda^+(t)} bl(s), or w(t) without successors
+ *   *d_cp = CP = max_t bl(t)
+ *   NOD_a(t) = sum_{s in lambda^+(t), s enabled on a} 1/|{p in lambda^-(s) :
+ *             p enabled on a}| for (t,a) enabled, else 0 (reading c10); each
+ *             term is floor(2^32/k), the sum an exact 64-bit integer, converted
+ *             once to binary32 and scaled by 2^-32 (reading c11).
+ * d_dur: float[n][A]; h_workers: int32[A]; d_bl: float[n]; d_cp: float[1];
+ * d_nod: float[n][A] or NULL.  Domain errors -> device flag (mp_check).
+ */
+mp_status mp_bottom_level(mp_dag* dag, int32_t n_arch, const float* d_dur,
+                          const int32_t* h_workers, float* d_bl, float* d_cp,
+                          float* d_nod, void* stream);
+
+/*
+ * a6: gain heuristic, eq. 1 (P:l.172), hd(a) (P:l.176), Table II (P:l.180-187).
+ *   ref(t,a) = min over enabled a' != a of delta(t,a')   (reading c6)
+ *   d(t,a)   = ref - delta(t,a)
+ *   hd(a)    = max |d(t,a)| over tasks with >= 2 enabled archs incl. a (c4, c5)
+ *   gain     = 1 if t has one enabled arch (P:l.170, c7); 0.5 if hd(a) = 0 (c8);
+ *              else (d + hd) / (hd + hd); 0 where (t,a) is not enabled.
+ * d_gain: float[n][A]; d_hd: float[A];
+ * d_flags: uint8[n][A], bit0 = enabled(t,a), bit1 = delta(t,a) == w(t)
+ *   ("normalized_speedup(t,a) == 1", Alg. 1, reading c15).
+ */
+mp_status mp_affinity(mp_dag* dag, int32_t n_arch, const float* d_dur,
+                      const int32_t* h_workers, float* d_gain, float* d_hd,
+                      uint8_t* d_flags, void* stream);
+
+/*
+ * a7: normalised criticality and the combined key.  "All values are
+ * normalized between 0 and 1" (P:l.166): crit_n = crit / max crit (reading
+ * c9; 0 when the max is 0).  Tasks are ordered by gain first, criticality on
+ * equal gain (P:l.138, l.322):
+ *   key(t,a) = ((0x3F800000 - bits(gain)) << 32) | (0x3F800000 - bits(crit_n))
+ * so ascending key = (gain desc, crit_n desc); UINT64_MAX where not enabled.
+ * kind = MP_CRIT_BOTTOM_LEVEL: d_crit = bl float[n], d_crit_norm float[n];
+ * kind = MP_CRIT_NOD: d_crit = nod float[n][A], normalised per arch over
+ *   enabled tasks, d_crit_norm float[n][A].   d_key: uint64[n][A].
+ */
+mp_status mp_score(mp_dag* dag, int32_t n_arch, mp_crit kind, const float* d_crit,
+                   const float* d_gain, const uint8_t* d_flags, float* d_crit_norm,
+                   uint64_t* d_key, void* stream);
+
+/*
+ * a8 + a9: one priority queue per architecture type (the heaps h_m of
+ * P:l.97-106, l.130; memory nodes of one arch share a queue, reading c13).
+ * Queue a holds {t : enabled(t,a) and (d_done == NULL or ready(t))},
+ * ready(t) = !done(t) and all predecessors done (P:l.91, reading c18),
+ * sorted by (key ascending, id ascending) (reading c12); a sorted array is a
+ * valid binary max-heap.  d_qptr: int64[A+1] offsets into d_qtask (capacity
+ * n*A int32); d_sum: mp_queue_summary[A] (count, head, best_remaining_work
+ * over entries with flags bit1).  d_dur supplies delta for the brw sums.
+ */
+mp_status mp_build_queues(mp_dag* dag, int32_t n_arch, const uint64_t* d_key,
+                          const uint8_t* d_flags, const float* d_dur,
+                          const uint8_t* d_done, int64_t* d_qptr, int32_t* d_qtask,
+                          mp_queue_summary* d_sum, void* stream);
+
+/*
+ * a10: batched replicas.  For r in [r0, r0+R):
+ *   delta_r(t,a) = delta(t,a) * (1 + sigma * (2u - 1)), u = (splitmix64(seed
+ *   + c * 0x9E3779B97F4A7C15) >> 40) * 2^-24 with counter
+ *   c = (r*n + t)*A + a + 1, each float op RN binary32 (north_star
+ *   "duration-perturbed instances of one DAG"); then a3-a9 with
+ *   MP_CRIT_BOTTOM_LEVEL in ALL mode.  Replica results depend only on the
+ *   global replica id r (world-size invariant).
+ * d_base_dur: float[n][A]; d_cp: float[R]; d_sum: mp_queue_summary[R][A];
+ * d_qtask: int32[R][n*A] (queue a of replica r at offset r*n*A + qoff_a, where
+ *   qoff_a = sum of that replica's counts of archs < a) or NULL.
+ */
+mp_status mp_replicas_run(mp_dag* dag, int32_t n_arch, const float* d_base_dur,
+                          const int32_t* h_workers, uint64_t seed, float sigma,
+                          int64_t r0, int32_t R, float* d_cp, mp_queue_summary* d_sum,
+                          int32_t* d_qtask, void* stream);
+
+/* Synchronise `stream`, then return (and clear) the handle's device error
+ * flag: MP_OK or MP_ERR_DOMAIN; MP_ERR_CUDA on a pending CUDA error. */
+mp_status mp_check(mp_dag* dag, void* stream);
+
+/* NULL-safe.  Synchronises the device before releasing the buffers. */
+void mp_free(mp_dag* dag);
+
+const char* mp_status_str(mp_status s);
+const char* mp_last_error(void);
+
+/* Library introspection for tests: "sm_100a", version string. */
+const char* mp_build_info(void);
+
+/* Diagnostics.  mp_launch_count: kernels libmp has launched in this process.
+ * mp_prof_enable(1): bracket every launch with CUDA events on its stream;
+ * mp_prof_query synchronises on those events and returns the summed device
+ * time (ms) and launch count of kernel `name` (e.g. "k_sort_pass") since the
+ * last mp_prof_reset.  Host-side bookkeeping only; results are unaffected. */
+uint64_t mp_launch_count(void);
+void mp_prof_enable(int on);
+void mp_prof_reset(void);
+mp_status mp_prof_query(const char* name, double* total_ms, int64_t* launches);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* MP_H */

@@ -1,0 +1,424 @@
+// build.cuh -- a1 + a2: DAG ingest (deduplicated successor CSR) and topological
+// levels, plus the reverse-level "q-space" layouts the bottom-level kernels
+// walk.  PAPER.md l.83-84 (Table I: lambda^-, lambda^+ as sets), l.89 (G=(V,E)),
+// l.91 (a task is ready when all its predecessors are done).
+#pragma once
+#include <cooperative_groups.h>
+
+#include <vector>
+
+#include "handle.cuh"
+
+namespace cg = cooperative_groups;
+
+namespace mpk {
+
+// validate and pack (src, dst) into sortable keys src << b | dst
+__global__ void k_pack_edges(const int32_t* src, const int32_t* dst, int64_t m, int32_t n, int b,
+                             uint64_t* keys, uint32_t* err) {
+    int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    bool bad = false;
+    for (; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t u = src[i], v = dst[i];
+        if (u < 0 || u >= n || v < 0 || v >= n || u == v) {
+            bad = true;
+            keys[i] = 0;
+        } else {
+            keys[i] = ((uint64_t)(uint32_t)u << b) | (uint32_t)v;
+        }
+    }
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(err, ERR_ARG_BIT);
+}
+
+__global__ void k_dedup_flags(const SortPlan* plan, uint64_t* const* kb, int64_t m, int32_t* flag) {
+    const uint64_t* k = kb[plan->final_sel];
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
+        flag[i] = (i == 0 || k[i] != k[i - 1]) ? 1 : 0;
+}
+
+__global__ void k_compact_edges(const SortPlan* plan, uint64_t* const* kb, int64_t m, int b,
+                                const int32_t* flag_in, const int32_t* pos, int32_t* col, int32_t* outdeg,
+                                int32_t* indeg) {
+    const uint64_t* k = kb[plan->final_sel];
+    const uint64_t mask = (1ull << b) - 1;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+        bool uniq = (i == 0 || k[i] != k[i - 1]);
+        (void)flag_in;
+        if (!uniq) continue;
+        uint64_t key = k[i];
+        int32_t u = (int32_t)(key >> b), v = (int32_t)(key & mask);
+        col[pos[i]] = v;
+        atomicAdd(&outdeg[u], 1);
+        atomicAdd(&indeg[v], 1);
+    }
+}
+
+struct KahnArgs {
+    int32_t n;
+    const int32_t* row_ptr;
+    const int32_t* col;
+    const int32_t* indeg;
+    int32_t* rem;
+    int32_t* level;
+    int32_t* front[2];
+    int32_t* counts;      // [n+2], zeroed: counts[k] = size of frontier k
+    int32_t* out;         // [0] = number of levels L, [1] = processed
+    uint32_t* err;
+};
+
+// Kahn level-synchronous frontier expansion in one cooperative kernel with a
+// grid barrier per level; appends use warp-aggregated atomics.
+__global__ void k_kahn(KahnArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = gtid; v < a.n; v += gsz) {
+        int32_t d = a.indeg[v];
+        a.rem[v] = d;
+        a.level[v] = 0;
+        if (d == 0) {
+            cg::coalesced_group g = cg::coalesced_threads();
+            int32_t base = 0;
+            if (g.thread_rank() == 0) base = atomicAdd(&a.counts[0], (int32_t)g.size());
+            base = g.shfl(base, 0);
+            a.front[0][base + g.thread_rank()] = (int32_t)v;
+        }
+    }
+    grid.sync();
+    int32_t k = 0;
+    int64_t processed = 0;
+    while (true) {
+        const int32_t cnt = *((volatile int32_t*)&a.counts[k]);
+        if (cnt == 0) break;
+        processed += cnt;
+        const int32_t* cur = a.front[k & 1];
+        int32_t* nxt = a.front[(k + 1) & 1];
+        for (int64_t i = gtid; i < cnt; i += gsz) {
+            int32_t u = cur[i];
+            for (int32_t e = a.row_ptr[u]; e < a.row_ptr[u + 1]; e++) {
+                int32_t v = a.col[e];
+                if (atomicSub(&a.rem[v], 1) == 1) {
+                    a.level[v] = k + 1;
+                    cg::coalesced_group g = cg::coalesced_threads();
+                    int32_t base = 0;
+                    if (g.thread_rank() == 0) base = atomicAdd(&a.counts[k + 1], (int32_t)g.size());
+                    base = g.shfl(base, 0);
+                    nxt[base + g.thread_rank()] = v;
+                }
+            }
+        }
+        k++;
+        grid.sync();
+    }
+    if (gtid == 0) {
+        a.out[0] = k;
+        a.out[1] = (int32_t)processed;
+        if (processed < a.n) atomicOr(a.err, ERR_CYCLE_BIT);
+    }
+}
+
+__global__ void k_iota_level_keys(const int32_t* level, int32_t n, uint64_t* keys, uint32_t* vals) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        keys[v] = (uint64_t)(uint32_t)level[v];
+        vals[v] = (uint32_t)v;
+    }
+}
+
+__global__ void k_level_order(const SortPlan* plan, uint64_t* const* kb, uint32_t* const* vb, int32_t n,
+                              int32_t* level_order, int32_t* level_ptr, int32_t* pos) {
+    const uint64_t* k = kb[plan->final_sel];
+    const uint32_t* v = vb[plan->final_sel];
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t id = (int32_t)v[i];
+        level_order[i] = id;
+        pos[id] = (int32_t)i;
+        if (i == 0 || k[i] != k[i - 1]) level_ptr[k[i]] = (int32_t)i;
+    }
+}
+
+// q-space maps: reverse levels, ids ascending inside a level; and the padded variant.
+__global__ void k_qmaps(int32_t n, const int32_t* level, const int32_t* level_ptr, const int32_t* pos,
+                        const int32_t* lvlq, const int32_t* lvlp, int32_t L, const int32_t* row_ptr,
+                        int32_t* qof, int32_t* nodeq, int32_t* degq, int32_t* pof, int32_t* nodep,
+                        int32_t* degp) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        int32_t l = level[v];
+        int32_t i = pos[v] - level_ptr[l];
+        int32_t r = L - 1 - l;
+        int32_t q = lvlq[r] + i;
+        int32_t p = lvlp[r] + i;
+        int32_t d = row_ptr[v + 1] - row_ptr[v];
+        qof[v] = q;
+        nodeq[q] = (int32_t)v;
+        degq[q] = d;
+        pof[v] = p;
+        nodep[p] = (int32_t)v;
+        degp[p] = d;
+    }
+}
+
+// colX[rowX[x] + j] = map[col[row_ptr[v] + j]] for every position x of node v (warp per node)
+__global__ void k_qcols(int32_t npos, const int32_t* nodeX, const int32_t* rowX, const int32_t* row_ptr,
+                        const int32_t* col, const int32_t* map, int32_t* colX) {
+    const int lane = threadIdx.x & 31;
+    int64_t wid = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t x = wid; x < npos; x += nw) {
+        int32_t v = nodeX[x];
+        if (v < 0) continue;
+        int32_t b = row_ptr[v], e = row_ptr[v + 1], o = rowX[x];
+        for (int32_t j = b + lane; j < e; j += 32) colX[o + (j - b)] = map[col[j]];
+    }
+}
+
+}  // namespace mpk
+
+namespace mph {
+
+inline int bits_for(int64_t x) {  // smallest b >= 1 with x <= 2^b
+    int b = 1;
+    while ((1ll << b) < x) b++;
+    return b;
+}
+
+inline int grid_for(int64_t n, int threads = 256, int64_t cap = 148 * 32) {
+    int64_t g = (n + threads - 1) / threads;
+    if (g < 1) g = 1;
+    if (g > cap) g = cap;
+    return (int)g;
+}
+
+// (Re)build the DAG held by `dag`.  Device arrays are grow-only: rebuilding a
+// DAG no larger than a previous one allocates nothing.
+inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_src, const int32_t* d_dst,
+                            cudaStream_t st) {
+    using namespace mpk;
+    if (n < 0 || n >= (1 << 30)) return fail(MP_ERR_ARG, "n_tasks %d outside [0, 2^30)", n);
+    if (m < 0 || m >= (1ll << 31)) return fail(MP_ERR_ARG, "n_edges %lld outside [0, 2^31)", (long long)m);
+    if (m > 0 && (!d_src || !d_dst)) return fail(MP_ERR_ARG, "edge arrays are NULL");
+    if (m > 0 && n == 0) return fail(MP_ERR_ARG, "edges given for an empty task set");
+    auto cleanup = [&](mp_status s) {
+        dag->n = 0;
+        dag->E = 0;
+        dag->L = 0;
+        return s;
+    };
+    cudaGetDevice(&dag->device);
+    cudaDeviceGetAttribute(&dag->num_sms, cudaDevAttrMultiProcessorCount, dag->device);
+    dag->n = n;
+    const int64_t nn = n > 0 ? n : 1;
+    const int64_t mm = m > 0 ? m : 1;
+#define ALLOC(ptr, cnt)                                                                     \
+    do {                                                                                    \
+        mp_status s__ = grow_buf((void**)&(ptr), (size_t)(cnt) * sizeof(*(ptr)), dag, st); \
+        if (s__) return cleanup(s__);                                                       \
+    } while (0)
+#define CK(call)                                                                            \
+    do {                                                                                    \
+        cudaError_t e__ = (call);                                                           \
+        if (e__) return cleanup(fail(MP_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e__))); \
+    } while (0)
+
+    ALLOC(dag->err, 4);
+    ALLOC(dag->tickets, 64);
+    ALLOC(dag->row_ptr, nn + 1);
+    ALLOC(dag->indeg, nn);
+    ALLOC(dag->level, nn);
+    ALLOC(dag->level_ptr, nn + 1);
+    ALLOC(dag->level_order, nn);
+    ALLOC(dag->qof, nn);
+    ALLOC(dag->nodeq, nn);
+    ALLOC(dag->rowq, nn + 1);
+    CK(cudaMemsetAsync(dag->err, 0, 16, st));
+    CK(cudaMemsetAsync(dag->tickets, 0, 64 * 4, st));
+    CK(cudaMemsetAsync(dag->row_ptr, 0, (nn + 1) * 4, st));
+    CK(cudaMemsetAsync(dag->indeg, 0, nn * 4, st));
+
+    // ---- a1: sort (src,dst) pairs, dedup, CSR -------------------------------------------
+    const int b = bits_for(n > 1 ? n : 2);
+    const int npass = (2 * b + 7) / 8;
+    const int64_t tps = (mm + SORT_TILE - 1) / SORT_TILE;
+    size_t bytes = sort_bytes(mm, 1, npass, false) + 2 * align256(mm * 4) + align256(64);
+    {
+        mp_status s = ensure_ws(dag, bytes, st);
+        if (s) return cleanup(s);
+        s = ensure_sort_status(dag, (size_t)tps * 256, st);
+        if (s) return cleanup(s);
+    }
+    Arena ar{dag->ws, dag->ws_cap};
+    SortArgs sa = carve_sort(ar, dag, mm, 1, 0, npass, false);
+    int32_t* flag = ar.take<int32_t>(mm);
+    int32_t* posb = ar.take<int32_t>(mm);
+    uint64_t** kb = ar.take<uint64_t*>(2);
+    int32_t* d_scal = ar.take<int32_t>(8);  // [0]=E
+    ALLOC(dag->col, mm);
+    if (m > 0) {
+        uint64_t* hk[2] = {sa.keys[0], sa.keys[1]};
+        CK(cudaMemcpyAsync(kb, hk, sizeof(hk), cudaMemcpyHostToDevice, st));
+        MP_LAUNCH(k_pack_edges, grid_for(m), 256, 0, st, d_src, d_dst, m, n, b, sa.keys[0], dag->err);
+        sa.seg_len = m;
+        {
+            mp_status s = run_sort(dag, sa, st);
+            if (s) return cleanup(s);
+        }
+        MP_LAUNCH(k_dedup_flags, grid_for(m), 256, 0, st, sa.plans, kb, m, flag);
+        {
+            mp_status s = scan(dag, flag, posb, m, d_scal, st);
+            if (s) return cleanup(s);
+        }
+        MP_LAUNCH(k_compact_edges, grid_for(m), 256, 0, st, sa.plans, kb, m, b, flag, posb, dag->col, dag->row_ptr,
+                                                      dag->indeg);
+    } else {
+        CK(cudaMemsetAsync(d_scal, 0, 4, st));
+    }
+    if (n > 0) {
+        mp_status s = scan(dag, dag->row_ptr, dag->row_ptr, (int64_t)n + 1, nullptr, st);
+        if (s) return cleanup(s);
+    }
+
+    // ---- a2: Kahn levels ----------------------------------------------------------------
+    ALLOC(dag->b_rem, nn);
+    ALLOC(dag->b_f0, nn);
+    ALLOC(dag->b_f1, nn);
+    ALLOC(dag->b_counts, nn + 2);
+    ALLOC(dag->b_kout, 4);
+    int32_t* rem = dag->b_rem;
+    int32_t* f0 = dag->b_f0;
+    int32_t* f1 = dag->b_f1;
+    int32_t* counts = dag->b_counts;
+    int32_t* kout = dag->b_kout;
+    CK(cudaMemsetAsync(counts, 0, (nn + 2) * 4, st));
+    CK(cudaMemsetAsync(kout, 0, 16, st));
+    if (n > 0) {
+        KahnArgs ka{n, dag->row_ptr, dag->col, dag->indeg, rem, dag->level, {f0, f1}, counts, kout, dag->err};
+        int bps = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_kahn, 256, 0));
+        int64_t want = (n + 255) / 256;
+        int64_t g = (int64_t)bps * dag->num_sms;
+        if (want < g) g = want;
+        if (g < 1) g = 1;
+        void* args[] = {&ka};
+        mph::ProfScope kahn_scope("k_kahn", st);
+        CK(cudaLaunchCooperativeKernel((void*)k_kahn, dim3((unsigned)g), dim3(256), args, 0, st));
+    }
+    int32_t h_scal[2] = {0, 0};
+    int32_t h_k[2] = {0, 0};
+    uint32_t h_err = 0;
+    CK(cudaMemcpyAsync(h_scal, d_scal, 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h_k, kout, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&h_err, dag->err, 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (h_err & ERR_ARG_BIT) return cleanup(fail(MP_ERR_ARG, "edge id outside [0, n) or self-loop"));
+    if (h_err & ERR_CYCLE_BIT) return cleanup(fail(MP_ERR_CYCLE, "edges contain a cycle (%d of %d tasks levelled)", h_k[1], n));
+    dag->E = m > 0 ? h_scal[0] : 0;
+    dag->L = h_k[0];
+    const int32_t L = dag->L;
+
+    // ---- canonical level order: stable sort of ids by level ---------------------------
+    if (n > 0) {
+        const int lb = bits_for(L + 1);
+        const int lp = (lb + 7) / 8;
+        Arena ar2{dag->ws, dag->ws_cap};
+        size_t need = sort_bytes(nn, 1, lp, true) + align256(64);
+        {
+            mp_status s = ensure_ws(dag, need, st);
+            if (s) return cleanup(s);
+            ar2 = Arena{dag->ws, dag->ws_cap};
+        }
+        SortArgs ls = carve_sort(ar2, dag, n, 1, 0, lp, true);
+        uint64_t** kb2 = ar2.take<uint64_t*>(2);
+        uint32_t** vb2 = ar2.take<uint32_t*>(2);
+        uint64_t* hk[2] = {ls.keys[0], ls.keys[1]};
+        uint32_t* hv[2] = {ls.vals[0], ls.vals[1]};
+        CK(cudaMemcpyAsync(kb2, hk, sizeof(hk), cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(vb2, hv, sizeof(hv), cudaMemcpyHostToDevice, st));
+        MP_LAUNCH(k_iota_level_keys, grid_for(n), 256, 0, st, dag->level, n, ls.keys[0], ls.vals[0]);
+        {
+            mp_status s = run_sort(dag, ls, st);
+            if (s) return cleanup(s);
+        }
+        // pos[] reuses rem (free after)
+        MP_LAUNCH(k_level_order, grid_for(n), 256, 0, st, ls.plans, kb2, vb2, n, dag->level_order, dag->level_ptr, rem);
+        CK(cudaMemcpyAsync(dag->level_ptr + L, &dag->n, 4, cudaMemcpyHostToDevice, st));
+        std::vector<int32_t> lp_h((size_t)L + 1);
+        CK(cudaMemcpyAsync(lp_h.data(), dag->level_ptr, ((size_t)L + 1) * 4, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        lp_h[L] = n;
+        // reverse-level offsets, unpadded and padded to 32
+        std::vector<int32_t> lq((size_t)L + 1), lpp((size_t)L + 1);
+        int32_t mw = 0;
+        lq[0] = 0;
+        lpp[0] = 0;
+        for (int32_t r = 0; r < L; r++) {
+            int32_t l = L - 1 - r;
+            int32_t w = lp_h[l + 1] - lp_h[l];
+            if (w > mw) mw = w;
+            lq[r + 1] = lq[r] + w;
+            lpp[r + 1] = lpp[r] + ((w + 31) / 32) * 32;
+        }
+        dag->max_width = mw;
+        dag->P = lpp[L];
+        const int64_t P = dag->P;
+        ALLOC(dag->lvlq, L + 1);
+        ALLOC(dag->lvlp, L + 1);
+        ALLOC(dag->nodep, P);
+        ALLOC(dag->rowp, P + 1);
+        ALLOC(dag->colq, dag->E > 0 ? dag->E : 1);
+        ALLOC(dag->colp, dag->E > 0 ? dag->E : 1);
+        ALLOC(dag->b_pof, nn);
+        int32_t* pof = dag->b_pof;
+        CK(cudaMemcpyAsync(dag->lvlq, lq.data(), ((size_t)L + 1) * 4, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(dag->lvlp, lpp.data(), ((size_t)L + 1) * 4, cudaMemcpyHostToDevice, st));
+        CK(cudaMemsetAsync(dag->nodep, 0xff, P * 4, st));
+        CK(cudaMemsetAsync(dag->rowp, 0, (P + 1) * 4, st));
+        CK(cudaMemsetAsync(dag->rowq, 0, (nn + 1) * 4, st));
+        MP_LAUNCH(k_qmaps, grid_for(n), 256, 0, st, n, dag->level, dag->level_ptr, rem, dag->lvlq, dag->lvlp, L,
+                                             dag->row_ptr, dag->qof, dag->nodeq, dag->rowq, pof, dag->nodep,
+                                             dag->rowp);
+        {
+            mp_status s = scan(dag, dag->rowq, dag->rowq, (int64_t)n + 1, nullptr, st);
+            if (s) return cleanup(s);
+            s = scan(dag, dag->rowp, dag->rowp, P + 1, nullptr, st);
+            if (s) return cleanup(s);
+        }
+        if (dag->E > 0) {
+            MP_LAUNCH(k_qcols, grid_for((int64_t)n * 32), 256, 0, st, n, dag->nodeq, dag->rowq, dag->row_ptr, dag->col,
+                                                              dag->qof, dag->colq);
+            MP_LAUNCH(k_qcols, grid_for(P * 32), 256, 0, st, (int32_t)P, dag->nodep, dag->rowp, dag->row_ptr, dag->col,
+                                                     pof, dag->colp);
+        }
+    } else {
+        ALLOC(dag->lvlq, 1);
+        ALLOC(dag->lvlp, 1);
+        ALLOC(dag->nodep, 1);
+        ALLOC(dag->rowp, 1);
+        ALLOC(dag->colq, 1);
+        ALLOC(dag->colp, 1);
+        CK(cudaMemsetAsync(dag->lvlq, 0, 4, st));
+        CK(cudaMemsetAsync(dag->lvlp, 0, 4, st));
+        CK(cudaMemsetAsync(dag->rowp, 0, 4, st));
+        CK(cudaMemsetAsync(dag->rowq, 0, 4, st));
+        CK(cudaMemsetAsync(dag->level_ptr, 0, 4, st));
+    }
+    CK(cudaStreamSynchronize(st));
+    CK(cudaGetLastError());
+#undef ALLOC
+#undef CK
+    return MP_OK;
+}
+
+inline mp_status build_dag(int32_t n, int64_t m, const int32_t* d_src, const int32_t* d_dst, cudaStream_t st,
+                           mp_dag** out) {
+    if (!out) return fail(MP_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    mp_dag* dag = new mp_dag();
+    mp_status s = build_into(dag, n, m, d_src, d_dst, st);
+    if (s != MP_OK) {
+        mp_free(dag);
+        return s;
+    }
+    *out = dag;
+    return MP_OK;
+}
+
+}  // namespace mph

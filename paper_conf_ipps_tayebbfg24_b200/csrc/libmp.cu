@@ -1,0 +1,132 @@
+// libmp.cu -- the C-ABI of include/mp.h.  Single translation unit: every
+// kernel lives in the headers included below.  Argument marshalling and
+// launch sequencing only; every step of the path runs in those kernels.
+#include <cstdarg>
+#include <vector>
+
+#include "replicas.cuh"
+
+static inline cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
+
+extern "C" {
+
+mp_status mp_build_dag(int32_t n_tasks, int64_t n_edges, const int32_t* d_src, const int32_t* d_dst, void* stream,
+                       mp_dag** out) {
+    return mph::build_dag(n_tasks, n_edges, d_src, d_dst, as_stream(stream), out);
+}
+
+mp_status mp_dag_rebuild(mp_dag* dag, int32_t n_tasks, int64_t n_edges, const int32_t* d_src,
+                         const int32_t* d_dst, void* stream) {
+    if (!dag) return mph::fail(MP_ERR_ARG, "dag is NULL");
+    return mph::build_into(dag, n_tasks, n_edges, d_src, d_dst, as_stream(stream));
+}
+
+mp_status mp_dag_get_info(const mp_dag* dag, mp_dag_info* out) {
+    if (!dag || !out) return mph::fail(MP_ERR_ARG, "NULL argument");
+    out->n_tasks = dag->n;
+    out->n_edges = dag->E;
+    out->n_levels = dag->L;
+    out->max_width = dag->max_width;
+    out->d_row_ptr = dag->row_ptr;
+    out->d_col = dag->col;
+    out->d_indeg = dag->indeg;
+    out->d_level = dag->level;
+    out->d_level_ptr = dag->level_ptr;
+    out->d_level_order = dag->level_order;
+    return MP_OK;
+}
+
+mp_status mp_bottom_level(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers, float* d_bl,
+                          float* d_cp, float* d_nod, void* stream) {
+    return mph::bottom_level(dag, n_arch, d_dur, h_workers, d_bl, d_cp, d_nod, as_stream(stream));
+}
+
+mp_status mp_affinity(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers, float* d_gain,
+                      float* d_hd, uint8_t* d_flags, void* stream) {
+    return mph::affinity(dag, n_arch, d_dur, h_workers, d_gain, d_hd, d_flags, as_stream(stream));
+}
+
+mp_status mp_score(mp_dag* dag, int32_t n_arch, mp_crit kind, const float* d_crit, const float* d_gain,
+                   const uint8_t* d_flags, float* d_crit_norm, uint64_t* d_key, void* stream) {
+    return mph::score(dag, n_arch, (int32_t)kind, d_crit, d_gain, d_flags, d_crit_norm, d_key, as_stream(stream));
+}
+
+mp_status mp_build_queues(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, const uint8_t* d_flags,
+                          const float* d_dur, const uint8_t* d_done, int64_t* d_qptr, int32_t* d_qtask,
+                          mp_queue_summary* d_sum, void* stream) {
+    return mph::build_queues(dag, n_arch, d_key, d_flags, d_dur, d_done, d_qptr, d_qtask, d_sum, as_stream(stream));
+}
+
+mp_status mp_replicas_run(mp_dag* dag, int32_t n_arch, const float* d_base_dur, const int32_t* h_workers,
+                          uint64_t seed, float sigma, int64_t r0, int32_t R, float* d_cp, mp_queue_summary* d_sum,
+                          int32_t* d_qtask, void* stream) {
+    return mph::replicas_run(dag, n_arch, d_base_dur, h_workers, seed, sigma, r0, R, d_cp, d_sum, d_qtask,
+                             as_stream(stream));
+}
+
+mp_status mp_check(mp_dag* dag, void* stream) {
+    if (!dag) return mph::fail(MP_ERR_ARG, "dag is NULL");
+    cudaStream_t st = as_stream(stream);
+    MP_CUDA(cudaStreamSynchronize(st));
+    MP_CUDA(cudaGetLastError());
+    uint32_t e = 0;
+    MP_CUDA(cudaMemcpy(&e, dag->err, 4, cudaMemcpyDeviceToHost));
+    if (e) MP_CUDA(cudaMemset(dag->err, 0, 4));
+    if (e & mpk::ERR_DOMAIN_BIT)
+        return mph::fail(MP_ERR_DOMAIN, "duration outside {+inf, 0} U [2^-41, 2^20), NaN, or no enabled arch");
+    if (e & mpk::ERR_ARG_BIT) return mph::fail(MP_ERR_ARG, "device-detected argument error");
+    return MP_OK;
+}
+
+void mp_free(mp_dag* dag) {
+    if (!dag) return;
+    cudaDeviceSynchronize();
+    void* ptrs[] = {dag->row_ptr, dag->col,  dag->indeg, dag->level, dag->level_ptr, dag->level_order,
+                    dag->qof,     dag->nodeq, dag->rowq, dag->colq,  dag->lvlq,      dag->nodep,
+                    dag->rowp,    dag->colp, dag->lvlp,  dag->err,   dag->ws,        dag->sort_status,
+                    dag->scan_status, dag->tickets, dag->b_rem, dag->b_f0, dag->b_f1, dag->b_counts,
+                    dag->b_kout, dag->b_pof};
+    for (void* p : ptrs)
+        if (p) cudaFree(p);
+    delete dag;
+}
+
+const char* mp_status_str(mp_status s) {
+    switch (s) {
+        case MP_OK: return "MP_OK";
+        case MP_ERR_ARG: return "MP_ERR_ARG";
+        case MP_ERR_CYCLE: return "MP_ERR_CYCLE";
+        case MP_ERR_DOMAIN: return "MP_ERR_DOMAIN";
+        case MP_ERR_CUDA: return "MP_ERR_CUDA";
+        case MP_ERR_NOMEM: return "MP_ERR_NOMEM";
+    }
+    return "MP_ERR_UNKNOWN";
+}
+
+const char* mp_last_error(void) { return mph::g_last_error.c_str(); }
+
+const char* mp_build_info(void) { return "libmp 0.1 sm_100a (B200) cuda " MP_CUDA_VERSION_STR; }
+
+uint64_t mp_launch_count(void) { return mph::prof().launches.load(); }
+
+void mp_prof_enable(int on) { mph::prof().enabled.store(on ? 1 : 0); }
+
+void mp_prof_reset(void) {
+    auto& p = mph::prof();
+    std::lock_guard<std::mutex> g(p.mu);
+    p.drain();
+    p.totals.clear();
+}
+
+mp_status mp_prof_query(const char* name, double* total_ms, int64_t* launches) {
+    if (!name || !total_ms || !launches) return mph::fail(MP_ERR_ARG, "NULL argument");
+    auto& p = mph::prof();
+    std::lock_guard<std::mutex> g(p.mu);
+    p.drain();
+    auto it = p.totals.find(name);
+    *total_ms = it == p.totals.end() ? 0.0 : it->second.first;
+    *launches = it == p.totals.end() ? 0 : it->second.second;
+    return MP_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,520 @@
+// path.cuh -- a3..a9 for one DAG: bottom-level (+ NOD), gain, score key, queues.
+#pragma once
+#include "build.cuh"
+
+namespace mpk {
+
+constexpr int MAX_ARCH = 8;
+// Largest DAG whose bottom-levels live in one SM's shared memory.
+constexpr int SMALL_CAP = 50 * 1024;
+
+struct DurView {          // read-only duration table + enabled archs
+    const float* dur;     // [n][A]
+    int32_t A;
+    uint32_t emask;
+};
+
+// w(v) = min over enabled a of delta(v,a) (reading c2), with the domain check
+// (reading c20).  Sets `bad` on a domain violation or no enabled arch.
+MP_INLINE float task_weight(const DurView& d, int32_t v, bool& bad) {
+    float w = __uint_as_float(0x7f800000u);
+    bool any = false;
+    for (int a = 0; a < d.A; a++) {
+        float x = canon_dur(__ldg(d.dur + (int64_t)v * d.A + a), bad);
+        if (((d.emask >> a) & 1u) && !is_inf(x)) {
+            any = true;
+            w = x < w ? x : w;
+        }
+    }
+    if (!any) bad = true;
+    return any ? w : 0.0f;
+}
+
+// ---- a4, small DAGs: one CTA, bottom-levels resident in shared memory ------------
+// Levels are walked from the deepest (q-space is reverse level order) with one
+// __syncthreads per level; bl(v) = w(v) + max bl(succ) with a single RN add.
+__global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
+                                                   const int32_t* __restrict__ nodeq,
+                                                   const int32_t* __restrict__ rowq,
+                                                   const int32_t* __restrict__ colq, DurView d, float* bl,
+                                                   float* cp, uint32_t* err) {
+    extern __shared__ float sbl[];
+    bool bad = false;
+    float cpm = 0.0f;
+    for (int32_t r = 0; r < L; r++) {
+        const int32_t q1 = __ldg(lvlq + r + 1);
+        for (int32_t q = __ldg(lvlq + r) + threadIdx.x; q < q1; q += blockDim.x) {
+            const int32_t v = __ldg(nodeq + q);
+            const float w = task_weight(d, v, bad);
+            float m = 0.0f;  // bl >= 0, and w + 0 = w: same as "bl = w without successors"
+            const int32_t e1 = __ldg(rowq + q + 1);
+            for (int32_t e = __ldg(rowq + q); e < e1; e++) m = fmaxf(m, sbl[__ldg(colq + e)]);
+            const float b = __fadd_rn(w, m);
+            sbl[q] = b;
+            bl[v] = b;
+            cpm = fmaxf(cpm, b);
+        }
+        __syncthreads();
+    }
+    cpm = warp_max(cpm);
+    if ((threadIdx.x & 31) == 0) atomicMax((uint32_t*)cp, f2u(cpm));
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(err, ERR_DOMAIN_BIT);
+}
+
+// ---- a4, large DAGs: barrier-free dataflow ------------------------------------------
+// Padded q-space: every level is rounded up to a multiple of 32 positions, so a
+// warp's chunk of 32 positions lies in one level and never depends on itself.
+// Warps take chunks in increasing order from a ticket (deepest level first);
+// a chunk's successors are in strictly deeper levels = earlier chunks, already
+// taken by running warps, so spinning on them cannot deadlock.  The value is its
+// own ready flag (0xFFFFFFFF = not yet; bl is never NaN).  Successor loads are
+// edge-parallel across the warp (coalesced col reads) and max-reduced per node
+// in shared memory.
+constexpr int FLOW_THREADS = 256;
+constexpr uint32_t NOT_READY = 0xFFFFFFFFu;
+
+__global__ void __launch_bounds__(FLOW_THREADS) k_bl_flow(int32_t nchunks, const int32_t* __restrict__ nodep,
+                                                          const int32_t* __restrict__ rowp,
+                                                          const int32_t* __restrict__ colp, DurView d,
+                                                          uint32_t* blp, float* bl, float* cp, uint32_t* ticket,
+                                                          uint32_t* err) {
+    __shared__ uint32_t smax[FLOW_THREADS / 32][32];
+    __shared__ int32_t srow[FLOW_THREADS / 32][33];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    bool bad = false;
+    float cpm = 0.0f;
+    while (true) {
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(ticket, 1u);
+        c = __shfl_sync(0xffffffffu, c, 0);
+        if (c >= (uint32_t)nchunks) break;
+        const int32_t p = (int32_t)c * 32 + lane;
+        const int32_t v = __ldg(nodep + p);
+        const int32_t e0 = __ldg(rowp + p);
+        srow[w][lane] = e0;
+        if (lane == 31) srow[w][32] = __ldg(rowp + p + 1);
+        smax[w][lane] = 0u;
+        const float wt = v >= 0 ? task_weight(d, v, bad) : 0.0f;
+        __syncwarp();
+        const int32_t E0 = srow[w][0], E1 = srow[w][32];
+        for (int32_t e = E0 + lane; e < E1; e += 32) {
+            const int32_t sp = __ldg(colp + e);
+            uint32_t x;
+            do {
+                x = ld_relaxed(blp + sp);
+            } while (x == NOT_READY);
+            // owner: largest i with srow[i] <= e
+            int lo = 0, hi = 31;
+            while (lo < hi) {
+                int mid = (lo + hi + 1) >> 1;
+                if (srow[w][mid] <= e) lo = mid;
+                else hi = mid - 1;
+            }
+            atomicMax(&smax[w][lo], x);
+        }
+        __syncwarp();
+        if (v >= 0) {
+            const float b = __fadd_rn(wt, u2f(smax[w][lane]));
+            st_relaxed(blp + p, f2u(b));
+            bl[v] = b;
+            cpm = fmaxf(cpm, b);
+        }
+        __syncwarp();
+    }
+    cpm = warp_max(cpm);
+    if (lane == 0) atomicMax((uint32_t*)cp, f2u(cpm));
+    if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(err, ERR_DOMAIN_BIT);
+}
+
+// ---- a5: NOD (eq. 2) -----------------------------------------------------------------
+// indeg_a(s) = |{p in lambda^-(s) : p enabled on a}|
+__global__ void k_nod_indeg(int32_t n, const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                            DurView d, int32_t* inda) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t en = 0;
+        for (int a = 0; a < d.A; a++)
+            if (((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + u * d.A + a))) en |= 1u << a;
+        if (!en) continue;
+        for (int32_t e = row_ptr[u]; e < row_ptr[u + 1]; e++) {
+            int32_t s = col[e];
+            for (int a = 0; a < d.A; a++)
+                if ((en >> a) & 1u) atomicAdd(&inda[(int64_t)s * d.A + a], 1);
+        }
+    }
+}
+
+// NOD_a(t) = sum over enabled successors s of floor(2^32 / indeg_a(s)) (exact uint64),
+// converted once (RN) and scaled by 2^-32 (exact); 0 where (t,a) is not enabled.
+__global__ void k_nod_sum(int32_t n, const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                          DurView d, const int32_t* __restrict__ inda, float* nod) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+        for (int a = 0; a < d.A; a++) {
+            float out = 0.0f;
+            if (((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + t * d.A + a))) {
+                uint64_t acc = 0;
+                for (int32_t e = row_ptr[t]; e < row_ptr[t + 1]; e++) {
+                    int32_t s = col[e];
+                    if (((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + (int64_t)s * d.A + a)))
+                        acc += 4294967296ull / (uint64_t)inda[(int64_t)s * d.A + a];
+                }
+                out = __fmul_rn(__ull2float_rn(acc), 0x1p-32f);
+            }
+            nod[t * d.A + a] = out;
+        }
+    }
+}
+
+// ---- a6: gain (eq. 1) ------------------------------------------------------------------
+// pass 1: flags and hd(a) = max |d(t,a)| (non-negative floats ordered as uint32)
+__global__ void k_aff_hd(int32_t n, DurView d, uint8_t* flags, uint32_t* hdbits, uint32_t* err) {
+    bool bad = false;
+    uint32_t hl[MAX_ARCH];
+    for (int a = 0; a < MAX_ARCH; a++) hl[a] = 0;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+        float x[MAX_ARCH];
+        int k = 0;
+        float w = __uint_as_float(0x7f800000u);
+        uint32_t en = 0;
+        for (int a = 0; a < d.A; a++) {
+            x[a] = canon_dur(d.dur[t * d.A + a], bad);
+            if (((d.emask >> a) & 1u) && !is_inf(x[a])) {
+                en |= 1u << a;
+                k++;
+                w = x[a] < w ? x[a] : w;
+            }
+        }
+        if (!k) bad = true;
+        for (int a = 0; a < d.A; a++) {
+            uint8_t f = 0;
+            if ((en >> a) & 1u) {
+                f = 1 | (x[a] == w ? 2 : 0);
+                if (k >= 2) {
+                    float ref = __uint_as_float(0x7f800000u);
+                    for (int b = 0; b < d.A; b++)
+                        if (b != a && ((en >> b) & 1u)) ref = x[b] < ref ? x[b] : ref;
+                    float dd = __fsub_rn(ref, x[a]);
+                    uint32_t ab = f2u(fabsf(dd));
+                    hl[a] = ab > hl[a] ? ab : hl[a];
+                }
+            }
+            flags[t * d.A + a] = f;
+        }
+    }
+    for (int a = 0; a < d.A; a++) {
+        uint32_t v = warp_max(hl[a]);
+        if ((threadIdx.x & 31) == 0 && v) atomicMax(&hdbits[a], v);
+    }
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(err, ERR_DOMAIN_BIT);
+}
+
+// pass 2: gain = 1 (one enabled arch) | 0.5 (hd = 0) | (d + hd) / (hd + hd)
+__global__ void k_aff_gain(int32_t n, DurView d, const uint8_t* flags, const uint32_t* hdbits, float* gain,
+                           float* hd_out) {
+    if (blockIdx.x == 0 && threadIdx.x < d.A) hd_out[threadIdx.x] = u2f(hdbits[threadIdx.x]);
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+        float x[MAX_ARCH];
+        uint32_t en = 0;
+        int k = 0;
+        for (int a = 0; a < d.A; a++) {
+            bool dummy = false;
+            x[a] = canon_dur(d.dur[t * d.A + a], dummy);
+            if (flags[t * d.A + a] & 1) {
+                en |= 1u << a;
+                k++;
+            }
+        }
+        for (int a = 0; a < d.A; a++) {
+            float g = 0.0f;
+            if ((en >> a) & 1u) {
+                float h = u2f(hdbits[a]);
+                if (k == 1) g = 1.0f;
+                else if (h == 0.0f) g = 0.5f;
+                else {
+                    float ref = __uint_as_float(0x7f800000u);
+                    for (int b = 0; b < d.A; b++)
+                        if (b != a && ((en >> b) & 1u)) ref = x[b] < ref ? x[b] : ref;
+                    float dd = __fsub_rn(ref, x[a]);
+                    g = __fdiv_rn(__fadd_rn(dd, h), __fadd_rn(h, h));
+                }
+            }
+            gain[t * d.A + a] = g;
+        }
+    }
+}
+
+// ---- a7: crit_n and key -------------------------------------------------------------------
+__global__ void k_crit_max(int64_t cnt, int32_t A, int32_t kind, const float* crit, const uint8_t* flags,
+                           uint32_t* maxbits) {
+    uint32_t ml[MAX_ARCH];
+    for (int a = 0; a < MAX_ARCH; a++) ml[a] = 0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x) {
+        float c = crit[i];
+        if (kind == 0) {
+            if (c > 0.0f) ml[0] = f2u(c) > ml[0] ? f2u(c) : ml[0];
+        } else {
+            int a = (int)(i % A);
+            if ((flags[i] & 1) && c > 0.0f) {
+                for (int b = 0; b < MAX_ARCH; b++)
+                    if (b == a) ml[b] = f2u(c) > ml[b] ? f2u(c) : ml[b];
+            }
+        }
+    }
+    int na = kind == 0 ? 1 : A;
+    for (int a = 0; a < na; a++) {
+        uint32_t v = warp_max(ml[a]);
+        if ((threadIdx.x & 31) == 0 && v) atomicMax(&maxbits[a], v);
+    }
+}
+
+MP_INLINE uint64_t make_key(float g, float c) {
+    return ((uint64_t)(ONE_BITS - f2u(g)) << 32) | (uint64_t)(ONE_BITS - f2u(c));
+}
+
+__global__ void k_score(int32_t n, int32_t A, int32_t kind, const float* crit, const float* gain,
+                        const uint8_t* flags, const uint32_t* maxbits, float* crit_norm, uint64_t* key) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+        float cn0 = 0.0f;
+        if (kind == 0) {
+            float mx = u2f(maxbits[0]);
+            cn0 = mx > 0.0f ? __fdiv_rn(crit[t], mx) : 0.0f;
+            crit_norm[t] = cn0;
+        }
+        for (int a = 0; a < A; a++) {
+            int64_t i = t * A + a;
+            bool en = flags[i] & 1;
+            float c = cn0;
+            if (kind == 1) {
+                float mx = u2f(maxbits[a]);
+                c = (en && mx > 0.0f) ? __fdiv_rn(crit[i], mx) : 0.0f;
+                crit_norm[i] = c;
+            }
+            key[i] = en ? make_key(gain[i], c) : ~0ull;
+        }
+    }
+}
+
+// ---- a8/a9: queues -------------------------------------------------------------------------
+__global__ void k_copy_len(const int32_t* total, int64_t* len) { *len = *total; }
+
+__global__ void k_blocked(int32_t n, const int32_t* row_ptr, const int32_t* col, const uint8_t* done,
+                          uint8_t* blocked) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
+        if (done[u]) continue;
+        for (int32_t e = row_ptr[u]; e < row_ptr[u + 1]; e++) blocked[col[e]] = 1;
+    }
+}
+
+// membership flags in (arch, id) order + per-arch count and exact brw (blockIdx.y = arch)
+__global__ void k_q_member(int32_t n, int32_t A, const uint8_t* flags, const uint8_t* done,
+                           const uint8_t* blocked, const float* dur, int32_t* memb, int32_t* counts,
+                           unsigned long long* brw) {
+    const int a = blockIdx.y;
+    int32_t cnt = 0;
+    uint64_t lo = 0, hi = 0;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t nround = ((int64_t)n + stride - 1) / stride;
+    for (int64_t it = 0; it < nround; it++) {
+        int64_t t = it * stride + blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+        if (t < n) {
+            uint8_t f = flags[t * A + a];
+            bool m = (f & 1) && (!done || (!done[t] && !blocked[t]));
+            memb[(int64_t)a * n + t] = m ? 1 : 0;
+            if (m) {
+                cnt++;
+                if (f & 2) {
+                    bool dummy = false;
+                    uint64_t l, h;
+                    fixed64(canon_dur(dur[t * A + a], dummy), l, h);
+                    add128(lo, hi, l, h);
+                }
+            }
+        }
+    }
+    warp_sum128(lo, hi);
+    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+    if ((threadIdx.x & 31) == 0) {
+        if (cnt) atomicAdd(&counts[a], cnt);
+        atomic_add128(brw + 2 * a, lo, hi);
+    }
+}
+
+__global__ void k_q_scatter(int32_t n, int32_t A, const uint64_t* key, const int32_t* memb, const int32_t* pos,
+                            uint64_t* skey, uint32_t* sval) {
+    const int a = blockIdx.y;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+        int64_t i = (int64_t)a * n + t;
+        if (!memb[i]) continue;
+        uint64_t k = key[t * A + a];
+        uint64_t gc = k >> 32, cc = k & 0xffffffffull;  // both <= 0x3F800000 < 2^30
+        int32_t p = pos[i];
+        skey[p] = ((uint64_t)a << 60) | (gc << 30) | cc;
+        sval[p] = (uint32_t)t;
+    }
+}
+
+__global__ void k_q_out(const SortPlan* plan, uint32_t* const* vb, const int32_t* total, int32_t A,
+                        const int32_t* counts, const unsigned long long* brw, int64_t* qptr, int32_t* qtask,
+                        mp_queue_summary* sum) {
+    const int32_t Q = *total;
+    const uint32_t* v = Q > 0 ? vb[plan->final_sel] : nullptr;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < Q; i += (int64_t)gridDim.x * blockDim.x)
+        qtask[i] = (int32_t)v[i];
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        int64_t off = 0;
+        for (int a = 0; a < A; a++) {
+            qptr[a] = off;
+            mp_queue_summary s;
+            s.count = counts[a];
+            s.head = counts[a] > 0 ? (int32_t)v[off] : -1;
+            s.brw_lo = brw[2 * a];
+            s.brw_hi = (int64_t)brw[2 * a + 1];
+            s.brw = u128_to_double_scaled(brw[2 * a], brw[2 * a + 1]);
+            sum[a] = s;
+            off += counts[a];
+        }
+        qptr[A] = off;
+    }
+}
+
+}  // namespace mpk
+
+namespace mph {
+
+inline mp_status check_arch(int32_t A, const int32_t* h_workers) {
+    if (A < 1 || A > mpk::MAX_ARCH) return fail(MP_ERR_ARG, "n_arch %d outside [1, 8]", A);
+    if (!h_workers) return fail(MP_ERR_ARG, "h_workers is NULL");
+    return MP_OK;
+}
+
+inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const int32_t* h_workers, float* bl,
+                              float* cp, float* nod, cudaStream_t st) {
+    using namespace mpk;
+    if (!dag) return fail(MP_ERR_ARG, "dag is NULL");
+    MP_TRY(check_arch(A, h_workers));
+    if (!cp || (dag->n > 0 && (!dur || !bl))) return fail(MP_ERR_ARG, "NULL buffer");
+    DurView d{dur, A, enabled_mask(A, h_workers)};
+    MP_CUDA(cudaMemsetAsync(cp, 0, 4, st));
+    const int32_t n = dag->n;
+    if (n == 0) return MP_OK;
+    if (n <= SMALL_CAP) {
+        static int attr = 0;
+        size_t smem = (size_t)n * 4;
+        if (attr < (int)smem) {
+            MP_CUDA(cudaFuncSetAttribute(k_bl_small, cudaFuncAttributeMaxDynamicSharedMemorySize, SMALL_CAP * 4));
+            attr = SMALL_CAP * 4;
+        }
+        MP_LAUNCH(k_bl_small, 1, 1024, smem, st, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp, dag->err);
+    } else {
+        size_t need = align256((size_t)dag->P * 4);
+        MP_TRY(ensure_ws(dag, need, st));
+        uint32_t* blp = (uint32_t*)dag->ws;
+        MP_CUDA(cudaMemsetAsync(blp, 0xff, (size_t)dag->P * 4, st));
+        MP_CUDA(cudaMemsetAsync(dag->tickets + 62, 0, 4, st));
+        int bps = 0;
+        MP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_bl_flow, FLOW_THREADS, 0));
+        int32_t nchunks = dag->P / 32;
+        int64_t g = (int64_t)bps * dag->num_sms;
+        int64_t want = ((int64_t)nchunks + FLOW_THREADS / 32 - 1) / (FLOW_THREADS / 32);
+        if (want < g) g = want;
+        if (g < 1) g = 1;
+        MP_LAUNCH(k_bl_flow, (unsigned)g, FLOW_THREADS, 0, st, nchunks, dag->nodep, dag->rowp, dag->colp, d, blp, bl, cp,
+                                                        dag->tickets + 62, dag->err);
+    }
+    MP_CUDA(cudaGetLastError());
+    if (nod) {
+        size_t need = align256((size_t)n * A * 4);
+        MP_TRY(ensure_ws(dag, need, st));
+        int32_t* inda = (int32_t*)dag->ws;
+        MP_CUDA(cudaMemsetAsync(inda, 0, (size_t)n * A * 4, st));
+        MP_LAUNCH(k_nod_indeg, grid_for(n), 256, 0, st, n, dag->row_ptr, dag->col, d, inda);
+        MP_LAUNCH(k_nod_sum, grid_for(n), 256, 0, st, n, dag->row_ptr, dag->col, d, inda, nod);
+        MP_CUDA(cudaGetLastError());
+    }
+    return MP_OK;
+}
+
+inline mp_status affinity(mp_dag* dag, int32_t A, const float* dur, const int32_t* h_workers, float* gain,
+                          float* hd, uint8_t* flags, cudaStream_t st) {
+    using namespace mpk;
+    if (!dag) return fail(MP_ERR_ARG, "dag is NULL");
+    MP_TRY(check_arch(A, h_workers));
+    if (!hd || (dag->n > 0 && (!dur || !gain || !flags))) return fail(MP_ERR_ARG, "NULL buffer");
+    DurView d{dur, A, enabled_mask(A, h_workers)};
+    MP_TRY(ensure_ws(dag, 256, st));
+    uint32_t* hdbits = (uint32_t*)dag->ws;
+    MP_CUDA(cudaMemsetAsync(hdbits, 0, 4 * MAX_ARCH, st));
+    const int32_t n = dag->n;
+    if (n > 0) MP_LAUNCH(k_aff_hd, grid_for(n), 256, 0, st, n, d, flags, hdbits, dag->err);
+    MP_LAUNCH(k_aff_gain, grid_for(n > 0 ? n : 1), 256, 0, st, n, d, flags, hdbits, gain, hd);
+    MP_CUDA(cudaGetLastError());
+    return MP_OK;
+}
+
+inline mp_status score(mp_dag* dag, int32_t A, int32_t kind, const float* crit, const float* gain,
+                       const uint8_t* flags, float* crit_norm, uint64_t* key, cudaStream_t st) {
+    using namespace mpk;
+    if (!dag) return fail(MP_ERR_ARG, "dag is NULL");
+    if (A < 1 || A > MAX_ARCH) return fail(MP_ERR_ARG, "n_arch %d outside [1, 8]", A);
+    if (kind != 0 && kind != 1) return fail(MP_ERR_ARG, "unknown criticality kind %d", kind);
+    const int32_t n = dag->n;
+    if (n == 0) return MP_OK;
+    if (!crit || !gain || !flags || !crit_norm || !key) return fail(MP_ERR_ARG, "NULL buffer");
+    MP_TRY(ensure_ws(dag, 256, st));
+    uint32_t* mx = (uint32_t*)dag->ws;
+    MP_CUDA(cudaMemsetAsync(mx, 0, 4 * MAX_ARCH, st));
+    int64_t cnt = kind == 0 ? n : (int64_t)n * A;
+    MP_LAUNCH(k_crit_max, grid_for(cnt), 256, 0, st, cnt, A, kind, crit, flags, mx);
+    MP_LAUNCH(k_score, grid_for(n), 256, 0, st, n, A, kind, crit, gain, flags, mx, crit_norm, key);
+    MP_CUDA(cudaGetLastError());
+    return MP_OK;
+}
+
+inline mp_status build_queues(mp_dag* dag, int32_t A, const uint64_t* key, const uint8_t* flags, const float* dur,
+                              const uint8_t* done, int64_t* qptr, int32_t* qtask, mp_queue_summary* sum,
+                              cudaStream_t st) {
+    using namespace mpk;
+    if (!dag) return fail(MP_ERR_ARG, "dag is NULL");
+    if (A < 1 || A > MAX_ARCH) return fail(MP_ERR_ARG, "n_arch %d outside [1, 8]", A);
+    if (!qptr || !sum) return fail(MP_ERR_ARG, "NULL buffer");
+    const int32_t n = dag->n;
+    const int64_t nA = (int64_t)n * A;
+    if (n > 0 && (!key || !flags || !dur || !qtask)) return fail(MP_ERR_ARG, "NULL buffer");
+    const int64_t cap = nA > 0 ? nA : 1;
+    size_t bytes = sort_bytes(cap, 1, 8, true) + 2 * align256(cap * 4) + align256((size_t)n + 1) + 4 * 256;
+    MP_TRY(ensure_ws(dag, bytes, st));
+    Arena ar{dag->ws, dag->ws_cap};
+    SortArgs sa = carve_sort(ar, dag, cap, 1, 0, 8, true);
+    int32_t* memb = ar.take<int32_t>(cap);
+    int32_t* pos = ar.take<int32_t>(cap);
+    uint8_t* blocked = ar.take<uint8_t>((size_t)n + 1);
+    int32_t* counts = ar.take<int32_t>(MAX_ARCH);
+    unsigned long long* brw = ar.take<unsigned long long>(2 * MAX_ARCH);
+    int32_t* total = ar.take<int32_t>(2);
+    uint32_t** vb = ar.take<uint32_t*>(2);
+    int64_t* dlen = ar.take<int64_t>(1);
+    MP_CUDA(cudaMemsetAsync(counts, 0, 4 * MAX_ARCH, st));
+    MP_CUDA(cudaMemsetAsync(brw, 0, 16 * MAX_ARCH, st));
+    MP_CUDA(cudaMemsetAsync(total, 0, 8, st));
+    uint32_t* hv[2] = {sa.vals[0], sa.vals[1]};
+    MP_CUDA(cudaMemcpyAsync(vb, hv, sizeof(hv), cudaMemcpyHostToDevice, st));
+    if (n > 0) {
+        if (done) {
+            MP_CUDA(cudaMemsetAsync(blocked, 0, (size_t)n, st));
+            MP_LAUNCH(k_blocked, grid_for(n), 256, 0, st, n, dag->row_ptr, dag->col, done, blocked);
+        }
+        dim3 g(grid_for(n, 256, 148 * 8), A);
+        MP_LAUNCH(k_q_member, g, 256, 0, st, n, A, flags, done, blocked, dur, memb, counts, brw);
+        MP_TRY(scan(dag, memb, pos, nA, total, st));
+        MP_LAUNCH(k_q_scatter, g, 256, 0, st, n, A, key, memb, pos, sa.keys[0], sa.vals[0]);
+        // device-side length: the sort reads Q from `total` (int32) via an int64 mirror
+        sa.seg_len = nA;
+        sa.d_len = dlen;
+        MP_LAUNCH(k_copy_len, 1, 1, 0, st, total, dlen);
+        MP_TRY(run_sort(dag, sa, st));
+    }
+    MP_LAUNCH(k_q_out, grid_for(nA > 0 ? nA : 1), 256, 0, st, sa.plans, vb, total, A, counts, brw, qptr, qtask, sum);
+    MP_CUDA(cudaGetLastError());
+    return MP_OK;
+}
+
+}  // namespace mph

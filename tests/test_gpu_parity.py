@@ -1,0 +1,259 @@
+"""GPU parity: libmp (sm_100a, through the C-ABI) vs the CPU oracle, bit-exact.
+
+Every float output is compared on its bit pattern; integer / index outputs are
+compared exactly; queue orders are unique (ties broken by id) so they must be
+identical.  Inputs are the seeded workloads of DESIGN.md §3.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workloads
+from workloads import random_dags
+
+pytestmark = pytest.mark.gpu
+
+mp = pytest.importorskip("paper_conf_ipps_tayebbfg24_b200")
+
+DEV = "cuda"
+
+
+def to_dev(a, dtype=None):
+    t = torch.from_numpy(np.ascontiguousarray(a))
+    if dtype is not None:
+        t = t.to(dtype)
+    return t.to(DEV)
+
+
+def bits(a):
+    return np.ascontiguousarray(a, dtype=np.float32).view(np.uint32)
+
+
+def gpu_path(n, src, dst, dur, workers, kind=0, done=None):
+    dag = mp.build_dag(n, to_dev(src, torch.int32), to_dev(dst, torch.int32))
+    r = mp.score_and_queue(dag, to_dev(dur), workers, kind, None if done is None else to_dev(done))
+    mp.check(dag)
+    out = {k: (v.cpu().numpy() if isinstance(v, torch.Tensor) else v) for k, v in r.items()}
+    out["arrays"] = {k: v.cpu().numpy() for k, v in dag.arrays().items()}
+    out["dag"] = dag
+    return out
+
+
+def compare(n, src, dst, dur, workers, kind=0, done=None):
+    g = gpu_path(n, src, dst, dur, workers, kind, done)
+    od = oracle.build_dag(n, src, dst)
+    ga = g["arrays"]
+    assert g["dag"].n_edges == od.n_edges and g["dag"].n_levels == od.n_levels
+    assert np.array_equal(ga["row_ptr"], od.row_ptr)
+    assert np.array_equal(ga["col"], od.col)
+    assert np.array_equal(ga["indeg"], od.indeg)
+    assert np.array_equal(ga["level"], od.level)
+    assert np.array_equal(ga["level_ptr"], od.level_ptr)
+    assert np.array_equal(ga["level_order"], od.level_order)
+    if n == 0:
+        return g
+    o = oracle.score_and_queue(od, dur, workers, kind, done)
+    assert np.array_equal(bits(g["bl"]), bits(o["bl"])), "bottom-level"
+    assert bits(g["cp"])[0] == bits(np.float32(o["cp"]))
+    assert np.array_equal(g["flags"], o["flags"])
+    assert np.array_equal(bits(g["hd"]), bits(o["hd"]))
+    assert np.array_equal(bits(g["gain"]), bits(o["gain"])), "gain"
+    if kind == oracle.CRIT_NOD:
+        assert np.array_equal(bits(g["nod"]), bits(o["crit"])), "NOD"
+    assert np.array_equal(bits(g["crit_norm"]), bits(o["crit_norm"])), "crit_norm"
+    assert np.array_equal(g["key"].view(np.uint64), o["key"]), "key"
+    assert np.array_equal(g["qptr"], o["qptr"])
+    Q = int(o["qptr"][-1])
+    assert np.array_equal(g["qtask"][:Q], o["qtask"]), "queue order"
+    gs = g["summary"].view(mp.SUMMARY_DTYPE)
+    assert gs.tobytes() == o["summary"].tobytes(), (gs, o["summary"])
+    return g
+
+
+@pytest.mark.parametrize("name", ["c1", "c2", "c3"])
+def test_configs_bit_exact(name):
+    w = workloads.config(name)
+    compare(w.n, w.src, w.dst, w.dur, w.workers)
+
+
+def test_c4_bit_exact():
+    w = workloads.config("c4")
+    compare(w.n, w.src, w.dst, w.dur, w.workers)
+
+
+@pytest.mark.parametrize("name", ["c1", "c2"])
+def test_nod_bit_exact(name):
+    w = workloads.config(name)
+    compare(w.n, w.src, w.dst, w.dur, w.workers, kind=oracle.CRIT_NOD)
+
+
+def test_nod_three_arch_masks():
+    w = workloads.qr(24)
+    compare(w.n, w.src, w.dst, w.dur, w.workers, kind=oracle.CRIT_NOD)
+
+
+@pytest.mark.parametrize("seed,n,deg,A,p_inf,tiny", [
+    (0, 1, 0.0, 2, 0.0, False),
+    (1, 2, 1.0, 1, 0.0, False),
+    (2, 777, 2.5, 2, 0.2, False),
+    (3, 5000, 3.0, 3, 0.3, True),
+    (4, 40000, 4.0, 2, 0.1, True),
+    (5, 60000, 2.0, 2, 0.0, False),      # > SMALL_CAP: dataflow kernel
+    (6, 250000, 3.0, 3, 0.25, True),     # dataflow, 3 archs, ties
+])
+def test_random_dags(seed, n, deg, A, p_inf, tiny):
+    src, dst = random_dags.random_dag(n, deg, seed, dup=0.3, max_span=64)
+    dur = random_dags.dyadic_durations(n, A, seed, p_inf=p_inf, tiny_set=tiny)
+    compare(n, src, dst, dur, np.ones(A, np.int32))
+
+
+def test_deep_chain_and_wide_star():
+    n = 6000
+    s, d = random_dags.chain(n)
+    compare(n, s, d, random_dags.dyadic_durations(n, 2, 1), np.ones(2, np.int32))
+    n = 70000
+    s, d = random_dags.chain(n)             # deep chain through the dataflow kernel
+    compare(n, s, d, random_dags.dyadic_durations(n, 2, 2), np.ones(2, np.int32))
+    n = 100000
+    s, d = random_dags.star(n)              # one node with 99,999 successors
+    compare(n, s, d, random_dags.dyadic_durations(n, 2, 3), np.ones(2, np.int32))
+    s2, d2 = d.copy(), s.copy()             # fan-in of 99,999
+    compare(n, s2, d2, random_dags.dyadic_durations(n, 2, 4), np.ones(2, np.int32))
+
+
+def test_layered_skewed_fanin():
+    n, s, d = random_dags.layered_dag([3000, 50, 20000, 7, 40000, 1], fan=40, seed=9)
+    compare(n, s, d, random_dags.dyadic_durations(n, 2, 9, tiny_set=True), np.ones(2, np.int32))
+
+
+def test_empty_and_edgeless():
+    compare(0, np.zeros(0, np.int32), np.zeros(0, np.int32), np.zeros((0, 2), np.float32), np.ones(2, np.int32))
+    n = 5000
+    compare(n, np.zeros(0, np.int32), np.zeros(0, np.int32), random_dags.dyadic_durations(n, 2, 5),
+            np.ones(2, np.int32))
+
+
+def test_workers_disable_and_zero_durations():
+    w = workloads.config("c2")
+    dur = w.dur.copy()
+    dur[::7, 0] = 0.0
+    dur[::11, 1] = -0.0
+    compare(w.n, w.src, w.dst, dur, np.array([3, 1], np.int32))
+    compare(w.n, w.src, w.dst, dur, np.array([0, 2], np.int32))
+
+
+def test_ready_mode():
+    w = workloads.config("c2")
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    rng = np.random.default_rng(1)
+    done = np.zeros(w.n, np.uint8)
+    done[od.level_order[: w.n // 4]] = 1
+    done[rng.integers(0, w.n, 100)] = 1
+    compare(w.n, w.src, w.dst, w.dur, w.workers, done=done)
+
+
+def test_domain_and_graph_errors():
+    n = 4
+    ok_dur = np.ones((n, 2), np.float32)
+    with pytest.raises(mp.MPError) as e:
+        mp.build_dag(n, to_dev(np.array([0, 1, 2], np.int32)), to_dev(np.array([1, 2, 0], np.int32)))
+    assert e.value.code == mp.MP_ERR_CYCLE
+    with pytest.raises(mp.MPError) as e:
+        mp.build_dag(n, to_dev(np.array([0], np.int32)), to_dev(np.array([0], np.int32)))
+    assert e.value.code == mp.MP_ERR_ARG
+    with pytest.raises(mp.MPError) as e:
+        mp.build_dag(n, to_dev(np.array([0], np.int32)), to_dev(np.array([4], np.int32)))
+    assert e.value.code == mp.MP_ERR_ARG
+    dag = mp.build_dag(n, to_dev(np.array([0, 1], np.int32)), to_dev(np.array([1, 2], np.int32)))
+    for bad in (np.nan, -1.0, 2.0 ** -42, 2.0 ** 20, -np.inf):
+        d = ok_dur.copy()
+        d[2, 1] = bad
+        mp.bottom_level(dag, to_dev(d), [1, 1])
+        with pytest.raises(mp.MPError) as e:
+            mp.check(dag)
+        assert e.value.code == mp.MP_ERR_DOMAIN
+    d = ok_dur.copy()
+    d[1] = np.inf
+    mp.affinity(dag, to_dev(d), [1, 1])
+    with pytest.raises(mp.MPError):
+        mp.check(dag)
+    mp.check(dag)  # flag cleared
+    with pytest.raises(ValueError):
+        mp.bottom_level(dag, to_dev(ok_dur), [1, 1, 1])
+    with pytest.raises(TypeError):                      # no CPU path
+        mp.bottom_level(dag, torch.from_numpy(ok_dur), [1, 1])
+
+
+def test_deterministic_repeat():
+    w = workloads.config("c3")
+    a = gpu_path(w.n, w.src, w.dst, w.dur, w.workers)
+    b = gpu_path(w.n, w.src, w.dst, w.dur, w.workers)
+    for k in ("bl", "gain", "key", "qtask", "summary"):
+        assert np.array_equal(a[k], b[k])
+
+
+# ----------------------------------------------------------------------------
+# a10 replicas
+# ----------------------------------------------------------------------------
+
+def _replica_check(w, R, r0, sample, sigma=workloads.C5_SIGMA, seed=workloads.C5_SEED):
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    base = to_dev(w.dur)
+    cp, summ, q = mp.replicas_run(dag, base, w.workers, seed, sigma, r0, R, want_queues=True)
+    mp.check(dag)
+    cp = cp.cpu().numpy()
+    gs = mp.summaries(summ).reshape(R, w.n_arch)
+    q = q.cpu().numpy()
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    for i in sample:
+        ocp, osum, oq, oqptr = oracle.replica(od, w.dur, w.workers, seed, sigma, r0 + i)
+        assert bits(cp[i:i + 1])[0] == bits(np.float32(ocp)), i
+        assert gs[i].tobytes() == osum.tobytes(), (i, gs[i], osum)
+        assert np.array_equal(q[i, :len(oq)], oq), i
+    return cp, gs, q
+
+
+def test_replicas_c1_all():
+    w = workloads.config("c1")
+    _replica_check(w, 300, 0, range(300))
+
+
+def test_replicas_c5_sampled_full_size():
+    w = workloads.config("c5")
+    R = workloads.C5_REPLICAS
+    rng = np.random.default_rng(0)
+    sample = sorted(set([0, 1, R - 1] + rng.integers(0, R, 40).tolist()))
+    cp, gs, q = _replica_check(w, R, 0, sample)
+    # world-size invariance: two half-range calls give identical bytes
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    base = to_dev(w.dur)
+    h = R // 2
+    cp2, s2, q2 = mp.replicas_run(dag, base, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, h, R - h)
+    mp.check(dag)
+    assert np.array_equal(bits(cp2.cpu().numpy()), bits(cp[h:]))
+    assert mp.summaries(s2).tobytes() == gs[h:].tobytes()
+    assert np.array_equal(q2.cpu().numpy(), q[h:])
+
+
+def test_replicas_sigma_zero_equals_single_dag():
+    w = workloads.config("c2")
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    cp, summ, q = mp.replicas_run(dag, to_dev(w.dur), w.workers, 7, 0.0, 0, 3)
+    one = mp.score_and_queue(dag, to_dev(w.dur), w.workers)
+    mp.check(dag)
+    for i in range(3):
+        assert bits(cp.cpu().numpy())[i] == bits(one["cp"].cpu().numpy())[0]
+        assert np.array_equal(q.cpu().numpy()[i], one["qtask"].cpu().numpy())
+        assert mp.summaries(summ)[i * 2:(i + 1) * 2].tobytes() == one["summary"].cpu().numpy().tobytes()
+
+
+def test_replicas_large_dag_path():
+    w = workloads.qr(40)                       # n = 22,140 < cap, force the large path with a bigger DAG
+    src, dst = random_dags.random_dag(60000, 2.0, 3, max_span=64)
+    dur = random_dags.dyadic_durations(60000, 2, 3)
+    W = workloads.Workload("r", 60000, src, dst, dur, ("CPU", "GPU"), np.ones(2, np.int32))
+    _replica_check(W, 3, 11, range(3))
+    _replica_check(w, 5, 100, range(5))
