@@ -313,7 +313,7 @@ def run_ours(args):
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
     ms_per_step = float(tot.item()) / args.steps
     value = tasks_per_step / (ms_per_step * 1e-3)
-    prof = {k: mp.prof_query(k) for k in KERNELS}
+    prof = {k: mp.prof_query(k) for k in mp.prof_names()}
     step_dev_ms = {k: v[0] / args.steps for k, v in prof.items() if v[1] > 0}
     dom = max(step_dev_ms, key=step_dev_ms.get)
     dom_ms, dom_launches = prof[dom]

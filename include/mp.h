@@ -208,6 +208,9 @@ uint64_t mp_launch_count(void);
 void mp_prof_enable(int on);
 void mp_prof_reset(void);
 mp_status mp_prof_query(const char* name, double* total_ms, int64_t* launches);
+/* Comma-separated names of every kernel timed since the last mp_prof_reset;
+ * returns the length needed (excluding the NUL); writes at most len bytes. */
+int64_t mp_prof_names(char* buf, int64_t len);
 
 #ifdef __cplusplus
 }

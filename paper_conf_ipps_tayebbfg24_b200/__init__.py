@@ -260,3 +260,11 @@ def prof_query(name: str):
     cnt = C.c_int64()
     _lib.check(_lib.lib().mp_prof_query(name.encode(), C.byref(ms), C.byref(cnt)), "mp_prof_query")
     return ms.value, cnt.value
+
+
+def prof_names() -> list:
+    """Kernels timed since prof_reset (mp_prof_names)."""
+    need = int(_lib.lib().mp_prof_names(None, 0))
+    buf = C.create_string_buffer(need + 1)
+    _lib.lib().mp_prof_names(buf, need + 1)
+    return [x for x in buf.value.decode().split(",") if x]

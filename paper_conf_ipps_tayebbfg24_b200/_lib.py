@@ -17,7 +17,7 @@ MP_CRIT_BOTTOM_LEVEL, MP_CRIT_NOD = 0, 1
 EXPORTS = (
     "mp_build_dag", "mp_dag_rebuild", "mp_dag_get_info", "mp_bottom_level", "mp_affinity", "mp_score",
     "mp_build_queues", "mp_replicas_run", "mp_check", "mp_free", "mp_status_str",
-    "mp_last_error", "mp_build_info", "mp_launch_count", "mp_prof_enable", "mp_prof_reset", "mp_prof_query",
+    "mp_last_error", "mp_build_info", "mp_launch_count", "mp_prof_enable", "mp_prof_reset", "mp_prof_query", "mp_prof_names",
 )
 
 
@@ -68,9 +68,11 @@ def lib():
     L.mp_prof_enable.restype = None
     L.mp_prof_reset.restype = None
     L.mp_prof_query.argtypes = [C.c_char_p, C.POINTER(C.c_double), C.POINTER(C.c_int64)]
+    L.mp_prof_names.argtypes = [C.c_char_p, C.c_int64]
+    L.mp_prof_names.restype = C.c_int64
     for name in EXPORTS:
         if name not in ("mp_free", "mp_status_str", "mp_last_error", "mp_build_info", "mp_dag_get_info",
-                        "mp_launch_count", "mp_prof_enable", "mp_prof_reset"):
+                        "mp_launch_count", "mp_prof_enable", "mp_prof_reset", "mp_prof_names"):
             getattr(L, name).restype = C.c_int
     L.mp_dag_get_info.restype = C.c_int
     _lib = L

@@ -66,25 +66,49 @@ struct KahnArgs {
     uint32_t* err;
 };
 
-// Kahn level-synchronous frontier expansion in one cooperative kernel with a
-// grid barrier per level; appends use warp-aggregated atomics.
-__global__ void k_kahn(KahnArgs a) {
-    cg::grid_group grid = cg::this_grid();
+// Light grid barrier for a co-resident (cooperative) grid: one monotonically
+// increasing arrival counter, thread 0 of each block spins with acquire loads.
+MP_INLINE void grid_barrier(unsigned* bar, unsigned& epoch) {
+    __syncthreads();
+    epoch++;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(bar, 1u);
+        const unsigned target = epoch * gridDim.x;
+        unsigned v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+        } while ((int)(v - target) < 0);
+    }
+    __syncthreads();
+}
+
+MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int32_t v) {
+    cg::coalesced_group g = cg::coalesced_threads();
+    int32_t base = 0;
+    if (g.thread_rank() == 0) base = atomicAdd(counter, (int32_t)g.size());
+    base = g.shfl(base, 0);
+    list[base + g.thread_rank()] = v;
+}
+
+// Kahn, level-synchronous (a task is ready when all its predecessors are done,
+// P:l.91): level k+1 = successors whose last remaining predecessor is in level
+// k.  Cooperative grid (one block per SM) with a light grid barrier per level;
+// frontier appends use warp-aggregated atomics.  With one block the barrier is
+// a __syncthreads and the remaining-predecessor counters live in shared memory.
+__global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int smem_rem) {
+    extern __shared__ int32_t srem[];
     const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+    int32_t* rem = smem_rem ? srem : a.rem;
+    unsigned epoch = 0;
     for (int64_t v = gtid; v < a.n; v += gsz) {
         int32_t d = a.indeg[v];
-        a.rem[v] = d;
+        rem[v] = d;
         a.level[v] = 0;
-        if (d == 0) {
-            cg::coalesced_group g = cg::coalesced_threads();
-            int32_t base = 0;
-            if (g.thread_rank() == 0) base = atomicAdd(&a.counts[0], (int32_t)g.size());
-            base = g.shfl(base, 0);
-            a.front[0][base + g.thread_rank()] = (int32_t)v;
-        }
+        if (d == 0) kahn_append(&a.counts[0], a.front[0], (int32_t)v);
     }
-    grid.sync();
+    if (gridDim.x == 1) __syncthreads(); else grid_barrier(bar, epoch);
     int32_t k = 0;
     int64_t processed = 0;
     while (true) {
@@ -94,21 +118,18 @@ __global__ void k_kahn(KahnArgs a) {
         const int32_t* cur = a.front[k & 1];
         int32_t* nxt = a.front[(k + 1) & 1];
         for (int64_t i = gtid; i < cnt; i += gsz) {
-            int32_t u = cur[i];
-            for (int32_t e = a.row_ptr[u]; e < a.row_ptr[u + 1]; e++) {
-                int32_t v = a.col[e];
-                if (atomicSub(&a.rem[v], 1) == 1) {
+            const int32_t u = cur[i];
+            const int32_t e1 = a.row_ptr[u + 1];
+            for (int32_t e = a.row_ptr[u]; e < e1; e++) {
+                const int32_t v = a.col[e];
+                if (atomicSub(&rem[v], 1) == 1) {
                     a.level[v] = k + 1;
-                    cg::coalesced_group g = cg::coalesced_threads();
-                    int32_t base = 0;
-                    if (g.thread_rank() == 0) base = atomicAdd(&a.counts[k + 1], (int32_t)g.size());
-                    base = g.shfl(base, 0);
-                    nxt[base + g.thread_rank()] = v;
+                    kahn_append(&a.counts[k + 1], nxt, v);
                 }
             }
         }
         k++;
-        grid.sync();
+        if (gridDim.x == 1) __syncthreads(); else grid_barrier(bar, epoch);
     }
     if (gtid == 0) {
         a.out[0] = k;
@@ -291,15 +312,26 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     CK(cudaMemsetAsync(kout, 0, 16, st));
     if (n > 0) {
         KahnArgs ka{n, dag->row_ptr, dag->col, dag->indeg, rem, dag->level, {f0, f1}, counts, kout, dag->err};
-        int bps = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_kahn, 256, 0));
-        int64_t want = (n + 255) / 256;
-        int64_t g = (int64_t)bps * dag->num_sms;
-        if (want < g) g = want;
-        if (g < 1) g = 1;
-        void* args[] = {&ka};
+        unsigned* bar = (unsigned*)(dag->tickets + 60);
+        CK(cudaMemsetAsync(bar, 0, 4, st));
+        // small DAGs: one CTA, remaining-predecessor counters in shared memory
+        const int64_t kSmemRem = 48 * 1024;
+        int smem_rem = (int64_t)n <= kSmemRem ? 1 : 0;
+        int g = 1;
+        if (!smem_rem) {
+            int bps = 0;
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_kahn, 1024, 0));
+            g = std::max(1, std::min(bps, 1) * dag->num_sms);
+        }
+        size_t smem = smem_rem ? (size_t)n * 4 : 0;
+        static bool attr = false;
+        if (!attr) {
+            CK(cudaFuncSetAttribute(k_kahn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSmemRem * 4)));
+            attr = true;
+        }
+        void* args[] = {&ka, &bar, &smem_rem};
         mph::ProfScope kahn_scope("k_kahn", st);
-        CK(cudaLaunchCooperativeKernel((void*)k_kahn, dim3((unsigned)g), dim3(256), args, 0, st));
+        CK(cudaLaunchCooperativeKernel((void*)k_kahn, dim3((unsigned)g), dim3(1024), args, smem, st));
     }
     int32_t h_scal[2] = {0, 0};
     int32_t h_k[2] = {0, 0};

@@ -4,7 +4,7 @@
 #include <cstdarg>
 #include <vector>
 
-#include "replicas.cuh"
+#include "rep2.cuh"
 
 static inline cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
 
@@ -127,6 +127,23 @@ mp_status mp_prof_query(const char* name, double* total_ms, int64_t* launches) {
     *total_ms = it == p.totals.end() ? 0.0 : it->second.first;
     *launches = it == p.totals.end() ? 0 : it->second.second;
     return MP_OK;
+}
+
+int64_t mp_prof_names(char* buf, int64_t len) {
+    auto& p = mph::prof();
+    std::lock_guard<std::mutex> g(p.mu);
+    p.drain();
+    std::string all;
+    for (auto& kv : p.totals) {
+        if (!all.empty()) all += ",";
+        all += kv.first;
+    }
+    if (buf && len > 0) {
+        int64_t m = std::min<int64_t>(len - 1, (int64_t)all.size());
+        memcpy(buf, all.data(), (size_t)m);
+        buf[m] = 0;
+    }
+    return (int64_t)all.size();
 }
 
 }  // extern "C"

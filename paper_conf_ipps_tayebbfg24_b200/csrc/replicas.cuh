@@ -219,6 +219,16 @@ __global__ void k_perturb(int32_t n, int32_t A, const float* base, uint64_t seed
 
 namespace mph {
 
+inline bool rep2_eligible(const mp_dag* dag, int32_t A);
+inline mp_status replicas_run2(mp_dag* dag, int32_t A, const float* base, uint32_t emask, uint64_t seed, float sigma,
+                               int64_t r0, int32_t R, float* cp, mp_queue_summary* sum, int32_t* qtask,
+                               cudaStream_t st);
+// MP_REPLICA_PATH=v1 forces the generic batched path (used by tests to cross-check the two)
+inline bool rep2_path_enabled() {
+    const char* e = getenv("MP_REPLICA_PATH");
+    return !(e && e[0] == 'v' && e[1] == '1');
+}
+
 inline mp_status replicas_run(mp_dag* dag, int32_t A, const float* base, const int32_t* h_workers, uint64_t seed,
                               float sigma, int64_t r0, int32_t R, float* cp, mp_queue_summary* sum,
                               int32_t* qtask, cudaStream_t st) {
@@ -239,6 +249,8 @@ inline mp_status replicas_run(mp_dag* dag, int32_t A, const float* base, const i
         MP_CUDA(cudaStreamSynchronize(st));
         return MP_OK;
     }
+    if (rep2_path_enabled() && rep2_eligible(dag, A))
+        return replicas_run2(dag, A, base, emask, seed, sigma, r0, R, cp, sum, qtask, st);
     if (n <= SMALL_CAP) {
         const int64_t per = (int64_t)A * n;
         int32_t RB = (int32_t)std::min<int64_t>(R, std::max<int64_t>(1, (int64_t)(256ll << 20) / (per * 24)));

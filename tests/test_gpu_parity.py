@@ -257,3 +257,23 @@ def test_replicas_large_dag_path():
     W = workloads.Workload("r", 60000, src, dst, dur, ("CPU", "GPU"), np.ones(2, np.int32))
     _replica_check(W, 3, 11, range(3))
     _replica_check(w, 5, 100, range(5))
+
+
+def test_replicas_three_arch_masks_all():
+    w = workloads.qr(10)              # A = 3, ACC column has +inf entries
+    _replica_check(w, 70, 5, range(70))
+
+
+def test_replicas_one_arch_and_disabled_arch():
+    w = workloads.config("c2")
+    one = workloads.Workload("c2a1", w.n, w.src, w.dst, np.ascontiguousarray(w.dur[:, :1]), ("CPU",),
+                             np.ones(1, np.int32))
+    _replica_check(one, 33, 0, [0, 17, 32])
+    dis = workloads.Workload("c2dis", w.n, w.src, w.dst, w.dur, w.arch_names, np.array([1, 0], np.int32))
+    _replica_check(dis, 33, 64, [0, 31, 32])
+
+
+def test_replicas_ties_stream_path():
+    """sigma = 0 on c2: 41,664 GEMMs share one gain -> key ranges with one value > 16384 entries."""
+    w = workloads.config("c2")
+    _replica_check(w, 40, 0, [0, 39], sigma=0.0)
