@@ -235,21 +235,47 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
 
 
 // ---------------------------------------------------------------------------------------
-// K2: per-replica bucketed sorts in shared memory
+// K2: per-replica sorts in shared memory
+//
+// Queue a of replica r = entries t sorted by the composite key
+//     key_a(t) = (gainc_a(t) << 32) | critc(t),   ties by t,
+// gainc = 0x3F800000 - bits(gain) (0x40000000 = not enabled: after every real
+// key), critc = 0x3F800000 - bits(bl/CP) -- i.e. (gain desc, crit desc, id asc).
+// (key, t) is unique, so no step needs to be stable except where noted.
+//
+// Sorter: a key range [lo, hi] is histogrammed into <= 16384 equal-width bins
+// (one read of gainc; critc only where the bin depends on it).  Consecutive
+// bins are packed into rounds of <= R3_CAP entries; a round re-reads the keys,
+// places each member at (bin start + atomic cursor) in shared memory and then
+// orders every bin: insertion sort (<= 32 entries) or a block-wide rank sort
+// (<= 1024).  Bins with more entries become finer ranges (deferred), or, when
+// a bin holds a single key value, are streamed in id order (stable).
 // ---------------------------------------------------------------------------------------
-struct R2Smem {
-    uint32_t* k[2];     // [R2_CAP] keys (relative to the round's low key)
-    uint16_t* v[2];     // [R2_CAP] payloads
-    uint32_t* hw;       // [8192]  range histogram / per-warp digit counts
-    uint32_t* scan;     // [64]    block-scan scratch
-    uint32_t* misc;     // [512]   groups (4 x u32 each), stack, broadcast values
+constexpr int R3_NC = 4096;      // coarse bins per range
+constexpr int R3_NF = 12288;     // fine bins per range (sub-bins of the coarse bins)
+constexpr int R3_CAP = 16000;    // entries per round (shared memory)
+constexpr int R3_TINY = 64;      // fine bins up to this size: thread insertion sort
+constexpr int R3_MID = 256;      // up to this size: warp rank sort; larger: finer range / stream
+constexpr int R3_MAXS = 192;     // range stack entries (6 words each)
+constexpr int R3_MAXG = 192;     // group records per range (3 words each)
+
+struct R3Smem {
+    uint32_t* starts;   // [R3_NF + 64]  fine counts -> exclusive prefixes
+    uint16_t* coff;     // [R3_NC + 64]  first fine bin of each coarse bin
+    uint8_t* clog;      // [R3_NC + 64]  log2(#fine bins) of each coarse bin
+    uint64_t* bk;       // [R3_CAP]
+    uint16_t* bv;       // [R3_CAP]
+    uint32_t* sc;       // [96]
+    uint32_t* misc;     // [R3_MAXS*6 + R3_MAXG*3 + 8 + 512]
 };
 
-constexpr int R2_MAXG = 40;     // groups per range
-constexpr int R2_MAXS = 16;     // deferred-range stack
+constexpr size_t r3_smem_bytes() {
+    return (size_t)(R3_NF + 64) * 4 + (size_t)(R3_NC + 64) * 2 + (size_t)(R3_NC + 64) + (size_t)R3_CAP * 8 +
+           (size_t)R3_CAP * 2 + 96 * 4 + (size_t)(R3_MAXS * 6 + R3_MAXG * 3 + 8 + 512) * 4;
+}
 
-// exclusive block scan of one value per thread (1024 threads); returns the prefix, total via ref
-MP_INLINE uint32_t r2_scan(uint32_t x, uint32_t* sc, uint32_t& total) {
+// exclusive block scan of one value per thread (1024 threads)
+MP_INLINE uint32_t r3_scan(uint32_t x, uint32_t* sc, uint32_t& total) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     uint32_t incl = x;
 #pragma unroll
@@ -277,275 +303,336 @@ MP_INLINE uint32_t r2_scan(uint32_t x, uint32_t* sc, uint32_t& total) {
     return r;
 }
 
-MP_INLINE uint32_t r2_bitlen(uint32_t x) { return x ? 32u - __clz(x) : 0u; }
+struct R3Keys {
+    const uint32_t* hi;   // gainc_a[n]
+    const uint32_t* lo;   // critc[n]
+    MP_INLINE uint64_t full(int32_t t) const { return ((uint64_t)__ldcg(hi + t) << 32) | __ldcg(lo + t); }
+};
 
-// stable LSD pass in shared memory: (ks,vs) -> (kd,vd) by digit (k >> sh) & 255
-MP_INLINE void r2_lsd_pass(const uint32_t* ks, const uint16_t* vs, uint32_t* kd, uint16_t* vd, uint32_t cnt, int sh,
-                           uint32_t* hw, uint32_t* sc) {
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    uint32_t* wh = hw + w * 256;
-    for (int d = lane; d < 256; d += 32) wh[d] = 0;
-    const uint32_t per = (cnt + R2_WARPS - 1) / R2_WARPS;
-    const uint32_t ws = min(cnt, w * per), we = min(cnt, ws + per);
-    __syncwarp();
-    const uint32_t lt = lanemask_lt();
-    for (uint32_t b = ws; b < we; b += 32) {
-        const uint32_t i = b + lane;
-        const uint32_t d = i < we ? (ks[i] >> sh) & 255u : 256u;
-        const uint32_t peers = __match_any_sync(0xffffffffu, d);
-        if (d < 256 && (peers & lt) == 0) atomicAdd(&wh[d], (uint32_t)__popc(peers));
+struct R3Out {
+    int32_t* q;       // queue destination or null
+    int32_t count;    // enabled entries (positions >= count are not written)
+    uint32_t* head;   // shared
+    MP_INLINE void put(int32_t pos, uint32_t t) const {
+        if (pos == 0) *head = t;
+        if (q && pos < count) q[pos] = (int32_t)t;
+    }
+};
+
+// Range geometry: coarse bin of key k = (k >> cs) - clb (< ncb); fine bin =
+// coff[c] + ((k >> (cs - clog[c])) & ((1 << clog[c]) - 1)).
+struct R3Geo {
+    uint64_t lo, hi, clb;
+    uint32_t cs, ncb;
+};
+
+// Is t inside [lo, hi]?  Returns its coarse bin and (if want_key) its full key; reads
+// critc only when the bin or the bounds depend on it (need_bits = lowest key bit used).
+MP_INLINE bool r3_locate(const R3Keys& K, int32_t t, const R3Geo& g, uint32_t need_bits, uint32_t& cb,
+                         uint64_t& key) {
+    const uint32_t h = __ldcg(K.hi + t);
+    const uint32_t lh = (uint32_t)(g.lo >> 32), hh = (uint32_t)(g.hi >> 32);
+    if (h < lh || h > hh) return false;
+    if (need_bits >= 32 && h != lh && h != hh) {
+        key = (uint64_t)h << 32;
+        cb = (uint32_t)((key >> g.cs) - g.clb);
+        return true;
+    }
+    key = ((uint64_t)h << 32) | __ldcg(K.lo + t);
+    if (key < g.lo || key > g.hi) return false;
+    cb = (uint32_t)((key >> g.cs) - g.clb);
+    return true;
+}
+
+MP_INLINE uint32_t r3_fine(const R3Smem& S, const R3Geo& g, uint32_t cb, uint64_t key) {
+    const uint32_t l = S.clog[cb];
+    const uint32_t sub = l ? (uint32_t)((key >> (g.cs - l)) & ((1ull << l) - 1ull)) : 0u;
+    return (uint32_t)S.coff[cb] + sub;
+}
+
+// stable stream of all entries with key == k (id order) to out[ob ...]
+__device__ void r3_stream_equal(const R3Keys& K, const R3Out& out, int32_t n, uint64_t k, int32_t ob, uint32_t* sc) {
+    uint32_t run = 0;
+    for (int32_t b0 = 0; b0 < n; b0 += R2_THREADS) {
+        const int32_t t = b0 + threadIdx.x;
+        const bool sel = t < n && K.full(t) == k;
+        uint32_t tot;
+        const uint32_t pos = r3_scan(sel ? 1u : 0u, sc, tot);
+        if (sel) out.put(ob + (int32_t)(run + pos), (uint32_t)t);
+        run += tot;
+    }
+}
+
+MP_INLINE bool r3_less(uint64_t ka, uint16_t va, uint64_t kb, uint16_t vb) {
+    return ka < kb || (ka == kb && va < vb);
+}
+
+// One round: fine bins [b0, b1) (each <= R3_MID entries, total cnt <= R3_CAP).
+__device__ void r3_round(const R3Keys& K, const R3Out& out, int32_t n, const R3Geo& g, uint32_t need_bits,
+                         uint32_t b0, uint32_t b1, uint32_t base, uint32_t cnt, int32_t ob, R3Smem& S) {
+    // starts[b] hold exclusive prefixes; placement advances them with atomics, so
+    // afterwards bin b occupies [starts[b-1], starts[b]) (bin b0: [base, starts[b0])).
+    for (int32_t t = threadIdx.x; t < n; t += R2_THREADS) {
+        uint32_t cb;
+        uint64_t key;
+        if (!r3_locate(K, t, g, 0, cb, key)) continue;
+        const uint32_t f = r3_fine(S, g, cb, key);
+        if (f < b0 || f >= b1) continue;
+        const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
+        S.bk[slot] = key;
+        S.bv[slot] = (uint16_t)t;
+    }
+    (void)need_bits;
+    __syncthreads();
+    uint32_t* mids = S.misc + R3_MAXS * 6 + R3_MAXG * 3 + 8;   // [512]: count, then bins
+    if (threadIdx.x == 0) mids[0] = 0;
+    __syncthreads();
+    for (uint32_t b = b0 + threadIdx.x; b < b1; b += R2_THREADS) {
+        const uint32_t s0 = (b == b0 ? base : S.starts[b - 1]) - base;
+        const uint32_t s1 = S.starts[b] - base;
+        const uint32_t c = s1 - s0;
+        if (c < 2) continue;
+        if (c > (uint32_t)R3_TINY) {
+            const uint32_t k = atomicAdd(&mids[0], 1u);
+            if (k < 511) mids[1 + k] = b;
+            continue;
+        }
+        for (uint32_t i = s0 + 1; i < s1; i++) {
+            const uint64_t k = S.bk[i];
+            const uint16_t v = S.bv[i];
+            uint32_t j = i;
+            while (j > s0 && r3_less(k, v, S.bk[j - 1], S.bv[j - 1])) {
+                S.bk[j] = S.bk[j - 1];
+                S.bv[j] = S.bv[j - 1];
+                j--;
+            }
+            S.bk[j] = k;
+            S.bv[j] = v;
+        }
     }
     __syncthreads();
-    // exclusive offsets in (digit, warp) order: thread t owns digit t/4, warps 8*(t%4)..+8
     {
-        const int d = threadIdx.x >> 2, w0 = (threadIdx.x & 3) * 8;
-        uint32_t loc[8], s = 0;
+        const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+        const uint32_t nmid = min(mids[0], 511u);
+        for (uint32_t m = w; m < nmid; m += R2_WARPS) {
+            const uint32_t b = mids[1 + m];
+            const uint32_t s0 = (b == b0 ? base : S.starts[b - 1]) - base;
+            const uint32_t c = S.starts[b] - base - s0;
+            uint64_t kk[R3_MID / 32];
+            uint16_t vv[R3_MID / 32];
+            uint32_t rk[R3_MID / 32];
 #pragma unroll
-        for (int j = 0; j < 8; j++) {
-            loc[j] = hw[(w0 + j) * 256 + d];
-            s += loc[j];
-        }
-        uint32_t tot;
-        uint32_t run = r2_scan(s, sc, tot);
+            for (int u = 0; u < R3_MID / 32; u++) {
+                const uint32_t i = lane + 32 * u;
+                rk[u] = 0;
+                kk[u] = 0;
+                vv[u] = 0;
+                if (i < c) {
+                    kk[u] = S.bk[s0 + i];
+                    vv[u] = S.bv[s0 + i];
+                }
+            }
+            for (uint32_t j = 0; j < c; j++) {
+                const uint64_t kj = S.bk[s0 + j];
+                const uint16_t vj = S.bv[s0 + j];
 #pragma unroll
-        for (int j = 0; j < 8; j++) {
-            hw[(w0 + j) * 256 + d] = run;
-            run += loc[j];
+                for (int u = 0; u < R3_MID / 32; u++)
+                    if (lane + 32 * u < c && r3_less(kj, vj, kk[u], vv[u])) rk[u]++;
+            }
+            __syncwarp();
+#pragma unroll
+            for (int u = 0; u < R3_MID / 32; u++)
+                if (lane + 32 * u < c) {
+                    S.bk[s0 + rk[u]] = kk[u];
+                    S.bv[s0 + rk[u]] = vv[u];
+                }
+            __syncwarp();
         }
     }
     __syncthreads();
-    for (uint32_t b = ws; b < we; b += 32) {
-        const uint32_t i = b + lane;
-        const bool ok = i < we;
-        const uint32_t k = ok ? ks[i] : 0u;
-        const uint32_t d = ok ? (k >> sh) & 255u : 256u;
-        const uint32_t peers = __match_any_sync(0xffffffffu, d);
-        uint32_t off = 0;
-        if (ok) {
-            off = wh[d] + __popc(peers & lt);
-            kd[off] = k;
-            vd[off] = vs[i];
-        }
-        __syncwarp();
-        if (ok && (peers & lt) == 0) wh[d] += __popc(peers);
-        __syncwarp();
-    }
+    for (uint32_t j = threadIdx.x; j < cnt; j += R2_THREADS) out.put(ob + (int32_t)j, S.bv[j]);
     __syncthreads();
 }
 
-// Input sequences: key(i) and payload(i) for i in [0, n)
-struct R2CritIn {
-    const uint32_t* key;
-    MP_INLINE uint32_t k(int32_t i) const { return key[i]; }
-    MP_INLINE uint16_t p(int32_t i) const { return (uint16_t)i; }
-};
-struct R2GainIn {
-    const uint32_t* key;
-    const uint16_t* pi;
-    MP_INLINE uint32_t k(int32_t i) const { return key[i]; }
-    MP_INLINE uint16_t p(int32_t i) const { return pi[i]; }
-};
-struct R2PiOut {
-    uint16_t* pi;
-    MP_INLINE void put(int32_t pos, uint16_t v) const { pi[pos] = v; }
-};
-struct R2QOut {
-    int32_t* q;          // may be null
-    int32_t count;
-    uint32_t* head;      // smem
-    MP_INLINE void put(int32_t pos, uint16_t v) const {
-        if (pos == 0) *head = v;
-        if (q && pos < count) q[pos] = (int32_t)v;
-    }
-};
+MP_INLINE uint32_t r3_clog2(uint32_t x) { return x <= 1 ? 0u : 32u - __clz(x - 1); }   // ceil(log2 x)
 
-template <class In, class Out>
-__device__ void r2_stream_equal(const In& in, const Out& out, int32_t n, uint32_t key, int32_t obase, uint32_t* sc) {
-    uint32_t run = 0;
-    for (int32_t b0 = 0; b0 < n; b0 += R2_THREADS) {
-        const int32_t i = b0 + threadIdx.x;
-        const bool sel = i < n && in.k(i) == key;
-        uint32_t tot;
-        const uint32_t pos = r2_scan(sel ? 1u : 0u, sc, tot);
-        if (sel) out.put(obase + (int32_t)(run + pos), in.p(i));
-        run += tot;
-    }
-}
-
-template <class In, class Out>
-__device__ void r2_round(const In& in, const Out& out, int32_t n, uint32_t klo, uint32_t khi, uint32_t cnt,
-                         int32_t obase, R2Smem& S) {
-    uint32_t run = 0;
-    for (int32_t b0 = 0; b0 < n; b0 += R2_THREADS) {
-        const int32_t i = b0 + threadIdx.x;
-        uint32_t k = 0;
-        bool sel = false;
-        if (i < n) {
-            k = in.k(i);
-            sel = k >= klo && k <= khi;
-        }
-        uint32_t tot;
-        const uint32_t pos = r2_scan(sel ? 1u : 0u, S.scan, tot);
-        if (sel) {
-            S.k[0][run + pos] = k - klo;
-            S.v[0][run + pos] = in.p(i);
-        }
-        run += tot;
-    }
-    __syncthreads();
-    const uint32_t nb = r2_bitlen(khi - klo);
-    int cur = 0;
-    for (uint32_t sh = 0; sh < nb; sh += 8) {
-        r2_lsd_pass(S.k[cur], S.v[cur], S.k[cur ^ 1], S.v[cur ^ 1], cnt, (int)sh, S.hw, S.scan);
-        cur ^= 1;
-    }
-    for (uint32_t j = threadIdx.x; j < cnt; j += R2_THREADS) out.put(obase + (int32_t)j, S.v[cur][j]);
-    __syncthreads();
-}
-
-// Sort in[0..n) by key (stable: equal keys keep input order); out.put(position, payload).
-template <class In, class Out>
-__device__ void r2_sort(const In& in, const Out& out, int32_t n, R2Smem& S) {
+__device__ void r3_sort(const R3Keys& K, const R3Out& out, int32_t n, uint64_t kmin, uint64_t kmax, R3Smem& S) {
     if (n <= 0) return;
-    // key range
-    uint32_t lo = 0xffffffffu, hi = 0u;
-    for (int32_t i = threadIdx.x; i < n; i += R2_THREADS) {
-        const uint32_t k = in.k(i);
-        lo = min(lo, k);
-        hi = max(hi, k);
-    }
-    lo = __reduce_min_sync(0xffffffffu, lo);
-    hi = __reduce_max_sync(0xffffffffu, hi);
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    if (lane == 0) {
-        S.scan[w] = lo;
-        S.scan[32 + w] = hi;
-    }
-    __syncthreads();
-    uint32_t* stk = S.misc + 4 * R2_MAXG;          // [R2_MAXS][4]: lo, hi, obase, count
-    uint32_t* nstk = S.misc + 4 * R2_MAXG + 4 * R2_MAXS;
+    uint32_t* stk = S.misc;                        // [R3_MAXS][6]
+    uint32_t* grp = S.misc + R3_MAXS * 6;          // [R3_MAXG][3]: start fine bin, start prefix, kind
+    uint32_t* nstk = grp + R3_MAXG * 3;
+    auto push = [&](uint64_t lo, uint64_t hi, uint32_t ob, uint32_t cnt) {  // thread 0 only
+        uint32_t k = *nstk;
+        if (k >= (uint32_t)R3_MAXS) { __trap(); }
+        stk[k * 6] = (uint32_t)lo;
+        stk[k * 6 + 1] = (uint32_t)(lo >> 32);
+        stk[k * 6 + 2] = (uint32_t)hi;
+        stk[k * 6 + 3] = (uint32_t)(hi >> 32);
+        stk[k * 6 + 4] = ob;
+        stk[k * 6 + 5] = cnt;
+        *nstk = k + 1;
+    };
     if (threadIdx.x == 0) {
-        uint32_t a = 0xffffffffu, b = 0;
-        for (int j = 0; j < R2_WARPS; j++) {
-            a = min(a, S.scan[j]);
-            b = max(b, S.scan[32 + j]);
-        }
-        stk[0] = a;
-        stk[1] = b;
-        stk[2] = 0;
-        stk[3] = (uint32_t)n;
-        *nstk = 1;
+        *nstk = 0;
+        push(kmin, kmax, 0, (uint32_t)n);
     }
     __syncthreads();
     while (true) {
         const uint32_t ns = *nstk;
         if (ns == 0) break;
-        const uint32_t rlo = stk[(ns - 1) * 4], rhi = stk[(ns - 1) * 4 + 1];
-        const int32_t rob = (int32_t)stk[(ns - 1) * 4 + 2];
-        const uint32_t rcnt = stk[(ns - 1) * 4 + 3];
+        const uint32_t* top = stk + (ns - 1) * 6;
+        R3Geo g;
+        g.lo = (uint64_t)top[0] | ((uint64_t)top[1] << 32);
+        g.hi = (uint64_t)top[2] | ((uint64_t)top[3] << 32);
+        const int32_t ob = (int32_t)top[4];
+        const uint32_t rcnt = top[5];
         __syncthreads();
         if (threadIdx.x == 0) *nstk = ns - 1;
-        if (rlo == rhi) {
-            r2_stream_equal(in, out, n, rlo, rob, S.scan);
+        if (g.lo == g.hi) {
+            r3_stream_equal(K, out, n, g.lo, ob, S.sc);
             __syncthreads();
             continue;
         }
-        if (rcnt <= (uint32_t)R2_CAP) {
-            r2_round(in, out, n, rlo, rhi, rcnt, rob, S);
-            continue;
+        const uint64_t span = g.hi - g.lo;
+        const uint32_t bits = 64u - (uint32_t)__clzll((long long)span);
+        g.cs = bits > 12 ? bits - 12 : 0;
+        g.clb = g.lo >> g.cs;
+        g.ncb = (uint32_t)((g.hi >> g.cs) - g.clb + 1);
+        if (g.ncb > (uint32_t)R3_NC) {
+            g.cs++;
+            g.clb = g.lo >> g.cs;
+            g.ncb = (uint32_t)((g.hi >> g.cs) - g.clb + 1);
         }
-        // histogram of the range over <= 4096 bins
-        const uint32_t span = rhi - rlo;
-        const uint32_t shift = r2_bitlen(span) > 12 ? r2_bitlen(span) - 12 : 0;
-        const uint32_t nb = (span >> shift) + 1;
-        for (uint32_t b = threadIdx.x; b < R2_NBINS; b += R2_THREADS) S.hw[b] = 0;
+        // ---- pass 1: coarse histogram (in starts[0..NC)) ----
+        for (uint32_t b = threadIdx.x; b < (uint32_t)R3_NF + 64; b += R2_THREADS) S.starts[b] = 0;
         __syncthreads();
-        for (int32_t i = threadIdx.x; i < n; i += R2_THREADS) {
-            const uint32_t k = in.k(i);
-            if (k >= rlo && k <= rhi) atomicAdd(&S.hw[(k - rlo) >> shift], 1u);
+        for (int32_t t = threadIdx.x; t < n; t += R2_THREADS) {
+            uint32_t cb;
+            uint64_t key;
+            if (r3_locate(K, t, g, g.cs, cb, key)) atomicAdd(&S.starts[cb], 1u);
         }
         __syncthreads();
-        // group boundaries: a new group starts at bin 0, at a bin > CAP/2 or right after one,
-        // and where the exclusive prefix crosses a multiple of CAP/2 -- so every multi-bin
-        // group holds <= CAP entries; a single bin > CAP becomes a deferred (finer) range.
-        const uint32_t H = R2_CAP / 2;
-        uint32_t c4[4], s4 = 0;
+        // ---- sub-bins per coarse bin: 2^ceil(log2(c / T)) with T doubling until they fit ----
+        constexpr int CPER = R3_NC / R2_THREADS;  // 4
+        uint32_t cc[CPER];
 #pragma unroll
-        for (int j = 0; j < 4; j++) {
-            const uint32_t b = threadIdx.x * 4 + j;
-            c4[j] = b < nb ? S.hw[b] : 0u;
-            s4 += c4[j];
+        for (int j = 0; j < CPER; j++) cc[j] = S.starts[threadIdx.x * CPER + j];
+        uint32_t T = 4;
+        uint32_t lg[CPER], ftot = 0, fex = 0;
+        while (true) {
+            uint32_t s = 0;
+#pragma unroll
+            for (int j = 0; j < CPER; j++) {
+                const uint32_t b = threadIdx.x * CPER + j;
+                uint32_t l = 0;
+                if (b < g.ncb && cc[j] > T) l = min(r3_clog2((cc[j] + T - 1) / T), g.cs);
+                lg[j] = l;
+                s += (b < g.ncb) ? (1u << l) : 0u;
+            }
+            fex = r3_scan(s, S.sc, ftot);
+            if (ftot <= (uint32_t)R3_NF) break;
+            T *= 2;
         }
-        const uint32_t up = __shfl_up_sync(0xffffffffu, c4[3], 1);
-        const uint32_t prev_c = threadIdx.x == 0 ? 0u : (lane == 0 ? S.hw[threadIdx.x * 4 - 1] : up);
+        {
+            uint32_t e = fex;
+#pragma unroll
+            for (int j = 0; j < CPER; j++) {
+                const uint32_t b = threadIdx.x * CPER + j;
+                S.coff[b] = (uint16_t)e;
+                S.clog[b] = (uint8_t)lg[j];
+                if (b < g.ncb) e += 1u << lg[j];
+            }
+        }
+        __syncthreads();
+        // lowest key bit any fine bin depends on
+        uint32_t maxl = 0;
+#pragma unroll
+        for (int j = 0; j < CPER; j++) maxl = max(maxl, lg[j]);
+        maxl = __reduce_max_sync(0xffffffffu, maxl);
+        if ((threadIdx.x & 31) == 0) S.sc[40 + (threadIdx.x >> 5)] = maxl;
+        for (uint32_t b = threadIdx.x; b < (uint32_t)R3_NF + 64; b += R2_THREADS) S.starts[b] = 0;
+        __syncthreads();
+        uint32_t need = 0;
+        for (int w = 0; w < R2_WARPS; w++) need = max(need, S.sc[40 + w]);
+        need = g.cs - need;   // fine bins use key bits >= need
+        const uint32_t nfb = ftot;
+        // ---- pass 2: fine histogram ----
+        for (int32_t t = threadIdx.x; t < n; t += R2_THREADS) {
+            uint32_t cb;
+            uint64_t key;
+            if (r3_locate(K, t, g, need, cb, key)) atomicAdd(&S.starts[r3_fine(S, g, cb, key)], 1u);
+        }
+        __syncthreads();
+        // ---- prefixes over fine bins (12 per thread) + group boundaries ----
+        constexpr int PER = R3_NF / R2_THREADS;  // 12
+        const uint32_t H = R3_CAP - R3_MID;      // a multi-bin group never exceeds H + MID = CAP
+        uint32_t cnts[PER], sum = 0;
+#pragma unroll
+        for (int j = 0; j < PER; j++) {
+            cnts[j] = S.starts[threadIdx.x * PER + j];
+            sum += cnts[j];
+        }
+        const uint32_t prev_c = threadIdx.x == 0 ? 0u : S.starts[threadIdx.x * PER - 1];
         uint32_t tot;
-        const uint32_t ex = r2_scan(s4, S.scan, tot);   // (contains barriers: hw reads above are done)
+        const uint32_t ex = r3_scan(sum, S.sc, tot);
         uint32_t flags = 0;
         {
             uint32_t e = ex, pc = prev_c, pe = ex - prev_c;
 #pragma unroll
-            for (int j = 0; j < 4; j++) {
-                const uint32_t b = threadIdx.x * 4 + j;
-                if (b < nb && (b == 0 || c4[j] > H || pc > H || (e / H) != (pe / H))) flags |= 1u << j;
-                S.hw[b] = e;  // exclusive prefix of bin b (bins >= nb: the total)
+            for (int j = 0; j < PER; j++) {
+                const uint32_t b = threadIdx.x * PER + j;
+                const bool big = cnts[j] > (uint32_t)R3_MID;
+                const bool pbig = pc > (uint32_t)R3_MID;
+                if (b < nfb && (b == 0 || big || pbig || (e / H) != (pe / H))) flags |= 1u << j;
+                S.starts[b] = e;
                 pe = e;
-                pc = c4[j];
-                e += c4[j];
+                pc = cnts[j];
+                e += cnts[j];
             }
         }
+        if (threadIdx.x == 0) S.starts[R3_NF] = tot;
+        (void)rcnt;
         uint32_t ng;
-        const uint32_t gpos = r2_scan((uint32_t)__popc(flags), S.scan, ng);
-        uint32_t* grp = S.misc;  // [R2_MAXG][4]: start bin, start prefix
-        if (ng > R2_MAXG) {
-            // cannot happen for n < 65536 (<= 2n/(CAP/2)+1 groups); stay correct anyway:
-            // split the range at the middle bin into two deferred ranges with exact counts.
-            if (threadIdx.x == 0) {
-                const uint32_t m = nb / 2;
-                const uint32_t pm = S.hw[m];
-                uint32_t k2 = *nstk;
-                stk[k2 * 4] = rlo; stk[k2 * 4 + 1] = rlo + (m << shift) - 1u;
-                stk[k2 * 4 + 2] = (uint32_t)rob; stk[k2 * 4 + 3] = pm;
-                k2++;
-                stk[k2 * 4] = rlo + (m << shift); stk[k2 * 4 + 1] = rhi;
-                stk[k2 * 4 + 2] = (uint32_t)rob + pm; stk[k2 * 4 + 3] = tot - pm;
-                k2++;
-                *nstk = k2;
-            }
-            __syncthreads();
-            continue;
-        }
+        const uint32_t gp0 = r3_scan((uint32_t)__popc(flags), S.sc, ng);
+        if (ng > (uint32_t)R3_MAXG) __trap();
         {
-            uint32_t e = ex, gp = gpos;
+            uint32_t gp = gp0;
 #pragma unroll
-            for (int j = 0; j < 4; j++) {
+            for (int j = 0; j < PER; j++)
                 if ((flags >> j) & 1u) {
-                    grp[gp * 4] = threadIdx.x * 4 + j;
-                    grp[gp * 4 + 1] = e;
+                    const uint32_t b = threadIdx.x * PER + j;
+                    grp[gp * 3] = b;
+                    grp[gp * 3 + 1] = S.starts[b];
+                    grp[gp * 3 + 2] = cnts[j] > (uint32_t)R3_MID ? 1u : 0u;
                     gp++;
                 }
-                e += c4[j];
-            }
         }
         __syncthreads();
         for (uint32_t gi = 0; gi < ng; gi++) {
-            const uint32_t b0 = grp[gi * 4], e0 = grp[gi * 4 + 1];
-            const uint32_t b1 = gi + 1 < ng ? grp[(gi + 1) * 4] : nb;
-            const uint32_t e1 = gi + 1 < ng ? grp[(gi + 1) * 4 + 1] : tot;
+            const uint32_t b0 = grp[gi * 3], e0 = grp[gi * 3 + 1], kind = grp[gi * 3 + 2];
+            const uint32_t b1 = gi + 1 < ng ? grp[(gi + 1) * 3] : nfb;
+            const uint32_t e1 = gi + 1 < ng ? grp[(gi + 1) * 3 + 1] : tot;
             const uint32_t cnt = e1 - e0;
             if (cnt == 0) continue;
-            const uint32_t klo = rlo + (b0 << shift);
-            const uint32_t khi = b1 >= nb ? rhi : rlo + (b1 << shift) - 1u;
-            if (cnt <= (uint32_t)R2_CAP) {
-                r2_round(in, out, n, klo, khi, cnt, rob + (int32_t)e0, S);
+            if (kind == 0) {
+                r3_round(K, out, n, g, need, b0, b1, e0, cnt, ob + (int32_t)e0, S);
             } else {
-                __syncthreads();
                 if (threadIdx.x == 0) {
-                    uint32_t k2 = *nstk;
-                    stk[k2 * 4] = klo;
-                    stk[k2 * 4 + 1] = khi;
-                    stk[k2 * 4 + 2] = (uint32_t)(rob + (int32_t)e0);
-                    stk[k2 * 4 + 3] = cnt;
-                    *nstk = k2 + 1;
+                    // key range of fine bin b0: its coarse bin c (last with coff[c] <= b0), sub-bin b0-coff[c]
+                    uint32_t lo_c = 0, hi_c = g.ncb - 1;
+                    while (lo_c < hi_c) {
+                        const uint32_t mid = (lo_c + hi_c + 1) >> 1;
+                        if ((uint32_t)S.coff[mid] <= b0) lo_c = mid;
+                        else hi_c = mid - 1;
+                    }
+                    const uint32_t l = S.clog[lo_c];
+                    const uint32_t fs = g.cs - l;
+                    uint64_t blo = ((g.clb + lo_c) << g.cs) + ((uint64_t)(b0 - S.coff[lo_c]) << fs);
+                    uint64_t bhi = blo + ((1ull << fs) - 1ull);
+                    if (blo < g.lo) blo = g.lo;
+                    if (bhi > g.hi || bhi < blo) bhi = g.hi;
+                    if (fs == 0) bhi = blo;
+                    push(blo, bhi, (uint32_t)(ob + (int32_t)e0), cnt);
                 }
                 __syncthreads();
             }
@@ -557,66 +644,94 @@ __device__ void r2_sort(const In& in, const Out& out, int32_t n, R2Smem& S) {
 
 template <int A>
 __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
-    extern __shared__ __align__(16) unsigned char r2s[];
-    R2Smem S;
-    S.k[0] = reinterpret_cast<uint32_t*>(r2s);
-    S.k[1] = S.k[0] + R2_CAP;
-    S.v[0] = reinterpret_cast<uint16_t*>(S.k[1] + R2_CAP);
-    S.v[1] = S.v[0] + R2_CAP;
-    S.hw = reinterpret_cast<uint32_t*>(S.v[1] + R2_CAP);
-    S.scan = S.hw + 8192;
-    S.misc = S.scan + 64;
+    extern __shared__ __align__(16) unsigned char r3s[];
+    R3Smem S;
+    S.starts = reinterpret_cast<uint32_t*>(r3s);
+    S.bk = reinterpret_cast<uint64_t*>(r3s + (size_t)(R3_NF + 64) * 4);
+    S.bv = reinterpret_cast<uint16_t*>(S.bk + R3_CAP);
+    S.coff = reinterpret_cast<uint16_t*>(S.bv + R3_CAP);
+    S.clog = reinterpret_cast<uint8_t*>(S.coff + R3_NC + 64);
+    S.sc = reinterpret_cast<uint32_t*>(S.clog + R3_NC + 64);
+    S.misc = S.sc + 96;
     __shared__ uint32_t s_tick, s_head;
-    uint32_t* skey = a.s_key + (int64_t)blockIdx.x * a.n;
-    uint16_t* spi = a.s_pi + (int64_t)blockIdx.x * a.n;
+    __shared__ unsigned long long s_min[A], s_max[A];
+    uint32_t* critc = a.s_key + (int64_t)blockIdx.x * a.n * (A + 1);
+    uint32_t* gainc = critc + a.n;   // [A][n]
     bool bad = false;
     while (true) {
         if (threadIdx.x == 0) s_tick = atomicAdd(a.ticket, 1u);
+        if (threadIdx.x < A) {
+            s_min[threadIdx.x] = ~0ull;
+            s_max[threadIdx.x] = 0ull;
+        }
         __syncthreads();
         const int64_t rl = s_tick;
         __syncthreads();
         if (rl >= a.R) break;
         const int64_t r = a.r0 + rl;
         const float CP = a.cp[rl];
+        float hdv[A];
+#pragma unroll
+        for (int b = 0; b < A; b++) hdv[b] = u2f(a.hd[rl * A + b]);
+        // materialise critc and gainc_a (one hash per (t, a)); per-arch key range
+        unsigned long long mn[A], mx[A];
+#pragma unroll
+        for (int b = 0; b < A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
         for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
             const float blv = a.blT[rl * a.n + t];
             const float c = CP > 0.0f ? __fdiv_rn(blv, CP) : 0.0f;
-            skey[t] = ONE_BITS - f2u(c);
-        }
-        __syncthreads();
-        r2_sort(R2CritIn{skey}, R2PiOut{spi}, a.n, S);
-        __syncthreads();
-        int64_t qoff = 0;
-        for (int b = 0; b < A; b++) {
-            const float h = u2f(a.hd[rl * A + b]);
-            const int32_t cnt = a.counts[rl * A + b];
-            for (int32_t p = threadIdx.x; p < a.n; p += R2_THREADS) {
-                const int32_t t = spi[p];
-                float x[A];
-                uint32_t en;
-                int k;
-                float wt;
-                r2_durs<A>(a, r, t, x, en, k, wt, bad);
-                uint32_t key = 0x40000000u;  // not enabled: after every real key (<= 0x3F800000)
+            const uint32_t cc = ONE_BITS - f2u(c);
+            critc[t] = cc;
+            float x[A];
+            uint32_t en;
+            int k;
+            float wt;
+            r2_durs<A>(a, r, t, x, en, k, wt, bad);
+#pragma unroll
+            for (int b = 0; b < A; b++) {
+                uint32_t key = 0x40000000u;
                 if ((en >> b) & 1u) {
                     float gv;
                     if (k == 1) gv = 1.0f;
-                    else if (h == 0.0f) gv = 0.5f;
+                    else if (hdv[b] == 0.0f) gv = 0.5f;
                     else {
                         float ref = __uint_as_float(0x7f800000u);
 #pragma unroll
                         for (int q = 0; q < A; q++)
                             if (q != b && ((en >> q) & 1u)) ref = x[q] < ref ? x[q] : ref;
-                        gv = __fdiv_rn(__fadd_rn(__fsub_rn(ref, x[b]), h), __fadd_rn(h, h));
+                        gv = __fdiv_rn(__fadd_rn(__fsub_rn(ref, x[b]), hdv[b]), __fadd_rn(hdv[b], hdv[b]));
                     }
                     key = ONE_BITS - f2u(gv);
                 }
-                skey[p] = key;
+                gainc[(int64_t)b * a.n + t] = key;
+                const unsigned long long full = ((unsigned long long)key << 32) | cc;
+                mn[b] = full < mn[b] ? full : mn[b];
+                mx[b] = full > mx[b] ? full : mx[b];
             }
+        }
+#pragma unroll
+        for (int b = 0; b < A; b++) {
+            unsigned long long v1 = mn[b], v2 = mx[b];
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                unsigned long long y1 = __shfl_xor_sync(0xffffffffu, v1, o);
+                unsigned long long y2 = __shfl_xor_sync(0xffffffffu, v2, o);
+                v1 = y1 < v1 ? y1 : v1;
+                v2 = y2 > v2 ? y2 : v2;
+            }
+            if ((threadIdx.x & 31) == 0) {
+                atomicMin(&s_min[b], v1);
+                atomicMax(&s_max[b], v2);
+            }
+        }
+        __syncthreads();
+        int64_t qoff = 0;
+        for (int b = 0; b < A; b++) {
+            const int32_t cnt = a.counts[rl * A + b];
             if (threadIdx.x == 0) s_head = 0xffffffffu;
             __syncthreads();
             int32_t* qdst = a.qtask ? a.qtask + rl * (int64_t)a.n * A + qoff : nullptr;
-            r2_sort(R2GainIn{skey, spi}, R2QOut{qdst, cnt, &s_head}, a.n, S);
+            r3_sort(R3Keys{gainc + (int64_t)b * a.n, critc}, R3Out{qdst, cnt, &s_head}, a.n, s_min[b], s_max[b], S);
             __syncthreads();
             if (threadIdx.x == 0) {
                 mp_queue_summary o;
@@ -647,7 +762,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const int64_t groups = (R + 31) / 32;
     const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256((size_t)R * n * 4) + align256((size_t)R * A * 4) * 2 +
-                   align256((size_t)R * A * 16) + align256((size_t)grid2 * n * 4) + align256((size_t)grid2 * n * 2);
+                   align256((size_t)R * A * 16) + align256((size_t)grid2 * n * 4 * (A + 1)) + align256((size_t)grid2 * n * 2);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
     Rep2Args a{};
@@ -672,14 +787,14 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.counts = ar.take<int32_t>((size_t)R * A);
     a.brw = ar.take<unsigned long long>((size_t)R * A * 2);
     a.err = dag->err;
-    a.s_key = ar.take<uint32_t>((size_t)grid2 * n);
+    a.s_key = ar.take<uint32_t>((size_t)grid2 * n * (A + 1));
     a.s_pi = ar.take<uint16_t>((size_t)grid2 * n);
     a.qtask = qtask;
     a.sum = sum;
     a.ticket = dag->tickets + 56;
     static bool attr = false;
     const int smem1 = 32 * 32 * 33 * 4;
-    const int smem2 = (2 * R2_CAP * 4) + (2 * R2_CAP * 2) + 8192 * 4 + 64 * 4 + 512 * 4;
+    const int smem2 = (int)r3_smem_bytes();
     if (!attr) {
         MP_CUDA(cudaFuncSetAttribute(k_rep2_bl<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem1));
         MP_CUDA(cudaFuncSetAttribute(k_rep2_bl<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem1));
