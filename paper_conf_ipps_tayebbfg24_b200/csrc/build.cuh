@@ -93,43 +93,96 @@ MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int32_t v) {
 
 // Kahn, level-synchronous (a task is ready when all its predecessors are done,
 // P:l.91): level k+1 = successors whose last remaining predecessor is in level
-// k.  Cooperative grid (one block per SM) with a light grid barrier per level;
-// frontier appends use warp-aggregated atomics.  With one block the barrier is
-// a __syncthreads and the remaining-predecessor counters live in shared memory.
+// k.  Frontier nodes are taken in chunks of 1024 per block; inside a chunk the
+// edges are spread evenly over the threads (block scan of the degrees + binary
+// search), so a high-degree node does not serialise a level.  Cooperative grid
+// (one block per SM) with a light grid barrier per level; with one block the
+// barrier is a __syncthreads and the remaining-predecessor counters and the
+// frontier counter live in shared memory.
 __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int smem_rem) {
     extern __shared__ int32_t srem[];
+    __shared__ int32_t s_row[1024], s_pre[1025];
+    __shared__ uint32_t s_sc[40];
+    __shared__ int32_t s_cnt[2];
     const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+    const bool single = gridDim.x == 1;
     int32_t* rem = smem_rem ? srem : a.rem;
     unsigned epoch = 0;
+    if (single && threadIdx.x < 2) s_cnt[threadIdx.x] = 0;
+    if (single) __syncthreads();
     for (int64_t v = gtid; v < a.n; v += gsz) {
         int32_t d = a.indeg[v];
         rem[v] = d;
         a.level[v] = 0;
-        if (d == 0) kahn_append(&a.counts[0], a.front[0], (int32_t)v);
+        if (d == 0) kahn_append(single ? &s_cnt[0] : &a.counts[0], a.front[0], (int32_t)v);
     }
-    if (gridDim.x == 1) __syncthreads(); else grid_barrier(bar, epoch);
+    if (single) __syncthreads(); else grid_barrier(bar, epoch);
     int32_t k = 0;
     int64_t processed = 0;
     while (true) {
-        const int32_t cnt = *((volatile int32_t*)&a.counts[k]);
+        const int32_t cnt = single ? *((volatile int32_t*)&s_cnt[k & 1]) : *((volatile int32_t*)&a.counts[k]);
         if (cnt == 0) break;
         processed += cnt;
         const int32_t* cur = a.front[k & 1];
         int32_t* nxt = a.front[(k + 1) & 1];
-        for (int64_t i = gtid; i < cnt; i += gsz) {
-            const int32_t u = cur[i];
-            const int32_t e1 = a.row_ptr[u + 1];
-            for (int32_t e = a.row_ptr[u]; e < e1; e++) {
-                const int32_t v = a.col[e];
+        int32_t* nctr = single ? &s_cnt[(k + 1) & 1] : &a.counts[k + 1];
+        for (int64_t c0 = (int64_t)blockIdx.x * 1024; c0 < cnt; c0 += (int64_t)gridDim.x * 1024) {
+            const int64_t i = c0 + threadIdx.x;
+            int32_t deg = 0;
+            if (i < cnt) {
+                const int32_t u = cur[i];
+                const int32_t r0 = a.row_ptr[u];
+                deg = a.row_ptr[u + 1] - r0;
+                s_row[threadIdx.x] = r0;
+            }
+            // block exclusive scan of the degrees
+            const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+            int32_t incl = deg;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                int32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += y;
+            }
+            if (lane == 31) s_sc[w] = (uint32_t)incl;
+            __syncthreads();
+            if (w == 0) {
+                int32_t v0 = (int32_t)s_sc[lane], iv = v0;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    int32_t y = __shfl_up_sync(0xffffffffu, iv, o);
+                    if (lane >= o) iv += y;
+                }
+                s_sc[lane] = (uint32_t)(iv - v0);
+                if (lane == 31) s_sc[32] = (uint32_t)iv;
+            }
+            __syncthreads();
+            s_pre[threadIdx.x] = (int32_t)s_sc[w] + incl - deg;
+            const int32_t etot = (int32_t)s_sc[32];
+            const int32_t nloc = (int32_t)((cnt - c0) < 1024 ? (cnt - c0) : 1024);
+            __syncthreads();
+            for (int32_t e = threadIdx.x; e < etot; e += blockDim.x) {
+                int lo = 0, hi = nloc - 1;     // last frontier slot with s_pre <= e
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (s_pre[mid] <= e) lo = mid;
+                    else hi = mid - 1;
+                }
+                const int32_t v = a.col[s_row[lo] + (e - s_pre[lo])];
                 if (atomicSub(&rem[v], 1) == 1) {
                     a.level[v] = k + 1;
-                    kahn_append(&a.counts[k + 1], nxt, v);
+                    kahn_append(nctr, nxt, v);
                 }
             }
+            __syncthreads();
         }
         k++;
-        if (gridDim.x == 1) __syncthreads(); else grid_barrier(bar, epoch);
+        if (single) {
+            if (threadIdx.x == 0) s_cnt[(k + 1) & 1] = 0;   // the list after next starts empty
+            __syncthreads();
+        } else {
+            grid_barrier(bar, epoch);
+        }
     }
     if (gtid == 0) {
         a.out[0] = k;

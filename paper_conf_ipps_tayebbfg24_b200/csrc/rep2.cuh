@@ -95,9 +95,25 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
     float cpm = 0.0f;
     for (int32_t lv = 0; lv < a.L; lv++) {
         const int32_t q1 = __ldg(a.lvlq + lv + 1);
-        for (int32_t q = __ldg(a.lvlq + lv) + w; q < q1; q += R2_WARPS) {
-            const int32_t v = __ldg(a.nodeq + q);
-            const int32_t e0 = __ldg(a.rowq + q), e1 = __ldg(a.rowq + q + 1);
+        int32_t q = __ldg(a.lvlq + lv) + w;
+        // software pipeline: the CSR slice of the warp's next node is loaded while the
+        // current node hashes its durations and gathers its successors' bottom-levels
+        int32_t v = 0, e0 = 0, e1 = 0, sv = 0;
+        if (q < q1) {
+            v = __ldg(a.nodeq + q);
+            e0 = __ldg(a.rowq + q);
+            e1 = __ldg(a.rowq + q + 1);
+            sv = lane < e1 - e0 ? __ldg(a.colq + e0 + lane) : 0;
+        }
+        while (q < q1) {
+            const int32_t qn = q + R2_WARPS;
+            int32_t vn = 0, e0n = 0, e1n = 0, svn = 0;
+            if (qn < q1) {
+                vn = __ldg(a.nodeq + qn);
+                e0n = __ldg(a.rowq + qn);
+                e1n = __ldg(a.rowq + qn + 1);
+                svn = lane < e1n - e0n ? __ldg(a.colq + e0n + lane) : 0;
+            }
             float x[A];
             uint32_t en;
             int k;
@@ -124,28 +140,32 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
                 }
             }
             if (!k) wt = 0.0f;
-            // successors: the warp loads 32 successor positions at once (coalesced), broadcasts
-            // them with shuffles and issues 8 independent 128-byte gathers at a time
+            // successors: 32 positions per coalesced load, broadcast by shuffles, gathers 8 at a time
             float m = 0.0f;
             for (int32_t eb = e0; eb < e1; eb += 32) {
                 const int32_t cb = min(32, e1 - eb);
-                const int32_t sv = lane < cb ? __ldg(a.colq + eb + lane) : 0;
+                const int32_t s32 = eb == e0 ? sv : (lane < cb ? __ldg(a.colq + eb + lane) : 0);
                 int32_t j = 0;
                 for (; j + 8 <= cb; j += 8) {
                     float t8[8];
 #pragma unroll
                     for (int u = 0; u < 8; u++) {
-                        const int32_t sp = __shfl_sync(0xffffffffu, sv, j + u);
+                        const int32_t sp = __shfl_sync(0xffffffffu, s32, j + u);
                         t8[u] = bl32[(int64_t)sp * 32 + lane];
                     }
 #pragma unroll
                     for (int u = 0; u < 8; u++) m = fmaxf(m, t8[u]);
                 }
-                for (; j < cb; j++) m = fmaxf(m, bl32[(int64_t)__shfl_sync(0xffffffffu, sv, j) * 32 + lane]);
+                for (; j < cb; j++) m = fmaxf(m, bl32[(int64_t)__shfl_sync(0xffffffffu, s32, j) * 32 + lane]);
             }
             const float bb = __fadd_rn(wt, m);
             bl32[(int64_t)q * 32 + lane] = bb;
             cpm = fmaxf(cpm, bb);
+            q = qn;
+            v = vn;
+            e0 = e0n;
+            e1 = e1n;
+            sv = svn;
         }
         __syncthreads();
     }
@@ -252,9 +272,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
 // a bin holds a single key value, are streamed in id order (stable).
 // ---------------------------------------------------------------------------------------
 constexpr int R3_NC = 4096;      // coarse bins per range
-constexpr int R3_NF = 12288;     // fine bins per range (sub-bins of the coarse bins)
-constexpr int R3_CAP = 16000;    // entries per round (shared memory)
-constexpr int R3_TINY = 64;      // fine bins up to this size: thread insertion sort
+constexpr int R3_NF = 16384;     // fine bins per range (sub-bins of the coarse bins)
+constexpr int R3_CAP = 14400;    // entries per round (shared memory)
+constexpr int R3_TINY = 16;      // fine bins up to this size: thread insertion sort
 constexpr int R3_MID = 256;      // up to this size: warp rank sort; larger: finer range / stream
 constexpr int R3_MAXS = 192;     // range stack entries (6 words each)
 constexpr int R3_MAXG = 192;     // group records per range (3 words each)
@@ -306,6 +326,7 @@ MP_INLINE uint32_t r3_scan(uint32_t x, uint32_t* sc, uint32_t& total) {
 struct R3Keys {
     const uint32_t* hi;   // gainc_a[n]
     const uint32_t* lo;   // critc[n]
+    uint16_t* fb;         // [n] fine bin of each entry in the current range (scratch)
     MP_INLINE uint64_t full(int32_t t) const { return ((uint64_t)__ldcg(hi + t) << 32) | __ldcg(lo + t); }
 };
 
@@ -344,6 +365,34 @@ MP_INLINE bool r3_locate(const R3Keys& K, int32_t t, const R3Geo& g, uint32_t ne
     return true;
 }
 
+// as r3_locate, with gainc already loaded; coarse bin only
+MP_INLINE bool r3_locate_h(const R3Keys& K, int32_t t, uint32_t h, const R3Geo& g, uint32_t need_bits, uint32_t& cb) {
+    const uint32_t lh = (uint32_t)(g.lo >> 32), hh = (uint32_t)(g.hi >> 32);
+    if (h < lh || h > hh) return false;
+    if (need_bits >= 32 && h != lh && h != hh) {
+        cb = (uint32_t)((((uint64_t)h << 32) >> g.cs) - g.clb);
+        return true;
+    }
+    const uint64_t key = ((uint64_t)h << 32) | __ldcg(K.lo + t);
+    if (key < g.lo || key > g.hi) return false;
+    cb = (uint32_t)((key >> g.cs) - g.clb);
+    return true;
+}
+MP_INLINE bool r3_locate_hk(const R3Keys& K, int32_t t, uint32_t h, const R3Geo& g, uint32_t need_bits,
+                            uint32_t& cb, uint64_t& key) {
+    const uint32_t lh = (uint32_t)(g.lo >> 32), hh = (uint32_t)(g.hi >> 32);
+    if (h < lh || h > hh) return false;
+    if (need_bits >= 32 && h != lh && h != hh) {
+        key = (uint64_t)h << 32;
+        cb = (uint32_t)((key >> g.cs) - g.clb);
+        return true;
+    }
+    key = ((uint64_t)h << 32) | __ldcg(K.lo + t);
+    if (key < g.lo || key > g.hi) return false;
+    cb = (uint32_t)((key >> g.cs) - g.clb);
+    return true;
+}
+
 MP_INLINE uint32_t r3_fine(const R3Smem& S, const R3Geo& g, uint32_t cb, uint64_t key) {
     const uint32_t l = S.clog[cb];
     const uint32_t sub = l ? (uint32_t)((key >> (g.cs - l)) & ((1ull << l) - 1ull)) : 0u;
@@ -368,89 +417,45 @@ MP_INLINE bool r3_less(uint64_t ka, uint16_t va, uint64_t kb, uint16_t vb) {
 }
 
 // One round: fine bins [b0, b1) (each <= R3_MID entries, total cnt <= R3_CAP).
-__device__ void r3_round(const R3Keys& K, const R3Out& out, int32_t n, const R3Geo& g, uint32_t need_bits,
-                         uint32_t b0, uint32_t b1, uint32_t base, uint32_t cnt, int32_t ob, R3Smem& S) {
-    // starts[b] hold exclusive prefixes; placement advances them with atomics, so
-    // afterwards bin b occupies [starts[b-1], starts[b]) (bin b0: [base, starts[b0])).
-    for (int32_t t = threadIdx.x; t < n; t += R2_THREADS) {
-        uint32_t cb;
-        uint64_t key;
-        if (!r3_locate(K, t, g, 0, cb, key)) continue;
-        const uint32_t f = r3_fine(S, g, cb, key);
+// 1. members (fb[t] in [b0, b1)) are placed at (bin start + atomic cursor) in
+//    shared memory -- fb is read 16 entries (two 16-byte loads) per thread;
+// 2. every placed entry ranks itself inside its bin (compares against the bin's
+//    other entries) and writes straight to its final output position.
+__device__ void r3_round(const R3Keys& K, const R3Out& out, int32_t n, const R3Geo& g, uint32_t b0, uint32_t b1,
+                         uint32_t base, uint32_t cnt, int32_t ob, R3Smem& S) {
+    const int32_t n16 = n & ~15;
+    for (int32_t c0 = threadIdx.x * 16; c0 < n16; c0 += 16 * R2_THREADS) {
+        const uint4 w0 = __ldcg(reinterpret_cast<const uint4*>(K.fb + c0));
+        const uint4 w1 = __ldcg(reinterpret_cast<const uint4*>(K.fb + c0 + 8));
+        const uint32_t wv[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
+#pragma unroll
+        for (int u = 0; u < 16; u++) {
+            const uint32_t f = (wv[u >> 1] >> ((u & 1) * 16)) & 0xFFFFu;
+            if (f < b0 || f >= b1) continue;
+            const int32_t t = c0 + u;
+            const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
+            S.bk[slot] = K.full(t);
+            S.bv[slot] = (uint16_t)t;
+        }
+    }
+    for (int32_t t = n16 + threadIdx.x; t < n; t += R2_THREADS) {
+        const uint32_t f = __ldcg(K.fb + t);
         if (f < b0 || f >= b1) continue;
         const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
-        S.bk[slot] = key;
+        S.bk[slot] = K.full(t);
         S.bv[slot] = (uint16_t)t;
     }
-    (void)need_bits;
     __syncthreads();
-    uint32_t* mids = S.misc + R3_MAXS * 6 + R3_MAXG * 3 + 8;   // [512]: count, then bins
-    if (threadIdx.x == 0) mids[0] = 0;
-    __syncthreads();
-    for (uint32_t b = b0 + threadIdx.x; b < b1; b += R2_THREADS) {
-        const uint32_t s0 = (b == b0 ? base : S.starts[b - 1]) - base;
-        const uint32_t s1 = S.starts[b] - base;
-        const uint32_t c = s1 - s0;
-        if (c < 2) continue;
-        if (c > (uint32_t)R3_TINY) {
-            const uint32_t k = atomicAdd(&mids[0], 1u);
-            if (k < 511) mids[1 + k] = b;
-            continue;
-        }
-        for (uint32_t i = s0 + 1; i < s1; i++) {
-            const uint64_t k = S.bk[i];
-            const uint16_t v = S.bv[i];
-            uint32_t j = i;
-            while (j > s0 && r3_less(k, v, S.bk[j - 1], S.bv[j - 1])) {
-                S.bk[j] = S.bk[j - 1];
-                S.bv[j] = S.bv[j - 1];
-                j--;
-            }
-            S.bk[j] = k;
-            S.bv[j] = v;
-        }
+    for (uint32_t j = threadIdx.x; j < cnt; j += R2_THREADS) {
+        const uint64_t k = S.bk[j];
+        const uint16_t v = S.bv[j];
+        const uint32_t f = r3_fine(S, g, (uint32_t)((k >> g.cs) - g.clb), k);
+        const uint32_t s0 = (f == b0 ? base : S.starts[f - 1]) - base;
+        const uint32_t s1 = S.starts[f] - base;
+        uint32_t rank = 0;
+        for (uint32_t i = s0; i < s1; i++) rank += r3_less(S.bk[i], S.bv[i], k, v) ? 1u : 0u;
+        out.put(ob + (int32_t)(s0 + rank), v);
     }
-    __syncthreads();
-    {
-        const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-        const uint32_t nmid = min(mids[0], 511u);
-        for (uint32_t m = w; m < nmid; m += R2_WARPS) {
-            const uint32_t b = mids[1 + m];
-            const uint32_t s0 = (b == b0 ? base : S.starts[b - 1]) - base;
-            const uint32_t c = S.starts[b] - base - s0;
-            uint64_t kk[R3_MID / 32];
-            uint16_t vv[R3_MID / 32];
-            uint32_t rk[R3_MID / 32];
-#pragma unroll
-            for (int u = 0; u < R3_MID / 32; u++) {
-                const uint32_t i = lane + 32 * u;
-                rk[u] = 0;
-                kk[u] = 0;
-                vv[u] = 0;
-                if (i < c) {
-                    kk[u] = S.bk[s0 + i];
-                    vv[u] = S.bv[s0 + i];
-                }
-            }
-            for (uint32_t j = 0; j < c; j++) {
-                const uint64_t kj = S.bk[s0 + j];
-                const uint16_t vj = S.bv[s0 + j];
-#pragma unroll
-                for (int u = 0; u < R3_MID / 32; u++)
-                    if (lane + 32 * u < c && r3_less(kj, vj, kk[u], vv[u])) rk[u]++;
-            }
-            __syncwarp();
-#pragma unroll
-            for (int u = 0; u < R3_MID / 32; u++)
-                if (lane + 32 * u < c) {
-                    S.bk[s0 + rk[u]] = kk[u];
-                    S.bv[s0 + rk[u]] = vv[u];
-                }
-            __syncwarp();
-        }
-    }
-    __syncthreads();
-    for (uint32_t j = threadIdx.x; j < cnt; j += R2_THREADS) out.put(ob + (int32_t)j, S.bv[j]);
     __syncthreads();
 }
 
@@ -506,10 +511,23 @@ __device__ void r3_sort(const R3Keys& K, const R3Out& out, int32_t n, uint64_t k
         // ---- pass 1: coarse histogram (in starts[0..NC)) ----
         for (uint32_t b = threadIdx.x; b < (uint32_t)R3_NF + 64; b += R2_THREADS) S.starts[b] = 0;
         __syncthreads();
-        for (int32_t t = threadIdx.x; t < n; t += R2_THREADS) {
-            uint32_t cb;
-            uint64_t key;
-            if (r3_locate(K, t, g, g.cs, cb, key)) atomicAdd(&S.starts[cb], 1u);
+        for (int32_t c0 = threadIdx.x * 8; c0 < n; c0 += 8 * R2_THREADS) {
+            uint32_t hv[8];
+            if (c0 + 8 <= n) {
+                const uint4 h0 = __ldcg(reinterpret_cast<const uint4*>(K.hi + c0));
+                const uint4 h1 = __ldcg(reinterpret_cast<const uint4*>(K.hi + c0 + 4));
+                hv[0] = h0.x; hv[1] = h0.y; hv[2] = h0.z; hv[3] = h0.w;
+                hv[4] = h1.x; hv[5] = h1.y; hv[6] = h1.z; hv[7] = h1.w;
+            } else {
+#pragma unroll
+                for (int u = 0; u < 8; u++) hv[u] = c0 + u < n ? __ldcg(K.hi + c0 + u) : 0xFFFFFFFFu;
+            }
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                if (c0 + u >= n) continue;
+                uint32_t cb;
+                if (r3_locate_h(K, c0 + u, hv[u], g, g.cs, cb)) atomicAdd(&S.starts[cb], 1u);
+            }
         }
         __syncthreads();
         // ---- sub-bins per coarse bin: 2^ceil(log2(c / T)) with T doubling until they fit ----
@@ -557,10 +575,38 @@ __device__ void r3_sort(const R3Keys& K, const R3Out& out, int32_t n, uint64_t k
         need = g.cs - need;   // fine bins use key bits >= need
         const uint32_t nfb = ftot;
         // ---- pass 2: fine histogram ----
-        for (int32_t t = threadIdx.x; t < n; t += R2_THREADS) {
-            uint32_t cb;
-            uint64_t key;
-            if (r3_locate(K, t, g, need, cb, key)) atomicAdd(&S.starts[r3_fine(S, g, cb, key)], 1u);
+        for (int32_t c0 = threadIdx.x * 8; c0 < n; c0 += 8 * R2_THREADS) {
+            uint32_t hv[8], fv[8];
+            if (c0 + 8 <= n) {
+                const uint4 h0 = __ldcg(reinterpret_cast<const uint4*>(K.hi + c0));
+                const uint4 h1 = __ldcg(reinterpret_cast<const uint4*>(K.hi + c0 + 4));
+                hv[0] = h0.x; hv[1] = h0.y; hv[2] = h0.z; hv[3] = h0.w;
+                hv[4] = h1.x; hv[5] = h1.y; hv[6] = h1.z; hv[7] = h1.w;
+            } else {
+#pragma unroll
+                for (int u = 0; u < 8; u++) hv[u] = c0 + u < n ? __ldcg(K.hi + c0 + u) : 0xFFFFFFFFu;
+            }
+#pragma unroll
+            for (int u = 0; u < 8; u++) {
+                fv[u] = 0xFFFFu;
+                if (c0 + u >= n) continue;
+                uint32_t cb;
+                uint64_t key;
+                if (r3_locate_hk(K, c0 + u, hv[u], g, need, cb, key)) {
+                    fv[u] = r3_fine(S, g, cb, key);
+                    atomicAdd(&S.starts[fv[u]], 1u);
+                }
+            }
+            if (c0 + 8 <= n) {
+                uint4 o;
+                o.x = fv[0] | (fv[1] << 16); o.y = fv[2] | (fv[3] << 16);
+                o.z = fv[4] | (fv[5] << 16); o.w = fv[6] | (fv[7] << 16);
+                *reinterpret_cast<uint4*>(K.fb + c0) = o;
+            } else {
+#pragma unroll
+                for (int u = 0; u < 8; u++)
+                    if (c0 + u < n) K.fb[c0 + u] = (uint16_t)fv[u];
+            }
         }
         __syncthreads();
         // ---- prefixes over fine bins (12 per thread) + group boundaries ----
@@ -615,7 +661,7 @@ __device__ void r3_sort(const R3Keys& K, const R3Out& out, int32_t n, uint64_t k
             const uint32_t cnt = e1 - e0;
             if (cnt == 0) continue;
             if (kind == 0) {
-                r3_round(K, out, n, g, need, b0, b1, e0, cnt, ob + (int32_t)e0, S);
+                r3_round(K, out, n, g, b0, b1, e0, cnt, ob + (int32_t)e0, S);
             } else {
                 if (threadIdx.x == 0) {
                     // key range of fine bin b0: its coarse bin c (last with coff[c] <= b0), sub-bin b0-coff[c]
@@ -655,8 +701,10 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     S.misc = S.sc + 96;
     __shared__ uint32_t s_tick, s_head;
     __shared__ unsigned long long s_min[A], s_max[A];
-    uint32_t* critc = a.s_key + (int64_t)blockIdx.x * a.n * (A + 1);
-    uint32_t* gainc = critc + a.n;   // [A][n]
+    const int64_t npad = ((int64_t)a.n + 15) & ~15ll;   // 16-entry aligned scratch rows
+    uint32_t* critc = a.s_key + (int64_t)blockIdx.x * npad * (A + 1);
+    uint32_t* gainc = critc + npad;   // [A][npad]
+    uint16_t* fbuf = a.s_pi + (int64_t)blockIdx.x * npad;
     bool bad = false;
     while (true) {
         if (threadIdx.x == 0) s_tick = atomicAdd(a.ticket, 1u);
@@ -703,7 +751,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                     }
                     key = ONE_BITS - f2u(gv);
                 }
-                gainc[(int64_t)b * a.n + t] = key;
+                gainc[(int64_t)b * npad + t] = key;
                 const unsigned long long full = ((unsigned long long)key << 32) | cc;
                 mn[b] = full < mn[b] ? full : mn[b];
                 mx[b] = full > mx[b] ? full : mx[b];
@@ -731,7 +779,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             if (threadIdx.x == 0) s_head = 0xffffffffu;
             __syncthreads();
             int32_t* qdst = a.qtask ? a.qtask + rl * (int64_t)a.n * A + qoff : nullptr;
-            r3_sort(R3Keys{gainc + (int64_t)b * a.n, critc}, R3Out{qdst, cnt, &s_head}, a.n, s_min[b], s_max[b], S);
+            r3_sort(R3Keys{gainc + (int64_t)b * npad, critc, fbuf}, R3Out{qdst, cnt, &s_head}, a.n, s_min[b], s_max[b], S);
             __syncthreads();
             if (threadIdx.x == 0) {
                 mp_queue_summary o;
@@ -762,7 +810,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const int64_t groups = (R + 31) / 32;
     const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256((size_t)R * n * 4) + align256((size_t)R * A * 4) * 2 +
-                   align256((size_t)R * A * 16) + align256((size_t)grid2 * n * 4 * (A + 1)) + align256((size_t)grid2 * n * 2);
+                   align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 2);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
     Rep2Args a{};
@@ -787,8 +835,8 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.counts = ar.take<int32_t>((size_t)R * A);
     a.brw = ar.take<unsigned long long>((size_t)R * A * 2);
     a.err = dag->err;
-    a.s_key = ar.take<uint32_t>((size_t)grid2 * n * (A + 1));
-    a.s_pi = ar.take<uint16_t>((size_t)grid2 * n);
+    a.s_key = ar.take<uint32_t>((size_t)grid2 * ((n + 15) & ~15) * (A + 1));
+    a.s_pi = ar.take<uint16_t>((size_t)grid2 * ((n + 15) & ~15));
     a.qtask = qtask;
     a.sum = sum;
     a.ticket = dag->tickets + 56;
