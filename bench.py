@@ -184,19 +184,43 @@ def run_reference(args):
 # our arm
 # --------------------------------------------------------------------------------------------------
 def kernel_alg_bytes(name, ctx):
-    """Algorithmic (compulsory) bytes per launch of the dominant kernel (DESIGN.md §6 table)."""
+    """Algorithmic (compulsory) HBM bytes per launch of the dominant kernel (DESIGN.md §6 table).
+
+    k_rep2_sort : per replica, read bl[n] (4n) + write the A queues (4nA)
+    k_rep2_bl   : per 32-replica group, read the CSR (4(n+1)+4E) and base durations (4nA);
+                  per replica write bl[n] (4n)
+    k_sort_pass : per pass, read + write (8 B key + 4 B id) per entry
+    k_bl_flow / k_bl_small : CSR once (4(n+1)+4E), durations (4nA), bl out (4n)
+    """
     n, E, A = ctx["n"], ctx["E"], ctx["A"]
+    R = ctx.get("replicas_per_launch", 1)
+    if name.startswith("k_rep2_sort"):
+        return R * (4 * n + 4 * n * A)
+    if name.startswith("k_rep2_bl"):
+        groups = (R + 31) // 32
+        return groups * (4 * (n + 1) + 4 * E + 4 * n * A) + R * 4 * n
     if name == "k_rep_main":
-        # per replica: read base durations 4nA, CSR 4(n+1)+4E once per launch; write sort input 12 B per (t,a)
-        rb = ctx["replicas_per_launch"]
-        return 4 * n * A + 4 * (n + 1) + 4 * E + rb * 12 * n * A
+        return 4 * n * A + 4 * (n + 1) + 4 * E + R * 12 * n * A
     if name == "k_sort_pass":
         return 24 * ctx["sort_entries_per_launch"]
-    if name == "k_rep_out":
-        return ctx["replicas_per_launch"] * (4 * n * A * 2)
-    if name == "k_bl_flow" or name == "k_bl_small":
+    if name in ("k_bl_flow", "k_bl_small"):
         return 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n
+    if name == "k_kahn":
+        return 4 * (n + 1) + 4 * E + 4 * n * 2   # CSR + indeg in, level out
     return None
+
+
+TRAFFIC_FILE = os.path.join(ROOT, "profiles", "r01", "traffic.json")
+
+
+def measured_traffic(kernel, cfg):
+    """dram read+write bytes per launch from a committed `ncu --set full` capture, if any."""
+    try:
+        t = json.load(open(TRAFFIC_FILE))
+        e = t.get(cfg, {}).get(kernel)
+        return (e["dram_bytes_per_launch"], e["source"]) if e else (None, None)
+    except Exception:
+        return None, None
 
 
 def run_ours(args):
@@ -358,18 +382,17 @@ def run_ours(args):
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
     ctx = dict(n=n, E=E, A=A)
     if cfg == "c5":
-        per = (256 << 20) // (n * A * 24)
-        rpl = max(1, min(cnt, per, 1024))
-        ctx["replicas_per_launch"] = rpl
-        ctx["sort_entries_per_launch"] = rpl * A * n
+        ctx["replicas_per_launch"] = cnt      # one k_rep2_bl / k_rep2_sort launch covers the rank's block
+        ctx["sort_entries_per_launch"] = cnt * A * n
     else:
         ctx["replicas_per_launch"] = 1
         ctx["sort_entries_per_launch"] = n * A
     alg = kernel_alg_bytes(dom, ctx)
     avg_ms = dom_ms / max(dom_launches, 1)
     achieved = (alg / (avg_ms * 1e-3) / 1e9) if alg else None
+    traffic, traffic_src = measured_traffic(dom, cfg)
     roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": (achieved / peak) if achieved else None, "traffic": None,
+            "frac": (achieved / peak) if achieved else None, "traffic": traffic, "traffic_source": traffic_src,
             "alg_bytes_per_launch": alg, "avg_launch_ms": avg_ms, "launches": dom_launches,
             "share_of_step": (dom_ms / args.steps) / ms_per_step, "peak_source": peak_src,
             "per_kernel_ms_per_step": {k: round(v, 4) for k, v in sorted(step_dev_ms.items(), key=lambda x: -x[1])}}

@@ -5,7 +5,7 @@ import collections, csv, io, os, re, subprocess, sys, tempfile
 
 rep, kre, mangled = sys.argv[1], sys.argv[2], sys.argv[3]
 top = int(sys.argv[4]) if len(sys.argv) > 4 else 25
-lib = os.path.join(os.path.dirname(os.path.abspath(__file__)), "paper_conf_ipps_tayebbfg24_b200", "libmp.so")
+lib = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_ipps_tayebbfg24_b200", "libmp.so")
 tmp = tempfile.mkdtemp()
 subprocess.run(["cuobjdump", "-xelf", "all", lib], cwd=tmp, capture_output=True)
 cub = [f for f in os.listdir(tmp) if f.endswith(".cubin")][0]
