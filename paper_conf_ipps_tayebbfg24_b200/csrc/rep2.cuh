@@ -334,9 +334,18 @@ struct R3Out {
     int32_t* q;       // queue destination or null
     int32_t count;    // enabled entries (positions >= count are not written)
     uint32_t* head;   // shared
-    MP_INLINE void put(int32_t pos, uint32_t t) const {
+    MP_INLINE void put(int32_t pos, uint32_t t, uint64_t) const {
         if (pos == 0) *head = t;
-        if (q && pos < count) q[pos] = (int32_t)t;
+        if (q && pos < count) __stcs(q + pos, (int32_t)t);   // streaming: keep L2 for the scratch
+    }
+};
+
+struct R3PosOut {      // sorted order into scratch: P[pos] = t, Dk[pos] = high key word
+    uint16_t* P;
+    uint32_t* Dk;
+    MP_INLINE void put(int32_t pos, uint32_t t, uint64_t key) const {
+        P[pos] = (uint16_t)t;
+        Dk[pos] = (uint32_t)(key >> 32);
     }
 };
 
@@ -400,14 +409,15 @@ MP_INLINE uint32_t r3_fine(const R3Smem& S, const R3Geo& g, uint32_t cb, uint64_
 }
 
 // stable stream of all entries with key == k (id order) to out[ob ...]
-__device__ void r3_stream_equal(const R3Keys& K, const R3Out& out, int32_t n, uint64_t k, int32_t ob, uint32_t* sc) {
+template <class Out>
+__device__ void r3_stream_equal(const R3Keys& K, const Out& out, int32_t n, uint64_t k, int32_t ob, uint32_t* sc) {
     uint32_t run = 0;
     for (int32_t b0 = 0; b0 < n; b0 += R2_THREADS) {
         const int32_t t = b0 + threadIdx.x;
         const bool sel = t < n && K.full(t) == k;
         uint32_t tot;
         const uint32_t pos = r3_scan(sel ? 1u : 0u, sc, tot);
-        if (sel) out.put(ob + (int32_t)(run + pos), (uint32_t)t);
+        if (sel) out.put(ob + (int32_t)(run + pos), (uint32_t)t, k);
         run += tot;
     }
 }
@@ -421,7 +431,8 @@ MP_INLINE bool r3_less(uint64_t ka, uint16_t va, uint64_t kb, uint16_t vb) {
 //    shared memory -- fb is read 16 entries (two 16-byte loads) per thread;
 // 2. every placed entry ranks itself inside its bin (compares against the bin's
 //    other entries) and writes straight to its final output position.
-__device__ void r3_round(const R3Keys& K, const R3Out& out, int32_t n, const R3Geo& g, uint32_t b0, uint32_t b1,
+template <class Out>
+__device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo& g, uint32_t b0, uint32_t b1,
                          uint32_t base, uint32_t cnt, int32_t ob, R3Smem& S) {
     const int32_t n16 = n & ~15;
     for (int32_t c0 = threadIdx.x * 16; c0 < n16; c0 += 16 * R2_THREADS) {
@@ -454,14 +465,15 @@ __device__ void r3_round(const R3Keys& K, const R3Out& out, int32_t n, const R3G
         const uint32_t s1 = S.starts[f] - base;
         uint32_t rank = 0;
         for (uint32_t i = s0; i < s1; i++) rank += r3_less(S.bk[i], S.bv[i], k, v) ? 1u : 0u;
-        out.put(ob + (int32_t)(s0 + rank), v);
+        out.put(ob + (int32_t)(s0 + rank), v, k);
     }
     __syncthreads();
 }
 
 MP_INLINE uint32_t r3_clog2(uint32_t x) { return x <= 1 ? 0u : 32u - __clz(x - 1); }   // ceil(log2 x)
 
-__device__ void r3_sort(const R3Keys& K, const R3Out& out, int32_t n, uint64_t kmin, uint64_t kmax, R3Smem& S) {
+template <class Out>
+__device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmin, uint64_t kmax, R3Smem& S) {
     if (n <= 0) return;
     uint32_t* stk = S.misc;                        // [R3_MAXS][6]
     uint32_t* grp = S.misc + R3_MAXS * 6;          // [R3_MAXG][3]: start fine bin, start prefix, kind
@@ -688,6 +700,33 @@ __device__ void r3_sort(const R3Keys& K, const R3Out& out, int32_t n, uint64_t k
     __syncthreads();
 }
 
+// gain keys (0x3F800000 - bits(gain)) of both archs from the orderable difference D (two archs):
+// D = 0: arch-1-only (gain_1 = 1), D = ~0: arch-0-only (gain_0 = 1), else d = delta_1 - delta_0.
+MP_INLINE void r2_gains_from_D(uint32_t D, float hd, uint32_t& G0, uint32_t& G1) {
+    if (D == 0u) {
+        G0 = 0x40000000u;
+        G1 = 0u;
+        return;
+    }
+    if (D == 0xFFFFFFFFu) {
+        G0 = 0u;
+        G1 = 0x40000000u;
+        return;
+    }
+    const uint32_t db = (D & 0x80000000u) ? (D & 0x7FFFFFFFu) : ~D;
+    const float d = u2f(db);
+    float g0, g1;
+    if (hd == 0.0f) {
+        g0 = g1 = 0.5f;
+    } else {
+        const float den = __fadd_rn(hd, hd);
+        g0 = __fdiv_rn(__fadd_rn(d, hd), den);
+        g1 = __fdiv_rn(__fadd_rn(__fsub_rn(0.0f, d), hd), den);   // d(t, 1) = delta_0 - delta_1 = -d
+    }
+    G0 = ONE_BITS - f2u(g0);
+    G1 = ONE_BITS - f2u(g1);
+}
+
 template <int A>
 __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     extern __shared__ __align__(16) unsigned char r3s[];
@@ -699,16 +738,19 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     S.clog = reinterpret_cast<uint8_t*>(S.coff + R3_NC + 64);
     S.sc = reinterpret_cast<uint32_t*>(S.clog + R3_NC + 64);
     S.misc = S.sc + 96;
-    __shared__ uint32_t s_tick, s_head;
-    __shared__ unsigned long long s_min[A], s_max[A];
+    __shared__ uint32_t s_tick, s_head, s_flag, s_h0, s_h1;
+    __shared__ unsigned long long s_min[A + 1], s_max[A + 1];
     const int64_t npad = ((int64_t)a.n + 15) & ~15ll;   // 16-entry aligned scratch rows
-    uint32_t* critc = a.s_key + (int64_t)blockIdx.x * npad * (A + 1);
+    uint32_t* critc = a.s_key + (int64_t)blockIdx.x * npad * (A + 3);
     uint32_t* gainc = critc + npad;   // [A][npad]
-    uint16_t* fbuf = a.s_pi + (int64_t)blockIdx.x * npad;
+    uint32_t* dkey = gainc + (int64_t)A * npad;
+    uint16_t* fbuf = a.s_pi + (int64_t)blockIdx.x * npad * 2;
+    uint16_t* ppos = fbuf + npad;
+    uint32_t* dsorted = dkey + npad;   // (A == 2) D in sorted order (gains are recomputed from it)
     bool bad = false;
     while (true) {
         if (threadIdx.x == 0) s_tick = atomicAdd(a.ticket, 1u);
-        if (threadIdx.x < A) {
+        if (threadIdx.x <= A) {
             s_min[threadIdx.x] = ~0ull;
             s_max[threadIdx.x] = 0ull;
         }
@@ -721,12 +763,13 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         float hdv[A];
 #pragma unroll
         for (int b = 0; b < A; b++) hdv[b] = u2f(a.hd[rl * A + b]);
-        // materialise critc and gainc_a (one hash per (t, a)); per-arch key range
-        unsigned long long mn[A], mx[A];
+        // materialise critc, gainc_a (one hash per (t, a)) and, for two archs, the
+        // orderable difference D(t) of the two durations; key ranges
+        unsigned long long mn[A + 1], mx[A + 1];
 #pragma unroll
-        for (int b = 0; b < A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
+        for (int b = 0; b <= A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
         for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
-            const float blv = a.blT[rl * a.n + t];
+            const float blv = __ldcs(a.blT + rl * a.n + t);   // read once: evict-first
             const float c = CP > 0.0f ? __fdiv_rn(blv, CP) : 0.0f;
             const uint32_t cc = ONE_BITS - f2u(c);
             critc[t] = cc;
@@ -737,6 +780,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             r2_durs<A>(a, r, t, x, en, k, wt, bad);
 #pragma unroll
             for (int b = 0; b < A; b++) {
+                if (A == 2) break;   // two archs: gains are derived from D (general path re-materialises)
                 uint32_t key = 0x40000000u;
                 if ((en >> b) & 1u) {
                     float gv;
@@ -756,9 +800,25 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 mn[b] = full < mn[b] ? full : mn[b];
                 mx[b] = full > mx[b] ? full : mx[b];
             }
+            if constexpr (A == 2) {
+                // d = delta_1 - delta_0 (= d(t, arch 0) = -d(t, arch 1), exact negation): gain_0 is
+                // non-decreasing and gain_1 non-increasing in d (RN ops are monotone), so one order by
+                // d serves both queues.  Arch-0-only tasks sort last, arch-1-only first.
+                uint32_t D;
+                if (en == 3u) {
+                    const uint32_t db = f2u(__fsub_rn(x[1], x[0]));
+                    D = (db >> 31) ? ~db : (db | 0x80000000u);
+                } else {
+                    D = en == 1u ? 0xFFFFFFFFu : 0u;
+                }
+                dkey[t] = D;
+                const unsigned long long full = ((unsigned long long)D << 32) | cc;
+                mn[A] = full < mn[A] ? full : mn[A];
+                mx[A] = full > mx[A] ? full : mx[A];
+            }
         }
 #pragma unroll
-        for (int b = 0; b < A; b++) {
+        for (int b = 0; b <= A; b++) {
             unsigned long long v1 = mn[b], v2 = mx[b];
 #pragma unroll
             for (int o = 16; o > 0; o >>= 1) {
@@ -773,6 +833,172 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             }
         }
         __syncthreads();
+        bool done = false;
+        if constexpr (A == 2) {
+            // one sort by (D, critc, t) -> P; then both queues in one pass (runs of equal gain fixed up)
+            r3_sort(R3Keys{dkey, critc, fbuf}, R3PosOut{ppos, dsorted}, a.n, s_min[A], s_max[A], S);
+            if (threadIdx.x == 0) { s_flag = 0; s_h0 = 0xffffffffu; s_h1 = 0xffffffffu; }
+            __syncthreads();
+            const int32_t cC = a.counts[rl * 2 + 0], cG = a.counts[rl * 2 + 1];
+            const int32_t n1only = a.n - cC;            // arch-1-only tasks: sorted first
+            int32_t* q0 = a.qtask ? a.qtask + rl * (int64_t)a.n * 2 : nullptr;
+            int32_t* q1 = q0 ? q0 + cC : nullptr;
+            const float h2 = hdv[0];   // hd(0) == hd(1) for two archs
+            // sorted order into shared memory (the sort's buffers are free now) + neighbour-equality
+            // bits: e0/e1 = same gain as the next position (arch 0 / arch 1), eD = same D
+            uint16_t* Ps = reinterpret_cast<uint16_t*>(S.bk);
+            const int32_t nw = (a.n + 31) / 32;
+            uint32_t* e0 = reinterpret_cast<uint32_t*>(Ps + ((a.n + 63) & ~63));
+            uint32_t* e1 = e0 + nw;
+            uint32_t* eD = e1 + nw;
+            for (int32_t i = threadIdx.x; i < a.n; i += R2_THREADS) Ps[i] = ppos[i];
+            __syncthreads();
+            {
+                const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+                for (int32_t wb = w * 32; wb < a.n; wb += R2_THREADS) {
+                    const int32_t p = wb + lane;
+                    uint32_t G0 = 0xFFFFFFFFu, G1 = 0xFFFFFFFFu, DD = 0u;
+                    if (p < a.n) {
+                        DD = __ldcg(dsorted + p);
+                        r2_gains_from_D(DD, h2, G0, G1);
+                    }
+                    uint32_t N0 = __shfl_down_sync(0xffffffffu, G0, 1);
+                    uint32_t N1 = __shfl_down_sync(0xffffffffu, G1, 1);
+                    uint32_t ND = __shfl_down_sync(0xffffffffu, DD, 1);
+                    if (lane == 31) {
+                        N0 = 0xFFFFFFFEu; N1 = 0xFFFFFFFEu; ND = ~DD;
+                        if (p + 1 < a.n) {
+                            ND = __ldcg(dsorted + p + 1);
+                            r2_gains_from_D(ND, h2, N0, N1);
+                        }
+                    }
+                    const bool ok = p + 1 < a.n;
+                    const uint32_t b0 = __ballot_sync(0xffffffffu, ok && G0 == N0);
+                    const uint32_t b1 = __ballot_sync(0xffffffffu, ok && G1 == N1);
+                    const uint32_t bD = __ballot_sync(0xffffffffu, ok && DD == ND);
+                    if (lane == 0) {
+                        e0[wb >> 5] = b0;
+                        e1[wb >> 5] = b1;
+                        eD[wb >> 5] = bD;
+                    }
+                }
+            }
+            __syncthreads();
+            auto bit = [&](const uint32_t* e, int32_t i) -> bool { return (e[i >> 5] >> (i & 31)) & 1u; };
+            for (int32_t p = threadIdx.x; p < a.n; p += R2_THREADS) {
+                const uint32_t t = Ps[p];
+                // arch 1 (forward order), positions [0, cG); p and p+1 in one run iff bit(e1, p)
+                if (p < cG) {
+                    int32_t pos = p;
+                    const bool prev = p > 0 && bit(e1, p - 1);
+                    const bool next = p + 1 < cG && bit(e1, p);
+                    if (prev || next) {
+                        int32_t lo = p, hi = p;
+                        while (lo > 0 && p - lo < 64 && bit(e1, lo - 1)) lo--;
+                        while (hi + 1 < cG && hi - p < 64 && bit(e1, hi)) hi++;
+                        if ((lo > 0 && bit(e1, lo - 1)) || (hi + 1 < cG && bit(e1, hi))) s_flag = 1;
+                        bool oneD = true;
+                        for (int32_t i = lo; i < hi; i++) oneD = oneD && bit(eD, i);
+                        if (!oneD) {
+                            const uint64_t me = ((uint64_t)__ldcg(critc + t) << 16) | t;
+                            int32_t rk = 0;
+                            for (int32_t i = lo; i <= hi; i++) {
+                                const uint32_t ti = Ps[i];
+                                rk += (((uint64_t)__ldcg(critc + ti) << 16) | ti) < me ? 1 : 0;
+                            }
+                            pos = lo + rk;
+                        }
+                    }
+                    if (pos == 0) s_h1 = t;
+                    if (q1) __stcs(q1 + pos, (int32_t)t);
+                }
+                // arch 0 (reverse order), sorted positions [n1only, n)
+                if (p >= n1only) {
+                    int32_t pos = a.n - 1 - p;
+                    const bool prev = p > n1only && bit(e0, p - 1);
+                    const bool next = p + 1 < a.n && bit(e0, p);
+                    if (prev || next) {
+                        int32_t lo = p, hi = p;
+                        while (lo > n1only && p - lo < 64 && bit(e0, lo - 1)) lo--;
+                        while (hi + 1 < a.n && hi - p < 64 && bit(e0, hi)) hi++;
+                        if ((lo > n1only && bit(e0, lo - 1)) || (hi + 1 < a.n && bit(e0, hi))) s_flag = 1;
+                        const int32_t base = a.n - 1 - hi;   // the run's block in queue 0
+                        bool oneD = true;
+                        for (int32_t i = lo; i < hi; i++) oneD = oneD && bit(eD, i);
+                        pos = base + (p - lo);               // one d value: (critc, t) ascending = forward
+                        if (!oneD) {
+                            const uint64_t me = ((uint64_t)__ldcg(critc + t) << 16) | t;
+                            int32_t rk = 0;
+                            for (int32_t i = lo; i <= hi; i++) {
+                                const uint32_t ti = Ps[i];
+                                rk += (((uint64_t)__ldcg(critc + ti) << 16) | ti) < me ? 1 : 0;
+                            }
+                            pos = base + rk;
+                        }
+                    }
+                    if (pos == 0) s_h0 = t;
+                    if (q0) __stcs(q0 + pos, (int32_t)t);
+                }
+            }
+            __syncthreads();
+            if (!s_flag) {
+                done = true;
+                if (threadIdx.x < 2) {
+                    const int b = threadIdx.x;
+                    const int32_t cnt = a.counts[rl * 2 + b];
+                    mp_queue_summary o;
+                    o.count = cnt;
+                    o.head = cnt > 0 ? (int32_t)(b == 0 ? s_h0 : s_h1) : -1;
+                    const int64_t bo = (rl * 2 + b) * 2;
+                    o.brw_lo = a.brw[bo];
+                    o.brw_hi = (int64_t)a.brw[bo + 1];
+                    o.brw = u128_to_double_scaled(a.brw[bo], a.brw[bo + 1]);
+                    a.sum[rl * 2 + b] = o;
+                }
+            }
+            __syncthreads();
+        }
+        if (done) continue;
+        if constexpr (A == 2) {
+            // fallback for this replica: materialise both archs' gain keys and ranges
+            if (threadIdx.x < A) {
+                s_min[threadIdx.x] = ~0ull;
+                s_max[threadIdx.x] = 0ull;
+            }
+            __syncthreads();
+            unsigned long long fmn[A], fmx[A];
+#pragma unroll
+            for (int b = 0; b < A; b++) { fmn[b] = ~0ull; fmx[b] = 0ull; }
+            for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
+                const uint32_t cc = critc[t];
+                uint32_t G[2];
+                r2_gains_from_D(dkey[t], hdv[0], G[0], G[1]);
+#pragma unroll
+                for (int b = 0; b < A; b++) {
+                    gainc[(int64_t)b * npad + t] = G[b];
+                    const unsigned long long full = ((unsigned long long)G[b] << 32) | cc;
+                    fmn[b] = full < fmn[b] ? full : fmn[b];
+                    fmx[b] = full > fmx[b] ? full : fmx[b];
+                }
+            }
+#pragma unroll
+            for (int b = 0; b < A; b++) {
+                unsigned long long v1 = fmn[b], v2 = fmx[b];
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    unsigned long long y1 = __shfl_xor_sync(0xffffffffu, v1, o);
+                    unsigned long long y2 = __shfl_xor_sync(0xffffffffu, v2, o);
+                    v1 = y1 < v1 ? y1 : v1;
+                    v2 = y2 > v2 ? y2 : v2;
+                }
+                if ((threadIdx.x & 31) == 0) {
+                    atomicMin(&s_min[b], v1);
+                    atomicMax(&s_max[b], v2);
+                }
+            }
+            __syncthreads();
+        }
+        // general path (A != 2, or an equal-gain run of > 64 entries spanning several d values)
         int64_t qoff = 0;
         for (int b = 0; b < A; b++) {
             const int32_t cnt = a.counts[rl * A + b];
@@ -810,7 +1036,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const int64_t groups = (R + 31) / 32;
     const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256((size_t)R * n * 4) + align256((size_t)R * A * 4) * 2 +
-                   align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 2);
+                   align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 3)) + align256((size_t)grid2 * ((n + 15) & ~15) * 4);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
     Rep2Args a{};
@@ -835,8 +1061,8 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.counts = ar.take<int32_t>((size_t)R * A);
     a.brw = ar.take<unsigned long long>((size_t)R * A * 2);
     a.err = dag->err;
-    a.s_key = ar.take<uint32_t>((size_t)grid2 * ((n + 15) & ~15) * (A + 1));
-    a.s_pi = ar.take<uint16_t>((size_t)grid2 * ((n + 15) & ~15));
+    a.s_key = ar.take<uint32_t>((size_t)grid2 * ((n + 15) & ~15) * (A + 3));
+    a.s_pi = ar.take<uint16_t>((size_t)grid2 * ((n + 15) & ~15) * 2);
     a.qtask = qtask;
     a.sum = sum;
     a.ticket = dag->tickets + 56;
