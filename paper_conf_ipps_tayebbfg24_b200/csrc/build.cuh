@@ -69,16 +69,22 @@ struct KahnArgs {
 // Light grid barrier for a co-resident (cooperative) grid: one monotonically
 // increasing arrival counter, thread 0 of each block spins with acquire loads.
 MP_INLINE void grid_barrier(unsigned* bar, unsigned& epoch) {
+    // bar[0]: arrivals (monotonic); bar[32]: release flag (its own 128-byte line).  The last
+    // block to arrive publishes the epoch; the others poll the flag, not the atomic counter.
     __syncthreads();
     epoch++;
     if (threadIdx.x == 0) {
         __threadfence();
-        atomicAdd(bar, 1u);
         const unsigned target = epoch * gridDim.x;
-        unsigned v;
-        do {
-            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
-        } while ((int)(v - target) < 0);
+        const unsigned old = atomicAdd(bar, 1u);
+        if (old + 1u == target) {
+            asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(bar + 32), "r"(epoch) : "memory");
+        } else {
+            unsigned v;
+            do {
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar + 32) : "memory");
+            } while ((int)(v - epoch) < 0);
+        }
     }
     __syncthreads();
 }
@@ -356,6 +362,7 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     ALLOC(dag->b_f1, nn);
     ALLOC(dag->b_counts, nn + 2);
     ALLOC(dag->b_kout, 4);
+    ALLOC(dag->b_bar, 64);
     int32_t* rem = dag->b_rem;
     int32_t* f0 = dag->b_f0;
     int32_t* f1 = dag->b_f1;
@@ -365,8 +372,8 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     CK(cudaMemsetAsync(kout, 0, 16, st));
     if (n > 0) {
         KahnArgs ka{n, dag->row_ptr, dag->col, dag->indeg, rem, dag->level, {f0, f1}, counts, kout, dag->err};
-        unsigned* bar = (unsigned*)(dag->tickets + 60);
-        CK(cudaMemsetAsync(bar, 0, 4, st));
+        unsigned* bar = (unsigned*)dag->b_bar;
+        CK(cudaMemsetAsync(bar, 0, 64 * 4, st));
         // small DAGs: one CTA, remaining-predecessor counters in shared memory
         const int64_t kSmemRem = 48 * 1024;
         int smem_rem = (int64_t)n <= kSmemRem ? 1 : 0;

@@ -54,6 +54,7 @@ struct mp_dag {
     int32_t* b_counts = nullptr;
     int32_t* b_kout = nullptr;
     int32_t* b_pof = nullptr;
+    int32_t* b_bar = nullptr;   // grid barrier: arrivals [0], release flag [32]
     std::map<const void*, size_t> caps;  // capacity (bytes) of every grow-only field
 };
 

@@ -273,7 +273,10 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
 // ---------------------------------------------------------------------------------------
 constexpr int R3_NC = 4096;      // coarse bins per range
 constexpr int R3_NF = 16384;     // fine bins per range (sub-bins of the coarse bins)
-constexpr int R3_CAP = 14400;    // entries per round (shared memory)
+constexpr int R3_CAP = 14400;    // entries per round with 64-bit keys (shared memory)
+constexpr int R3_RB = R3_CAP * 10;   // round buffer bytes
+template <class KT>
+__host__ __device__ constexpr int r3_cap() { return R3_RB / (int)(sizeof(KT) + 2); }   // 14400 (u64 keys) / 24000 (u32)
 constexpr int R3_TINY = 16;      // fine bins up to this size: thread insertion sort
 constexpr int R3_MID = 256;      // up to this size: warp rank sort; larger: finer range / stream
 constexpr int R3_MAXS = 192;     // range stack entries (6 words each)
@@ -283,15 +286,13 @@ struct R3Smem {
     uint32_t* starts;   // [R3_NF + 64]  fine counts -> exclusive prefixes
     uint16_t* coff;     // [R3_NC + 64]  first fine bin of each coarse bin
     uint8_t* clog;      // [R3_NC + 64]  log2(#fine bins) of each coarse bin
-    uint64_t* bk;       // [R3_CAP]
-    uint16_t* bv;       // [R3_CAP]
+    unsigned char* bkraw;  // R3_RB bytes: keys (u64 x R3_CAP or u32 x R3_CAP32) then ids (u16)
     uint32_t* sc;       // [96]
     uint32_t* misc;     // [R3_MAXS*6 + R3_MAXG*3 + 8 + 512]
 };
 
 constexpr size_t r3_smem_bytes() {
-    return (size_t)(R3_NF + 64) * 4 + (size_t)(R3_NC + 64) * 2 + (size_t)(R3_NC + 64) + (size_t)R3_CAP * 8 +
-           (size_t)R3_CAP * 2 + 96 * 4 + (size_t)(R3_MAXS * 6 + R3_MAXG * 3 + 8 + 512) * 4;
+    return (size_t)(R3_NF + 64) * 4 + (size_t)(R3_NC + 64) * 2 + (size_t)(R3_NC + 64) + (size_t)R3_RB + 96 * 4 + (size_t)(R3_MAXS * 6 + R3_MAXG * 3 + 8 + 512) * 4;
 }
 
 // exclusive block scan of one value per thread (1024 threads)
@@ -327,7 +328,9 @@ struct R3Keys {
     const uint32_t* hi;   // gainc_a[n]
     const uint32_t* lo;   // critc[n]
     uint16_t* fb;         // [n] fine bin of each entry in the current range (scratch)
-    MP_INLINE uint64_t full(int32_t t) const { return ((uint64_t)__ldcg(hi + t) << 32) | __ldcg(lo + t); }
+    MP_INLINE uint64_t full(int32_t t) const {
+        return ((uint64_t)__ldcg(hi + t) << 32) | (lo ? __ldcg(lo + t) : 0u);   // lo == null: 32-bit keys
+    }
 };
 
 struct R3Out {
@@ -368,7 +371,7 @@ MP_INLINE bool r3_locate(const R3Keys& K, int32_t t, const R3Geo& g, uint32_t ne
         cb = (uint32_t)((key >> g.cs) - g.clb);
         return true;
     }
-    key = ((uint64_t)h << 32) | __ldcg(K.lo + t);
+    key = ((uint64_t)h << 32) | (K.lo ? __ldcg(K.lo + t) : 0u);
     if (key < g.lo || key > g.hi) return false;
     cb = (uint32_t)((key >> g.cs) - g.clb);
     return true;
@@ -382,7 +385,7 @@ MP_INLINE bool r3_locate_h(const R3Keys& K, int32_t t, uint32_t h, const R3Geo& 
         cb = (uint32_t)((((uint64_t)h << 32) >> g.cs) - g.clb);
         return true;
     }
-    const uint64_t key = ((uint64_t)h << 32) | __ldcg(K.lo + t);
+    const uint64_t key = ((uint64_t)h << 32) | (K.lo ? __ldcg(K.lo + t) : 0u);
     if (key < g.lo || key > g.hi) return false;
     cb = (uint32_t)((key >> g.cs) - g.clb);
     return true;
@@ -396,7 +399,7 @@ MP_INLINE bool r3_locate_hk(const R3Keys& K, int32_t t, uint32_t h, const R3Geo&
         cb = (uint32_t)((key >> g.cs) - g.clb);
         return true;
     }
-    key = ((uint64_t)h << 32) | __ldcg(K.lo + t);
+    key = ((uint64_t)h << 32) | (K.lo ? __ldcg(K.lo + t) : 0u);
     if (key < g.lo || key > g.hi) return false;
     cb = (uint32_t)((key >> g.cs) - g.clb);
     return true;
@@ -422,18 +425,24 @@ __device__ void r3_stream_equal(const R3Keys& K, const Out& out, int32_t n, uint
     }
 }
 
-MP_INLINE bool r3_less(uint64_t ka, uint16_t va, uint64_t kb, uint16_t vb) {
+template <class KT>
+MP_INLINE bool r3_less(KT ka, uint16_t va, KT kb, uint16_t vb) {
     return ka < kb || (ka == kb && va < vb);
 }
+template <class KT>
+MP_INLINE KT r3_store_key(uint64_t k) { return sizeof(KT) == 8 ? (KT)k : (KT)(k >> 32); }
 
 // One round: fine bins [b0, b1) (each <= R3_MID entries, total cnt <= R3_CAP).
 // 1. members (fb[t] in [b0, b1)) are placed at (bin start + atomic cursor) in
 //    shared memory -- fb is read 16 entries (two 16-byte loads) per thread;
 // 2. every placed entry ranks itself inside its bin (compares against the bin's
 //    other entries) and writes straight to its final output position.
-template <class Out>
+template <class KT, class Out>
 __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo& g, uint32_t b0, uint32_t b1,
                          uint32_t base, uint32_t cnt, int32_t ob, R3Smem& S) {
+    constexpr int CAPK = r3_cap<KT>();
+    KT* bk = reinterpret_cast<KT*>(S.bkraw);
+    uint16_t* bv = reinterpret_cast<uint16_t*>(S.bkraw + (size_t)CAPK * sizeof(KT));
     const int32_t n16 = n & ~15;
     for (int32_t c0 = threadIdx.x * 16; c0 < n16; c0 += 16 * R2_THREADS) {
         const uint4 w0 = __ldcg(reinterpret_cast<const uint4*>(K.fb + c0));
@@ -445,35 +454,37 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
             if (f < b0 || f >= b1) continue;
             const int32_t t = c0 + u;
             const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
-            S.bk[slot] = K.full(t);
-            S.bv[slot] = (uint16_t)t;
+            bk[slot] = r3_store_key<KT>(K.full(t));
+            bv[slot] = (uint16_t)t;
         }
     }
     for (int32_t t = n16 + threadIdx.x; t < n; t += R2_THREADS) {
         const uint32_t f = __ldcg(K.fb + t);
         if (f < b0 || f >= b1) continue;
         const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
-        S.bk[slot] = K.full(t);
-        S.bv[slot] = (uint16_t)t;
+        bk[slot] = r3_store_key<KT>(K.full(t));
+        bv[slot] = (uint16_t)t;
     }
     __syncthreads();
     for (uint32_t j = threadIdx.x; j < cnt; j += R2_THREADS) {
-        const uint64_t k = S.bk[j];
-        const uint16_t v = S.bv[j];
-        const uint32_t f = r3_fine(S, g, (uint32_t)((k >> g.cs) - g.clb), k);
+        const KT k = bk[j];
+        const uint16_t v = bv[j];
+        const uint64_t k64 = sizeof(KT) == 8 ? (uint64_t)k : ((uint64_t)k << 32);
+        const uint32_t f = r3_fine(S, g, (uint32_t)((k64 >> g.cs) - g.clb), k64);
         const uint32_t s0 = (f == b0 ? base : S.starts[f - 1]) - base;
         const uint32_t s1 = S.starts[f] - base;
         uint32_t rank = 0;
-        for (uint32_t i = s0; i < s1; i++) rank += r3_less(S.bk[i], S.bv[i], k, v) ? 1u : 0u;
-        out.put(ob + (int32_t)(s0 + rank), v, k);
+        for (uint32_t i = s0; i < s1; i++) rank += r3_less<KT>(bk[i], bv[i], k, v) ? 1u : 0u;
+        out.put(ob + (int32_t)(s0 + rank), v, k64);
     }
     __syncthreads();
 }
 
 MP_INLINE uint32_t r3_clog2(uint32_t x) { return x <= 1 ? 0u : 32u - __clz(x - 1); }   // ceil(log2 x)
 
-template <class Out>
+template <class KT, class Out>
 __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmin, uint64_t kmax, R3Smem& S) {
+    constexpr int CAPK = r3_cap<KT>();
     if (n <= 0) return;
     uint32_t* stk = S.misc;                        // [R3_MAXS][6]
     uint32_t* grp = S.misc + R3_MAXS * 6;          // [R3_MAXG][3]: start fine bin, start prefix, kind
@@ -623,7 +634,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         __syncthreads();
         // ---- prefixes over fine bins (12 per thread) + group boundaries ----
         constexpr int PER = R3_NF / R2_THREADS;  // 12
-        const uint32_t H = R3_CAP - R3_MID;      // a multi-bin group never exceeds H + MID = CAP
+        const uint32_t H = CAPK - R3_MID;        // a multi-bin group never exceeds H + MID = CAP
         uint32_t cnts[PER], sum = 0;
 #pragma unroll
         for (int j = 0; j < PER; j++) {
@@ -673,7 +684,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
             const uint32_t cnt = e1 - e0;
             if (cnt == 0) continue;
             if (kind == 0) {
-                r3_round(K, out, n, g, b0, b1, e0, cnt, ob + (int32_t)e0, S);
+                r3_round<KT>(K, out, n, g, b0, b1, e0, cnt, ob + (int32_t)e0, S);
             } else {
                 if (threadIdx.x == 0) {
                     // key range of fine bin b0: its coarse bin c (last with coff[c] <= b0), sub-bin b0-coff[c]
@@ -732,9 +743,8 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     extern __shared__ __align__(16) unsigned char r3s[];
     R3Smem S;
     S.starts = reinterpret_cast<uint32_t*>(r3s);
-    S.bk = reinterpret_cast<uint64_t*>(r3s + (size_t)(R3_NF + 64) * 4);
-    S.bv = reinterpret_cast<uint16_t*>(S.bk + R3_CAP);
-    S.coff = reinterpret_cast<uint16_t*>(S.bv + R3_CAP);
+    S.bkraw = r3s + (size_t)(R3_NF + 64) * 4;
+    S.coff = reinterpret_cast<uint16_t*>(S.bkraw + R3_RB);
     S.clog = reinterpret_cast<uint8_t*>(S.coff + R3_NC + 64);
     S.sc = reinterpret_cast<uint32_t*>(S.clog + R3_NC + 64);
     S.misc = S.sc + 96;
@@ -836,7 +846,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         bool done = false;
         if constexpr (A == 2) {
             // one sort by (D, critc, t) -> P; then both queues in one pass (runs of equal gain fixed up)
-            r3_sort(R3Keys{dkey, critc, fbuf}, R3PosOut{ppos, dsorted}, a.n, s_min[A], s_max[A], S);
+            r3_sort<uint32_t>(R3Keys{dkey, nullptr, fbuf}, R3PosOut{ppos, dsorted}, a.n, s_min[A] & ~0xFFFFFFFFull, s_max[A] & ~0xFFFFFFFFull, S);
             if (threadIdx.x == 0) { s_flag = 0; s_h0 = 0xffffffffu; s_h1 = 0xffffffffu; }
             __syncthreads();
             const int32_t cC = a.counts[rl * 2 + 0], cG = a.counts[rl * 2 + 1];
@@ -846,7 +856,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             const float h2 = hdv[0];   // hd(0) == hd(1) for two archs
             // sorted order into shared memory (the sort's buffers are free now) + neighbour-equality
             // bits: e0/e1 = same gain as the next position (arch 0 / arch 1), eD = same D
-            uint16_t* Ps = reinterpret_cast<uint16_t*>(S.bk);
+            uint16_t* Ps = reinterpret_cast<uint16_t*>(S.bkraw);
             const int32_t nw = (a.n + 31) / 32;
             uint32_t* e0 = reinterpret_cast<uint32_t*>(Ps + ((a.n + 63) & ~63));
             uint32_t* e1 = e0 + nw;
@@ -897,9 +907,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         while (lo > 0 && p - lo < 64 && bit(e1, lo - 1)) lo--;
                         while (hi + 1 < cG && hi - p < 64 && bit(e1, hi)) hi++;
                         if ((lo > 0 && bit(e1, lo - 1)) || (hi + 1 < cG && bit(e1, hi))) s_flag = 1;
-                        bool oneD = true;
-                        for (int32_t i = lo; i < hi; i++) oneD = oneD && bit(eD, i);
-                        if (!oneD) {
+                        {   // the sort ordered the run by (d, id): rank it by (critc, id)
                             const uint64_t me = ((uint64_t)__ldcg(critc + t) << 16) | t;
                             int32_t rk = 0;
                             for (int32_t i = lo; i <= hi; i++) {
@@ -923,10 +931,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         while (hi + 1 < a.n && hi - p < 64 && bit(e0, hi)) hi++;
                         if ((lo > n1only && bit(e0, lo - 1)) || (hi + 1 < a.n && bit(e0, hi))) s_flag = 1;
                         const int32_t base = a.n - 1 - hi;   // the run's block in queue 0
-                        bool oneD = true;
-                        for (int32_t i = lo; i < hi; i++) oneD = oneD && bit(eD, i);
-                        pos = base + (p - lo);               // one d value: (critc, t) ascending = forward
-                        if (!oneD) {
+                        {   // the sort ordered the run by (d, id): rank it by (critc, id)
                             const uint64_t me = ((uint64_t)__ldcg(critc + t) << 16) | t;
                             int32_t rk = 0;
                             for (int32_t i = lo; i <= hi; i++) {
@@ -1005,7 +1010,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             if (threadIdx.x == 0) s_head = 0xffffffffu;
             __syncthreads();
             int32_t* qdst = a.qtask ? a.qtask + rl * (int64_t)a.n * A + qoff : nullptr;
-            r3_sort(R3Keys{gainc + (int64_t)b * npad, critc, fbuf}, R3Out{qdst, cnt, &s_head}, a.n, s_min[b], s_max[b], S);
+            r3_sort<uint64_t>(R3Keys{gainc + (int64_t)b * npad, critc, fbuf}, R3Out{qdst, cnt, &s_head}, a.n, s_min[b], s_max[b], S);
             __syncthreads();
             if (threadIdx.x == 0) {
                 mp_queue_summary o;
