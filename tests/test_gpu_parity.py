@@ -277,3 +277,23 @@ def test_replicas_ties_stream_path():
     """sigma = 0 on c2: 41,664 GEMMs share one gain -> key ranges with one value > 16384 entries."""
     w = workloads.config("c2")
     _replica_check(w, 40, 0, [0, 39], sigma=0.0)
+
+
+def test_replicas_two_arch_mixed_one_arch_tasks():
+    """Two archs with CPU-only tasks (sparse-QR ASM, FMM P2M/M2M/L2L/L2P): d = +-inf classes."""
+    a = workloads.sparse_tree(12, 64, 32)
+    b = workloads.fmm_tree(5, 1 << 12, 3)
+    w = workloads.union(a, b, "mixed")
+    assert w.n < 65536 and (~np.isfinite(w.dur[:, 1])).any()
+    _replica_check(w, 40, 1000, range(40))
+
+
+def test_replicas_two_arch_gpu_only_tasks_and_hd_zero():
+    w = workloads.config("c1")
+    dur = w.dur.copy()
+    dur[::3, 0] = np.inf                       # GPU-only tasks
+    W = workloads.Workload("g", w.n, w.src, w.dst, dur, w.arch_names, w.workers)
+    _replica_check(W, 64, 0, range(64))
+    eq = np.ones_like(w.dur)                   # equal durations -> d = 0, hd = 0 -> gain 0.5
+    W2 = workloads.Workload("eq", w.n, w.src, w.dst, eq, w.arch_names, w.workers)
+    _replica_check(W2, 8, 0, range(8), sigma=0.0)
