@@ -448,14 +448,32 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
         const uint4 w0 = __ldcg(reinterpret_cast<const uint4*>(K.fb + c0));
         const uint4 w1 = __ldcg(reinterpret_cast<const uint4*>(K.fb + c0 + 8));
         const uint32_t wv[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
+        if constexpr (sizeof(KT) == 4) {
+            // 32-bit keys: read them with the scan (sequential 16-byte loads) instead of gathering
+            uint32_t hv[16];
 #pragma unroll
-        for (int u = 0; u < 16; u++) {
-            const uint32_t f = (wv[u >> 1] >> ((u & 1) * 16)) & 0xFFFFu;
-            if (f < b0 || f >= b1) continue;
-            const int32_t t = c0 + u;
-            const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
-            bk[slot] = r3_store_key<KT>(K.full(t));
-            bv[slot] = (uint16_t)t;
+            for (int u4 = 0; u4 < 4; u4++) {
+                const uint4 h = __ldcg(reinterpret_cast<const uint4*>(K.hi + c0 + 4 * u4));
+                hv[4 * u4] = h.x; hv[4 * u4 + 1] = h.y; hv[4 * u4 + 2] = h.z; hv[4 * u4 + 3] = h.w;
+            }
+#pragma unroll
+            for (int u = 0; u < 16; u++) {
+                const uint32_t f = (wv[u >> 1] >> ((u & 1) * 16)) & 0xFFFFu;
+                if (f < b0 || f >= b1) continue;
+                const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
+                bk[slot] = (KT)hv[u];
+                bv[slot] = (uint16_t)(c0 + u);
+            }
+        } else {
+#pragma unroll
+            for (int u = 0; u < 16; u++) {
+                const uint32_t f = (wv[u >> 1] >> ((u & 1) * 16)) & 0xFFFFu;
+                if (f < b0 || f >= b1) continue;
+                const int32_t t = c0 + u;
+                const uint32_t slot = atomicAdd(&S.starts[f], 1u) - base;
+                bk[slot] = r3_store_key<KT>(K.full(t));
+                bv[slot] = (uint16_t)t;
+            }
         }
     }
     for (int32_t t = n16 + threadIdx.x; t < n; t += R2_THREADS) {
@@ -778,8 +796,19 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         unsigned long long mn[A + 1], mx[A + 1];
 #pragma unroll
         for (int b = 0; b <= A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
-        for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
-            const float blv = __ldcs(a.blT + rl * a.n + t);   // read once: evict-first
+        const bool vec4 = (a.n & 3) == 0;   // 16-byte loads of bl when rows stay aligned
+        for (int32_t t0 = vec4 ? threadIdx.x * 4 : threadIdx.x; t0 < a.n; t0 += vec4 ? 4 * R2_THREADS : R2_THREADS) {
+          float blq[4];
+          if (vec4) {
+              const float4 v4 = __ldcs(reinterpret_cast<const float4*>(a.blT + rl * a.n + t0));   // read once
+              blq[0] = v4.x; blq[1] = v4.y; blq[2] = v4.z; blq[3] = v4.w;
+          } else {
+              blq[0] = __ldcs(a.blT + rl * a.n + t0);
+          }
+          const int nq = vec4 ? 4 : 1;
+          for (int uq = 0; uq < nq; uq++) {
+            const int32_t t = t0 + uq;
+            const float blv = blq[uq];
             const float c = CP > 0.0f ? __fdiv_rn(blv, CP) : 0.0f;
             const uint32_t cc = ONE_BITS - f2u(c);
             critc[t] = cc;
@@ -826,6 +855,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 mn[A] = full < mn[A] ? full : mn[A];
                 mx[A] = full > mx[A] ? full : mx[A];
             }
+          }
         }
 #pragma unroll
         for (int b = 0; b <= A; b++) {
@@ -865,31 +895,41 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             __syncthreads();
             {
                 const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-                for (int32_t wb = w * 32; wb < a.n; wb += R2_THREADS) {
-                    const int32_t p = wb + lane;
-                    uint32_t G0 = 0xFFFFFFFFu, G1 = 0xFFFFFFFFu, DD = 0u;
-                    if (p < a.n) {
-                        DD = __ldcg(dsorted + p);
-                        r2_gains_from_D(DD, h2, G0, G1);
+                for (int32_t wb0 = w * 32; wb0 < a.n; wb0 += 2 * R2_THREADS) {
+                    uint32_t DDv[2], NDv[2];
+#pragma unroll
+                    for (int h = 0; h < 2; h++) {      // loads of both chunks first
+                        const int32_t p = wb0 + h * R2_THREADS + lane;
+                        DDv[h] = p < a.n ? __ldcg(dsorted + p) : 0u;
+                        NDv[h] = (lane == 31 && p + 1 < a.n) ? __ldcg(dsorted + p + 1) : 0u;
                     }
-                    uint32_t N0 = __shfl_down_sync(0xffffffffu, G0, 1);
-                    uint32_t N1 = __shfl_down_sync(0xffffffffu, G1, 1);
-                    uint32_t ND = __shfl_down_sync(0xffffffffu, DD, 1);
-                    if (lane == 31) {
-                        N0 = 0xFFFFFFFEu; N1 = 0xFFFFFFFEu; ND = ~DD;
-                        if (p + 1 < a.n) {
-                            ND = __ldcg(dsorted + p + 1);
-                            r2_gains_from_D(ND, h2, N0, N1);
+#pragma unroll
+                    for (int h = 0; h < 2; h++) {
+                        const int32_t wb = wb0 + h * R2_THREADS;
+                        if (wb >= a.n) break;
+                        const int32_t p = wb + lane;
+                        uint32_t G0 = 0xFFFFFFFFu, G1 = 0xFFFFFFFFu;
+                        const uint32_t DD = DDv[h];
+                        if (p < a.n) r2_gains_from_D(DD, h2, G0, G1);
+                        uint32_t N0 = __shfl_down_sync(0xffffffffu, G0, 1);
+                        uint32_t N1 = __shfl_down_sync(0xffffffffu, G1, 1);
+                        uint32_t ND = __shfl_down_sync(0xffffffffu, DD, 1);
+                        if (lane == 31) {
+                            N0 = 0xFFFFFFFEu; N1 = 0xFFFFFFFEu; ND = ~DD;
+                            if (p + 1 < a.n) {
+                                ND = NDv[h];
+                                r2_gains_from_D(ND, h2, N0, N1);
+                            }
                         }
-                    }
-                    const bool ok = p + 1 < a.n;
-                    const uint32_t b0 = __ballot_sync(0xffffffffu, ok && G0 == N0);
-                    const uint32_t b1 = __ballot_sync(0xffffffffu, ok && G1 == N1);
-                    const uint32_t bD = __ballot_sync(0xffffffffu, ok && DD == ND);
-                    if (lane == 0) {
-                        e0[wb >> 5] = b0;
-                        e1[wb >> 5] = b1;
-                        eD[wb >> 5] = bD;
+                        const bool ok = p + 1 < a.n;
+                        const uint32_t b0 = __ballot_sync(0xffffffffu, ok && G0 == N0);
+                        const uint32_t b1 = __ballot_sync(0xffffffffu, ok && G1 == N1);
+                        const uint32_t bD = __ballot_sync(0xffffffffu, ok && DD == ND);
+                        if (lane == 0) {
+                            e0[wb >> 5] = b0;
+                            e1[wb >> 5] = b1;
+                            eD[wb >> 5] = bD;
+                        }
                     }
                 }
             }

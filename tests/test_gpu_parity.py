@@ -297,3 +297,17 @@ def test_replicas_two_arch_gpu_only_tasks_and_hd_zero():
     eq = np.ones_like(w.dur)                   # equal durations -> d = 0, hd = 0 -> gain 0.5
     W2 = workloads.Workload("eq", w.n, w.src, w.dst, eq, w.arch_names, w.workers)
     _replica_check(W2, 8, 0, range(8), sigma=0.0)
+
+
+def test_replica_paths_agree(monkeypatch):
+    """The lanes=replicas path and the generic batched path give identical bytes."""
+    w = workloads.config("c1")
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    base = to_dev(w.dur)
+    a = mp.replicas_run(dag, base, w.workers, 99, 0.125, 7, 50)
+    mp.check(dag)
+    monkeypatch.setenv("MP_REPLICA_PATH", "v1")
+    b = mp.replicas_run(dag, base, w.workers, 99, 0.125, 7, 50)
+    mp.check(dag)
+    for x, y in zip(a, b):
+        assert np.array_equal(x.cpu().numpy(), y.cpu().numpy())
