@@ -796,8 +796,29 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         unsigned long long mn[A + 1], mx[A + 1];
 #pragma unroll
         for (int b = 0; b <= A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
+        if constexpr (A == 2) {
+            // two archs: only the orderable d is needed to sort (crit is read for equal-gain runs)
+            for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
+                float x[A];
+                uint32_t en;
+                int k;
+                float wt;
+                r2_durs<A>(a, r, t, x, en, k, wt, bad);
+                uint32_t D;
+                if (en == 3u) {
+                    const uint32_t db = f2u(__fsub_rn(x[1], x[0]));
+                    D = (db >> 31) ? ~db : (db | 0x80000000u);
+                } else {
+                    D = en == 1u ? 0xFFFFFFFFu : 0u;
+                }
+                dkey[t] = D;
+                const unsigned long long full = (unsigned long long)D << 32;
+                mn[A] = full < mn[A] ? full : mn[A];
+                mx[A] = full > mx[A] ? full : mx[A];
+            }
+        }
         const bool vec4 = (a.n & 3) == 0;   // 16-byte loads of bl when rows stay aligned
-        for (int32_t t0 = vec4 ? threadIdx.x * 4 : threadIdx.x; t0 < a.n; t0 += vec4 ? 4 * R2_THREADS : R2_THREADS) {
+        for (int32_t t0 = vec4 ? threadIdx.x * 4 : threadIdx.x; A != 2 && t0 < a.n; t0 += vec4 ? 4 * R2_THREADS : R2_THREADS) {
           float blq[4];
           if (vec4) {
               const float4 v4 = __ldcs(reinterpret_cast<const float4*>(a.blT + rl * a.n + t0));   // read once
@@ -811,7 +832,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             const float blv = blq[uq];
             const float c = CP > 0.0f ? __fdiv_rn(blv, CP) : 0.0f;
             const uint32_t cc = ONE_BITS - f2u(c);
-            critc[t] = cc;
+            if (A != 2) critc[t] = cc;   // two archs: crit is only needed for equal-gain runs (below)
             float x[A];
             uint32_t en;
             int k;
@@ -884,6 +905,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             int32_t* q0 = a.qtask ? a.qtask + rl * (int64_t)a.n * 2 : nullptr;
             int32_t* q1 = q0 ? q0 + cC : nullptr;
             const float h2 = hdv[0];   // hd(0) == hd(1) for two archs
+            const float* blr = a.blT + rl * a.n;
+            auto critc_of = [&](uint32_t t) -> uint32_t {
+                const float c = CP > 0.0f ? __fdiv_rn(__ldcg(blr + t), CP) : 0.0f;
+                return ONE_BITS - f2u(c);
+            };
             // sorted order into shared memory (the sort's buffers are free now) + neighbour-equality
             // bits: e0/e1 = same gain as the next position (arch 0 / arch 1), eD = same D
             uint16_t* Ps = reinterpret_cast<uint16_t*>(S.bkraw);
@@ -948,11 +974,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         while (hi + 1 < cG && hi - p < 64 && bit(e1, hi)) hi++;
                         if ((lo > 0 && bit(e1, lo - 1)) || (hi + 1 < cG && bit(e1, hi))) s_flag = 1;
                         {   // the sort ordered the run by (d, id): rank it by (critc, id)
-                            const uint64_t me = ((uint64_t)__ldcg(critc + t) << 16) | t;
+                            const uint64_t me = ((uint64_t)critc_of(t) << 16) | t;
                             int32_t rk = 0;
                             for (int32_t i = lo; i <= hi; i++) {
                                 const uint32_t ti = Ps[i];
-                                rk += (((uint64_t)__ldcg(critc + ti) << 16) | ti) < me ? 1 : 0;
+                                rk += (((uint64_t)critc_of(ti) << 16) | ti) < me ? 1 : 0;
                             }
                             pos = lo + rk;
                         }
@@ -972,11 +998,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         if ((lo > n1only && bit(e0, lo - 1)) || (hi + 1 < a.n && bit(e0, hi))) s_flag = 1;
                         const int32_t base = a.n - 1 - hi;   // the run's block in queue 0
                         {   // the sort ordered the run by (d, id): rank it by (critc, id)
-                            const uint64_t me = ((uint64_t)__ldcg(critc + t) << 16) | t;
+                            const uint64_t me = ((uint64_t)critc_of(t) << 16) | t;
                             int32_t rk = 0;
                             for (int32_t i = lo; i <= hi; i++) {
                                 const uint32_t ti = Ps[i];
-                                rk += (((uint64_t)__ldcg(critc + ti) << 16) | ti) < me ? 1 : 0;
+                                rk += (((uint64_t)critc_of(ti) << 16) | ti) < me ? 1 : 0;
                             }
                             pos = base + rk;
                         }
@@ -1015,7 +1041,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
 #pragma unroll
             for (int b = 0; b < A; b++) { fmn[b] = ~0ull; fmx[b] = 0ull; }
             for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
-                const uint32_t cc = critc[t];
+                const float c = CP > 0.0f ? __fdiv_rn(__ldcg(a.blT + rl * a.n + t), CP) : 0.0f;
+                const uint32_t cc = ONE_BITS - f2u(c);
+                critc[t] = cc;
                 uint32_t G[2];
                 r2_gains_from_D(dkey[t], hdv[0], G[0], G[1]);
 #pragma unroll
