@@ -133,8 +133,12 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
         const int32_t* cur = a.front[k & 1];
         int32_t* nxt = a.front[(k + 1) & 1];
         int32_t* nctr = single ? &s_cnt[(k + 1) & 1] : &a.counts[k + 1];
-        for (int64_t c0 = (int64_t)blockIdx.x * 1024; c0 < cnt; c0 += (int64_t)gridDim.x * 1024) {
-            const int64_t i = c0 + threadIdx.x;
+        // chunk = frontier nodes per block: spread a level over all blocks (so each thread
+        // relaxes ~1 edge) but never more than one node per thread
+        int64_t chunk = (cnt + gridDim.x - 1) / gridDim.x;
+        chunk = chunk < 32 ? 32 : (chunk > 1024 ? 1024 : ((chunk + 31) & ~31ll));
+        for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < cnt; c0 += (int64_t)gridDim.x * chunk) {
+            const int64_t i = threadIdx.x < chunk ? c0 + threadIdx.x : cnt;
             int32_t deg = 0;
             if (i < cnt) {
                 const int32_t u = cur[i];
@@ -165,7 +169,7 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
             __syncthreads();
             s_pre[threadIdx.x] = (int32_t)s_sc[w] + incl - deg;
             const int32_t etot = (int32_t)s_sc[32];
-            const int32_t nloc = (int32_t)((cnt - c0) < 1024 ? (cnt - c0) : 1024);
+            const int32_t nloc = (int32_t)((cnt - c0) < chunk ? (cnt - c0) : chunk);
             __syncthreads();
             for (int32_t e = threadIdx.x; e < etot; e += blockDim.x) {
                 int lo = 0, hi = nloc - 1;     // last frontier slot with s_pre <= e
