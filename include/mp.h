@@ -186,6 +186,30 @@ mp_status mp_replicas_run(mp_dag* dag, int32_t n_arch, const float* d_base_dur,
                           int64_t r0, int32_t R, float* d_cp, mp_queue_summary* d_sum,
                           int32_t* d_qtask, void* stream);
 
+/*
+ * incremental READY-mode PUSH (the paper's dynamic setting,
+ * P:l.91 "a ready task is a task for which all dependencies are released",
+ * Alg. 1 PUSH at batch granularity).
+ * mp_ready_init: d_rem[t] = |lambda^-(t)| (predecessors not completed yet).
+ * mp_queues_push: given the current queues (d_qptr_in/d_qtask_in, e.g. from
+ * mp_build_queues with d_done = all-zero, i.e. the sources) and a batch of
+ * m completed tasks (d_batch, int32[m]; each was ready and is completed once),
+ *   - removes the batch's tasks from every queue (they were popped, Alg. 2),
+ *   - decrements d_rem of their successors; successors reaching 0 are newly
+ *     ready and join every queue whose arch can run them (P:l.104),
+ *   - writes the merged queues to d_qptr_out/d_qtask_out (capacity n*A; must
+ *     not alias the input), still sorted by (key asc, id asc), and summaries.
+ * Invariant (tested): after pushing batches B1..Bk the queues equal
+ * mp_build_queues in READY mode with done = B1 U .. U Bk.  d_key/d_flags/d_dur
+ * are the whole-DAG scores of mp_score/mp_affinity (reading c18).
+ * A task completed twice or an id outside [0,n) raises MP_ERR_ARG (mp_check).
+ */
+mp_status mp_ready_init(mp_dag* dag, int32_t* d_rem, void* stream);
+mp_status mp_queues_push(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, const uint8_t* d_flags,
+                         const float* d_dur, const int32_t* d_batch, int32_t m, int32_t* d_rem,
+                         const int64_t* d_qptr_in, const int32_t* d_qtask_in, int64_t* d_qptr_out,
+                         int32_t* d_qtask_out, mp_queue_summary* d_sum, void* stream);
+
 /* Synchronise `stream`, then return (and clear) the handle's device error
  * flag: MP_OK or MP_ERR_DOMAIN; MP_ERR_CUDA on a pending CUDA error. */
 mp_status mp_check(mp_dag* dag, void* stream);

@@ -221,6 +221,32 @@ def replicas_run(dag: Dag, base_dur: torch.Tensor, workers, seed: int, sigma: fl
     return out["cp"], out["summary"], out.get("qtask")
 
 
+def ready_init(dag: Dag, rem: torch.Tensor = None) -> torch.Tensor:
+    """mp_ready_init: per-task count of predecessors not completed yet (int32[n])."""
+    if rem is None:
+        rem = torch.empty(max(dag.n, 1), dtype=torch.int32, device=dag.device)
+    _lib.check(_lib.lib().mp_ready_init(dag.handle, _ptr(rem), _stream()), "mp_ready_init")
+    return rem
+
+
+def queues_push(dag: Dag, key: torch.Tensor, flags: torch.Tensor, dur: torch.Tensor, batch: torch.Tensor,
+                rem: torch.Tensor, qptr_in: torch.Tensor, qtask_in: torch.Tensor, out=None):
+    """mp_queues_push (N1): pop+complete `batch`, push the newly ready tasks -> (qptr, qtask, summary)."""
+    n, A = key.shape
+    dev = key.device
+    batch = batch.to(torch.int32).contiguous()
+    if out is None:
+        out = dict(qptr=torch.empty(A + 1, dtype=torch.int64, device=dev),
+                   qtask=torch.empty(max(n * A, 1), dtype=torch.int32, device=dev),
+                   summary=torch.empty(A * SUMMARY_BYTES, dtype=torch.uint8, device=dev))
+    m = batch.numel()
+    rc = _lib.lib().mp_queues_push(dag.handle, A, _ptr(key), _ptr(flags), _ptr(dur), _ptr(batch) if m else None, m,
+                                   _ptr(rem), _ptr(qptr_in), _ptr(qtask_in), _ptr(out["qptr"]), _ptr(out["qtask"]),
+                                   _ptr(out["summary"]), _stream())
+    _lib.check(rc, "mp_queues_push")
+    return out["qptr"], out["qtask"], out["summary"]
+
+
 def summaries(summary_bytes: torch.Tensor) -> np.ndarray:
     """Host view of mp_queue_summary records."""
     return summary_bytes.detach().cpu().numpy().view(SUMMARY_DTYPE)

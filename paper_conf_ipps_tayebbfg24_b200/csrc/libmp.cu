@@ -4,6 +4,7 @@
 #include <cstdarg>
 #include <vector>
 
+#include "push.cuh"
 #include "rep2.cuh"
 
 static inline cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
@@ -62,6 +63,18 @@ mp_status mp_replicas_run(mp_dag* dag, int32_t n_arch, const float* d_base_dur, 
                           int32_t* d_qtask, void* stream) {
     return mph::replicas_run(dag, n_arch, d_base_dur, h_workers, seed, sigma, r0, R, d_cp, d_sum, d_qtask,
                              as_stream(stream));
+}
+
+mp_status mp_ready_init(mp_dag* dag, int32_t* d_rem, void* stream) {
+    return mph::ready_init(dag, d_rem, as_stream(stream));
+}
+
+mp_status mp_queues_push(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, const uint8_t* d_flags,
+                         const float* d_dur, const int32_t* d_batch, int32_t m, int32_t* d_rem,
+                         const int64_t* d_qptr_in, const int32_t* d_qtask_in, int64_t* d_qptr_out,
+                         int32_t* d_qtask_out, mp_queue_summary* d_sum, void* stream) {
+    return mph::queues_push(dag, n_arch, d_key, d_flags, d_dur, d_batch, m, d_rem, d_qptr_in, d_qtask_in, d_qptr_out,
+                            d_qtask_out, d_sum, as_stream(stream));
 }
 
 mp_status mp_check(mp_dag* dag, void* stream) {

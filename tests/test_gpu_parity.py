@@ -311,3 +311,38 @@ def test_replica_paths_agree(monkeypatch):
     mp.check(dag)
     for x, y in zip(a, b):
         assert np.array_equal(x.cpu().numpy(), y.cpu().numpy())
+
+
+# ----------------------------------------------------------------------------
+# N1: incremental READY-mode push
+# ----------------------------------------------------------------------------
+
+@pytest.mark.parametrize("name,A,steps", [("c1", 2, 12), ("c2", 2, 25), ("qr", 3, 20)])
+def test_ready_push_sequence_equals_ready_rebuild(name, A, steps):
+    w = workloads.qr(10) if name == "qr" else workloads.config(name)
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    dur = to_dev(w.dur)
+    full = mp.score_and_queue(dag, dur, w.workers)
+    key, flags = full["key"], full["flags"]
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    okey = key.cpu().numpy().view(np.uint64)
+    oflags = flags.cpu().numpy()
+    done = np.zeros(w.n, np.uint8)
+    qptr, qtask, summ = mp.build_queues(dag, key, flags, dur, done=to_dev(done))
+    rem = mp.ready_init(dag)
+    rng = np.random.default_rng(3)
+    for step in range(steps):
+        qp = qptr.cpu().numpy()
+        qt = qtask.cpu().numpy()
+        ready = np.unique(qt[:qp[-1]])
+        if len(ready) == 0:
+            break
+        k = int(rng.integers(1, min(len(ready), 200) + 1))
+        batch = rng.choice(ready, k, replace=False).astype(np.int32)
+        done[batch] = 1
+        qptr, qtask, summ = mp.queues_push(dag, key, flags, dur, to_dev(batch), rem, qptr, qtask)
+        mp.check(dag)
+        oq_ptr, oq, osum = oracle.build_queues(od, okey, oflags, w.dur, done)
+        assert np.array_equal(qptr.cpu().numpy(), oq_ptr), step
+        assert np.array_equal(qtask.cpu().numpy()[:oq_ptr[-1]], oq), step
+        assert summ.cpu().numpy().tobytes() == osum.tobytes(), step
