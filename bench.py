@@ -43,6 +43,8 @@ CONFIG_TEXT = {
     "c3": "tiled QR DAG 128x128 tiles (707,264 tasks), 3 resource types",
     "c4": "sparse-QR-like elimination-tree DAG + FMM octree DAG (depth 8), 2,156,466 tasks, skewed fan-in",
     "c5": "4096 duration-perturbed replicas of the 64x64 Cholesky DAG sharded across 1/2/4/8 B200",
+    "c2push": "N1 incremental READY-mode push over the whole schedule of the 64x64 Cholesky DAG "
+              "(each step: sources, then one mp_queues_push per completion batch = every ready task)",
 }
 L2_FLUSH_BYTES = 256 << 20
 KERNELS = ("k_rep_main", "k_rep_out", "k_sort_pass", "k_sort_hist", "k_sort_plan", "k_kahn", "k_pack_edges",
@@ -58,7 +60,7 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5"))
+    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c2push"))
     p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -237,7 +239,7 @@ def run_ours(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     cfg = args.config
-    w = workloads.config("c2" if cfg == "c5" else cfg)
+    w = workloads.config("c2" if cfg in ("c5", "c2push") else cfg)
     A = w.n_arch
     n = w.n
     src_h = torch.from_numpy(w.src).pin_memory()
@@ -272,6 +274,32 @@ def run_ours(args):
             else:
                 gathered.copy_(local_rec)
             return gathered
+    elif cfg == "c2push":
+        R, cnt = 1, 1
+        tasks_per_step = n
+        full = mp.score_and_queue(dag, dur_d, w.workers)
+        key_d, flags_d = full["key"], full["flags"]
+        zeros = torch.zeros(n, dtype=torch.uint8, device=dev)
+        rem = torch.empty(n, dtype=torch.int32, device=dev)
+        bufs = [dict(qptr=torch.empty(A + 1, dtype=torch.int64, device=dev),
+                     qtask=torch.empty(n * A, dtype=torch.int32, device=dev),
+                     summary=torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev)) for _ in range(2)]
+        qhost = torch.empty(A + 1, dtype=torch.int64).pin_memory()
+        result_h = torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8).pin_memory()
+
+        def step():
+            mp.build_queues(dag, key_d, flags_d, dur_d, done=zeros, out=bufs[0])
+            mp.ready_init(dag, rem)
+            cur = 0
+            while True:
+                qhost.copy_(bufs[cur]["qptr"])          # the scheduler reads the ready count
+                m = int(qhost[1] - qhost[0])            # every task runs on arch 0: queue 0 = ready set
+                if m == 0:
+                    return bufs[cur]["summary"]
+                batch = bufs[cur]["qtask"][:m]
+                mp.queues_push(dag, key_d, flags_d, dur_d, batch, rem, bufs[cur]["qptr"], bufs[cur]["qtask"],
+                               out=bufs[cur ^ 1])
+                cur ^= 1
     else:
         R, cnt = 1, 1
         outs = {}
@@ -421,8 +449,10 @@ def run_ours(args):
                        "ms_per_dag": ms_per_step / (R if cfg == "c5" else 1) * world if cfg == "c5" else ms_per_step,
                        "l2": f"flushed between timed steps ({L2_FLUSH_BYTES >> 20} MiB write)",
                        "queues": "materialised in HBM for every replica" if cfg == "c5" else "materialised",
-                       "step": "mp_dag_rebuild + mp_replicas_run + allgather(records)" if cfg == "c5"
-                       else "mp_dag_rebuild + bottom_level + affinity + score + build_queues",
+                       "step": ("mp_dag_rebuild + mp_replicas_run + allgather(records)" if cfg == "c5" else
+                                "mp_build_queues(sources) + mp_queues_push per completion batch (scores precomputed)"
+                                if cfg == "c2push" else
+                                "mp_dag_rebuild + bottom_level + affinity + score + build_queues"),
                        "parallelism": f"replica shards x{world}" if cfg == "c5" else "single DAG"},
             "ms_per_dag": ms_per_step / (R / world) if cfg == "c5" else ms_per_step,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
