@@ -541,10 +541,11 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         }
         const uint64_t span = g.hi - g.lo;
         const uint32_t bits = 64u - (uint32_t)__clzll((long long)span);
-        g.cs = bits > 12 ? bits - 12 : 0;
+        constexpr uint32_t LOGNC = 31u - __builtin_clz((unsigned)R3_NC);   // NC is a power of two
+        g.cs = bits > LOGNC ? bits - LOGNC : 0;
         g.clb = g.lo >> g.cs;
         g.ncb = (uint32_t)((g.hi >> g.cs) - g.clb + 1);
-        if (g.ncb > (uint32_t)R3_NC) {
+        while (g.ncb > (uint32_t)R3_NC) {
             g.cs++;
             g.clb = g.lo >> g.cs;
             g.ncb = (uint32_t)((g.hi >> g.cs) - g.clb + 1);
