@@ -61,7 +61,11 @@ def parse():
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
     p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c2push"))
-    p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS)
+    p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS,
+                   help="c5: replicas per GPU (weak scaling, default) or in total (--scaling strong)")
+    p.add_argument("--scaling", choices=("weak", "strong"), default="weak",
+                   help="c5 sharding: weak = every rank scores its own block of --replicas replicas "
+                        "(global ids rank*R..), strong = --replicas in total split across ranks")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-budget-s", type=float, default=12.0)
@@ -253,7 +257,8 @@ def run_ours(args):
     stream = torch.cuda.current_stream()
 
     if cfg == "c5":
-        R = args.replicas
+        # replicas are independent problems keyed by their GLOBAL id (world-size invariant results)
+        R = args.replicas * world if args.scaling == "weak" else args.replicas
         r0, cnt = mpd.shard_range(R, world, rank)
         slots = mpd.shard_range(R, world, 0)[1]
         rb = mpd.record_bytes(A)
@@ -441,9 +446,12 @@ def run_ours(args):
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": "strong" if cfg == "c5" else "none", "vs_baseline": None, "dtype": "f32",
+            "scaling": args.scaling if cfg == "c5" else "none", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic",
-            "config": {"workload": CONFIG_TEXT[cfg], "name": cfg, "tasks_per_dag": n, "edges": E,
+            "config": {"workload": (CONFIG_TEXT[cfg] if cfg != "c5" else
+                                    f"{R} duration-perturbed replicas of the 64x64 Cholesky DAG ({cnt} per GPU, "
+                                    f"{args.scaling} scaling; BASELINE config 5 = 4096 in total = --scaling strong)"),
+                       "name": cfg, "tasks_per_dag": n, "edges": E,
                        "levels": dag.n_levels, "archs": A,
                        "replicas": R if cfg == "c5" else 1, "replicas_per_gpu": cnt,
                        "ms_per_dag": ms_per_step / (R if cfg == "c5" else 1) * world if cfg == "c5" else ms_per_step,

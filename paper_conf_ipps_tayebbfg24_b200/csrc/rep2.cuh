@@ -78,10 +78,20 @@ MP_INLINE void r2_durs(const Rep2Args& a, int64_t r, int32_t t, float (&x)[A], u
 // K1
 // ---------------------------------------------------------------------------------------
 template <int A>
+// A 32-replica group is run by a cluster of `cs` CTAs (cs = 1 when there are enough
+// groups to fill the GPU; up to 8 for small per-GPU replica counts): the nodes of a
+// level are spread over the cluster's warps and levels are separated by cluster
+// barriers (release/acquire at cluster scope, bl32 lines are written once and only
+// read after).
 __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
     extern __shared__ __align__(16) unsigned char r2_smem[];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int64_t g = blockIdx.x;
+    const int lane = threadIdx.x & 31, w0 = threadIdx.x >> 5;
+    cg::cluster_group cluster = cg::this_cluster();
+    const int cs = (int)cluster.num_blocks();
+    const int crank = (int)cluster.block_rank();
+    const int w = crank * R2_WARPS + w0;            // warp index within the group
+    const int WG = cs * R2_WARPS;                   // warps per group
+    const int64_t g = blockIdx.x / cs;
     const int64_t rl = g * 32 + lane;            // replica index within this call
     const bool live = rl < a.R;
     const int64_t r = a.r0 + rl;                 // global replica id
@@ -106,7 +116,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
             sv = lane < e1 - e0 ? __ldg(a.colq + e0 + lane) : 0;
         }
         while (q < q1) {
-            const int32_t qn = q + R2_WARPS;
+            const int32_t qn = q + WG;
             int32_t vn = 0, e0n = 0, e1n = 0, svn = 0;
             if (qn < q1) {
                 vn = __ldg(a.nodeq + qn);
@@ -167,25 +177,26 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
             e1 = e1n;
             sv = svn;
         }
-        __syncthreads();
+        if (cs == 1) __syncthreads();
+        else cluster.sync();
     }
     // ---- per-replica reductions across the 32 warps (column = lane = replica) ----
     uint32_t* red = reinterpret_cast<uint32_t*>(r2_smem);                 // [32][33]
     unsigned long long* red64 = reinterpret_cast<unsigned long long*>(r2_smem + 32 * 33 * 4 + 64);  // [32][33]
     auto colmax = [&](uint32_t val) -> uint32_t {
-        red[w * 33 + lane] = val;
+        red[w0 * 33 + lane] = val;
         __syncthreads();
         uint32_t m = 0;
-        if (w == 0)
+        if (w0 == 0)
             for (int i = 0; i < 32; i++) m = max(m, red[i * 33 + lane]);
         __syncthreads();
         return m;
     };
     auto colsum = [&](uint32_t val) -> uint32_t {
-        red[w * 33 + lane] = val;
+        red[w0 * 33 + lane] = val;
         __syncthreads();
         uint32_t m = 0;
-        if (w == 0)
+        if (w0 == 0)
             for (int i = 0; i < 32; i++) m += red[i * 33 + lane];
         __syncthreads();
         return m;
@@ -198,45 +209,42 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
         hdb[q] = colmax(hd[q]);
         cntb[q] = (int32_t)colsum((uint32_t)cnt[q]);
     }
-    // exact 128-bit column sums: lo words (counting carries), then hi words
+    // exact 128-bit column sums: lo words (counting carries), then hi words; CTAs of a
+    // cluster merge their partial statistics with atomics (zeroed by the host)
 #pragma unroll
     for (int q = 0; q < A; q++) {
-        red64[w * 33 + lane] = blo[q];
+        red64[w0 * 33 + lane] = blo[q];
         __syncthreads();
         uint64_t lo = 0, carry = 0;
-        if (w == 0)
+        if (w0 == 0)
             for (int i = 0; i < 32; i++) {
                 const uint64_t s2 = lo + red64[i * 33 + lane];
                 carry += (s2 < lo) ? 1ull : 0ull;
                 lo = s2;
             }
         __syncthreads();
-        red64[w * 33 + lane] = bhi[q];
+        red64[w0 * 33 + lane] = bhi[q];
         __syncthreads();
-        if (w == 0) {
+        if (w0 == 0) {
             uint64_t hi = carry;
             for (int i = 0; i < 32; i++) hi += red64[i * 33 + lane];
-            if (live) {
-                const int64_t o = (rl * A + q) * 2;
-                a.brw[o] = lo;
-                a.brw[o + 1] = hi;
-            }
+            if (live) atomic_add128(a.brw + (rl * A + q) * 2, lo, hi);
         }
         __syncthreads();
     }
-    if (w == 0 && live) {
-        a.cp[rl] = u2f(cpb);
+    if (w0 == 0 && live) {
+        atomicMax(reinterpret_cast<uint32_t*>(a.cp) + rl, cpb);
 #pragma unroll
         for (int q = 0; q < A; q++) {
-            a.hd[rl * A + q] = hdb[q];
-            a.counts[rl * A + q] = cntb[q];
+            atomicMax(&a.hd[rl * A + q], hdb[q]);
+            atomicAdd(&a.counts[rl * A + q], cntb[q]);
         }
     }
     if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(a.err, ERR_DOMAIN_BIT);
     // ---- transpose bl32 [q][32] -> blT [r][t] ----
-    float* tile = reinterpret_cast<float*>(r2_smem) + w * 32 * 33;
+    float* tile = reinterpret_cast<float*>(r2_smem) + w0 * 32 * 33;
     const int32_t nchunks = (a.n + 31) / 32;
-    for (int32_t c = w; c < nchunks; c += R2_WARPS) {
+    for (int32_t c = w; c < nchunks; c += WG) {
         const int32_t t0 = c * 32;
         for (int i = 0; i < 32; i++) {
             const int32_t t = t0 + i;
@@ -1154,7 +1162,36 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         MP_CUDA(cudaFuncSetAttribute(k_rep2_sort<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2));
         attr = true;
     }
-    MP_LAUNCH(k_rep2_bl<A>, (unsigned)groups, R2_THREADS, smem1, st, a);
+    // statistics are merged with atomics: zero them (and CP) first
+    MP_CUDA(cudaMemsetAsync(cp, 0, (size_t)R * 4, st));
+    MP_CUDA(cudaMemsetAsync(a.hd, 0, (size_t)R * A * 4, st));
+    MP_CUDA(cudaMemsetAsync(a.counts, 0, (size_t)R * A * 4, st));
+    MP_CUDA(cudaMemsetAsync(a.brw, 0, (size_t)R * A * 16, st));
+    // cluster size: enough CTAs per 32-replica group to cover the SMs (strong scaling keeps K1 short)
+    int cs = 1;
+    while (cs < 4 && groups * (cs * 2) <= dag->num_sms) cs *= 2;   // 8-CTA clusters measured slower
+    for (;; cs /= 2) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)(groups * cs));
+        cfg.blockDim = dim3(R2_THREADS);
+        cfg.dynamicSmemBytes = (size_t)smem1;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = (unsigned)cs;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cudaError_t e;
+        {
+            mph::ProfScope ps("k_rep2_bl<A>", st);
+            e = cudaLaunchKernelEx(&cfg, k_rep2_bl<A>, a);
+        }
+        if (e == cudaSuccess) break;
+        cudaGetLastError();
+        if (cs == 1) return fail(MP_ERR_CUDA, "k_rep2_bl launch: %s", cudaGetErrorString(e));
+    }
     MP_CUDA(cudaMemsetAsync(a.ticket, 0, 4, st));
     MP_LAUNCH(k_rep2_sort<A>, (unsigned)grid2, R2_THREADS, smem2, st, a);
     MP_CUDA(cudaGetLastError());
