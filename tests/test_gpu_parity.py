@@ -346,3 +346,32 @@ def test_ready_push_sequence_equals_ready_rebuild(name, A, steps):
         assert np.array_equal(qptr.cpu().numpy(), oq_ptr), step
         assert np.array_equal(qtask.cpu().numpy()[:oq_ptr[-1]], oq), step
         assert summ.cpu().numpy().tobytes() == osum.tobytes(), step
+
+
+# ----------------------------------------------------------------------------
+# randomised sweep: many small DAGs, 1-4 archs, masks, ties, duplicates, both criticalities
+# ----------------------------------------------------------------------------
+
+def test_random_sweep_single_dag_and_replicas():
+    rng = np.random.default_rng(2024)
+    for case in range(40):
+        n = int(rng.integers(1, 3000))
+        A = int(rng.integers(1, 5))
+        src, dst = random_dags.random_dag(n, float(rng.uniform(0.0, 4.0)), case, dup=float(rng.uniform(0, 0.5)),
+                                          max_span=int(rng.integers(1, 200)))
+        dur = random_dags.dyadic_durations(n, A, case, p_inf=float(rng.uniform(0, 0.5)) if A > 1 else 0.0,
+                                           tiny_set=bool(rng.integers(0, 2)))
+        if rng.random() < 0.2:
+            dur[rng.random((n, A)) < 0.1] = 0.0
+            dur[np.all(~np.isfinite(dur), 1)] = 1.0
+        workers = np.ones(A, np.int32)
+        if A > 1 and rng.random() < 0.2:
+            workers[int(rng.integers(0, A))] = 0
+            en = np.isfinite(dur) & (workers[None, :] > 0)
+            dur[~en.any(1), int(np.argmax(workers))] = 2.0
+        kind = oracle.CRIT_NOD if rng.random() < 0.3 else oracle.CRIT_BL
+        compare(n, src, dst, dur, workers, kind=kind)
+        W = workloads.Workload(f"r{case}", n, src, dst, dur, tuple(f"a{i}" for i in range(A)), workers)
+        R = int(rng.integers(1, 70))
+        _replica_check(W, R, int(rng.integers(0, 10000)), sorted(set([0, R - 1, R // 2])),
+                       sigma=float(rng.choice([0.0, 0.0625, 0.125, 0.25])), seed=int(rng.integers(0, 2**62)))
