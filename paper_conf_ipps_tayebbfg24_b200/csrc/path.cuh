@@ -413,6 +413,9 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
         int bps = 0;
         MP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_bl_flow, FLOW_THREADS, 0));
         int32_t nchunks = dag->P / 32;
+        // 4 blocks (32 warps) per SM: fewer spinning warps measured faster on c4 than full occupancy
+        static const int flow_bps = getenv("MP_FLOW_BPS") ? atoi(getenv("MP_FLOW_BPS")) : 4;
+        if (flow_bps > 0 && flow_bps < bps) bps = flow_bps;
         int64_t g = (int64_t)bps * dag->num_sms;
         int64_t want = ((int64_t)nchunks + FLOW_THREADS / 32 - 1) / (FLOW_THREADS / 32);
         if (want < g) g = want;
