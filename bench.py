@@ -47,8 +47,8 @@ CONFIG_TEXT = {
               "(each step: sources, then one mp_queues_push per completion batch = every ready task)",
 }
 L2_FLUSH_BYTES = 256 << 20
-KERNELS = ("k_rep_main", "k_rep_out", "k_sort_pass", "k_sort_hist", "k_sort_plan", "k_kahn", "k_pack_edges",
-           "k_dedup_flags", "k_compact_edges", "k_scan_excl", "k_iota_level_keys", "k_level_order", "k_qmaps",
+KERNELS = ("k_rep_main", "k_rep_out", "k_sort_pass", "k_sort_hist", "k_sort_plan", "k_kahn", "k_csr_count",
+           "k_csr_fill", "k_csr_rowsort", "k_csr_emit", "k_scan_excl", "k_iota_level_keys", "k_level_order", "k_qmaps",
            "k_qcols", "k_bl_small", "k_bl_flow", "k_aff_hd", "k_aff_gain", "k_crit_max", "k_score",
            "k_q_member", "k_q_scatter", "k_copy_len", "k_q_out", "k_blocked", "k_nod_indeg", "k_nod_sum",
            "k_perturb")

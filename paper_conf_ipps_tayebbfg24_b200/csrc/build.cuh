@@ -13,43 +13,246 @@ namespace cg = cooperative_groups;
 
 namespace mpk {
 
-// validate and pack (src, dst) into sortable keys src << b | dst
-__global__ void k_pack_edges(const int32_t* src, const int32_t* dst, int64_t m, int32_t n, int b,
-                             uint64_t* keys, uint32_t* err) {
-    int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+// ---- a1: counting-sort CSR ingest ------------------------------------------------------
+// Edges are bucketed by source (count -> scan -> fill), then every row is sorted and
+// deduplicated by one warp in registers; rows longer than CSR_WARP_MAX go through the
+// radix sorter instead.  The result is the deduplicated successor CSR with each row
+// ascending (the canonical order every later step relies on).
+constexpr int CSR_WARP_K = 8;                    // elements per lane
+constexpr int CSR_WARP_MAX = 32 * CSR_WARP_K;    // longest row a warp sorts (256)
+
+// warp-aggregated validation + out-degree count.  Invalid edges set ERR_ARG_BIT and are
+// dropped (the build then fails).
+__global__ void k_csr_count(const int32_t* src, const int32_t* dst, int64_t m, int32_t n, int32_t* cnt,
+                            uint32_t* err) {
+    const int lane = threadIdx.x & 31;
+    const int64_t wstride = (int64_t)gridDim.x * blockDim.x;
     bool bad = false;
-    for (; i < m; i += (int64_t)gridDim.x * blockDim.x) {
-        int32_t u = src[i], v = dst[i];
-        if (u < 0 || u >= n || v < 0 || v >= n || u == v) {
-            bad = true;
-            keys[i] = 0;
-        } else {
-            keys[i] = ((uint64_t)(uint32_t)u << b) | (uint32_t)v;
+    for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < m; base += wstride) {
+        int64_t i = base + lane;
+        int32_t u = -1;
+        if (i < m) {
+            int32_t uu = src[i], v = dst[i];
+            if (uu < 0 || uu >= n || v < 0 || v >= n || uu == v) bad = true;
+            else u = uu;
+        }
+        unsigned peers = __match_any_sync(0xffffffffu, u);
+        int leader = __ffs(peers) - 1;
+        if (u >= 0 && lane == leader) atomicAdd(&cnt[u], __popc(peers));
+    }
+    if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(err, ERR_ARG_BIT);
+}
+
+// scatter dst into its source's bucket: rs = exclusive scan of the counts; cnt counts down
+// to 0 (order inside a bucket is arbitrary, the row sort makes it canonical).
+__global__ void k_csr_fill(const int32_t* src, const int32_t* dst, int64_t m, int32_t n, const int32_t* rs,
+                           int32_t* cnt, int32_t* tmp) {
+    const int lane = threadIdx.x & 31;
+    const int64_t wstride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < m; base += wstride) {
+        int64_t i = base + lane;
+        int32_t u = -1, v = 0;
+        if (i < m) {
+            int32_t uu = src[i];
+            v = dst[i];
+            if (!(uu < 0 || uu >= n || v < 0 || v >= n || uu == v)) u = uu;
+        }
+        unsigned peers = __match_any_sync(0xffffffffu, u);
+        int leader = __ffs(peers) - 1;
+        int k = __popc(peers);
+        int old = 0;
+        if (u >= 0 && lane == leader) old = atomicSub(&cnt[u], k);
+        old = __shfl_sync(0xffffffffu, old, leader);
+        if (u >= 0) tmp[rs[u] + old - k + __popc(peers & lanemask_lt())] = v;
+    }
+}
+
+// one warp, one row of L <= 32*K entries: rank sort in registers (ties by slot) into a
+// shared-memory run, then dedup + compaction straight to srt.  Returns the unique count.
+template <int K>
+__device__ __forceinline__ int csr_row_sort(const int32_t* in, int32_t L, int32_t* run, int32_t* out, int lane) {
+    int32_t e[K];
+    int rank[K];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        int j = k * 32 + lane;
+        e[k] = j < L ? in[j] : 0x7fffffff;
+        rank[k] = 0;
+    }
+#pragma unroll
+    for (int kk = 0; kk < K; kk++) {
+        const int lim = min(32, L - kk * 32);
+        for (int l = 0; l < lim; l++) {
+            const int32_t y = __shfl_sync(0xffffffffu, e[kk], l);
+#pragma unroll
+            for (int k = 0; k < K; k++)
+                rank[k] += (y < e[k] || (y == e[k] && (kk < k || (kk == k && l < lane)))) ? 1 : 0;
         }
     }
-    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(err, ERR_ARG_BIT);
+#pragma unroll
+    for (int k = 0; k < K; k++)
+        if (k * 32 + lane < L) run[rank[k]] = e[k];
+    __syncwarp();
+    int cnt = 0;
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        const int j = k * 32 + lane;
+        int32_t x = 0;
+        bool keep = false;
+        if (j < L) {
+            x = run[j];
+            keep = (j == 0) || run[j - 1] != x;
+        }
+        unsigned bm = __ballot_sync(0xffffffffu, keep);
+        if (keep) out[cnt + __popc(bm & lanemask_lt())] = x;
+        cnt += __popc(bm);
+    }
+    __syncwarp();
+    return cnt;
 }
 
-__global__ void k_dedup_flags(const SortPlan* plan, uint64_t* const* kb, int64_t m, int32_t* flag) {
-    const uint64_t* k = kb[plan->final_sel];
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
-        flag[i] = (i == 0 || k[i] != k[i - 1]) ? 1 : 0;
+// one warp, one row of 32 < L <= P entries (P a power of two): bitonic sort of the
+// INT_MAX-padded run in shared memory, then dedup + compaction straight to out.
+template <int P>
+__device__ __forceinline__ int csr_row_bitonic(const int32_t* in, int32_t L, int32_t* run, int32_t* out, int lane) {
+#pragma unroll
+    for (int j = lane; j < P; j += 32) run[j] = j < L ? in[j] : 0x7fffffff;
+    __syncwarp();
+#pragma unroll
+    for (int k = 2; k <= P; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+#pragma unroll
+            for (int t = lane; t < P / 2; t += 32) {
+                const int i = ((t & ~(j - 1)) << 1) | (t & (j - 1));
+                const int32_t x = run[i], y = run[i + j];
+                const bool up = (i & k) == 0;
+                if ((x > y) == up) {
+                    run[i] = y;
+                    run[i + j] = x;
+                }
+            }
+            __syncwarp();
+        }
+    }
+    int cnt = 0;
+#pragma unroll
+    for (int k = 0; k < P / 32; k++) {
+        const int j = k * 32 + lane;
+        int32_t x = 0;
+        bool keep = false;
+        if (j < L) {
+            x = run[j];
+            keep = (j == 0) || run[j - 1] != x;
+        }
+        unsigned bm = __ballot_sync(0xffffffffu, keep);
+        if (keep) out[cnt + __popc(bm & lanemask_lt())] = x;
+        cnt += __popc(bm);
+    }
+    __syncwarp();
+    return cnt;
 }
 
-__global__ void k_compact_edges(const SortPlan* plan, uint64_t* const* kb, int64_t m, int b,
-                                const int32_t* flag_in, const int32_t* pos, int32_t* col, int32_t* outdeg,
-                                int32_t* indeg) {
+// one warp per row (rows longer than CSR_WARP_MAX are listed for the radix path).
+// srt[rs[r] .. rs[r] + ucnt[r]) = sorted distinct successors of r.
+__global__ void __launch_bounds__(256) k_csr_rowsort(int32_t n, const int32_t* rs, const int32_t* tmp, int32_t* srt,
+                                                     int32_t* ucnt, int32_t* big_list,
+                                                     int32_t* big_ctr /* [0]=rows, [1]=entries */,
+                                                     int32_t* big_off) {
+    __shared__ int32_t runs[8][CSR_WARP_MAX];
+    const int lane = threadIdx.x & 31;
+    int32_t* run = runs[threadIdx.x >> 5];
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {
+        const int32_t s = rs[r], L = rs[r + 1] - s;
+        int c;
+        if (L <= 1) {
+            if (L == 1 && lane == 0) srt[s] = tmp[s];
+            c = L;
+        } else if (L <= 32) {
+            c = csr_row_sort<1>(tmp + s, L, run, srt + s, lane);
+        } else if (L <= 64) {
+            c = csr_row_bitonic<64>(tmp + s, L, run, srt + s, lane);
+        } else if (L <= 128) {
+            c = csr_row_bitonic<128>(tmp + s, L, run, srt + s, lane);
+        } else if (L <= CSR_WARP_MAX) {
+            c = csr_row_bitonic<CSR_WARP_MAX>(tmp + s, L, run, srt + s, lane);
+        } else {
+            if (lane == 0) {
+                int idx = atomicAdd(&big_ctr[0], 1);
+                big_list[idx] = (int32_t)r;
+                big_off[idx] = atomicAdd(&big_ctr[1], L);
+            }
+            continue;
+        }
+        if (lane == 0) ucnt[r] = c;
+    }
+}
+
+// long rows: gather (row << b | dst) keys of every long row for the radix sorter
+__global__ void k_csr_big_gather(const int32_t* big_list, const int32_t* big_off, const int32_t* rs,
+                                 const int32_t* tmp, int b, uint64_t* keys) {
+    const int32_t r = big_list[blockIdx.x];
+    const int32_t s = rs[r], L = rs[r + 1] - s;
+    uint64_t* o = keys + big_off[blockIdx.x];
+    for (int j = threadIdx.x; j < L; j += blockDim.x) o[j] = ((uint64_t)(uint32_t)r << b) | (uint32_t)tmp[s + j];
+}
+
+// long rows after the sort: one block per row finds its run (binary search), keeps the
+// first of every equal run, and compacts into srt with a block-wide ballot scan.
+__global__ void k_csr_big_compact(const int32_t* big_list, const SortPlan* plan, uint64_t* const* kb, int64_t tot,
+                                  const int32_t* rs, int b, int32_t* srt, int32_t* ucnt) {
+    __shared__ int32_t wsum[32];
+    __shared__ int64_t start_s;
     const uint64_t* k = kb[plan->final_sel];
+    const int32_t r = big_list[blockIdx.x];
+    const int32_t s = rs[r], L = rs[r + 1] - s;
+    if (threadIdx.x == 0) {
+        const uint64_t want = (uint64_t)(uint32_t)r << b;
+        int64_t lo = 0, hi = tot;
+        while (lo < hi) {
+            int64_t mid = (lo + hi) >> 1;
+            if (k[mid] < want) lo = mid + 1;
+            else hi = mid;
+        }
+        start_s = lo;
+    }
+    __syncthreads();
+    const uint64_t* kr = k + start_s;
     const uint64_t mask = (1ull << b) - 1;
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
-        bool uniq = (i == 0 || k[i] != k[i - 1]);
-        (void)flag_in;
-        if (!uniq) continue;
-        uint64_t key = k[i];
-        int32_t u = (int32_t)(key >> b), v = (int32_t)(key & mask);
-        col[pos[i]] = v;
-        atomicAdd(&outdeg[u], 1);
-        atomicAdd(&indeg[v], 1);
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+    int32_t out = 0;
+    for (int base = 0; base < L; base += blockDim.x) {
+        int j = base + threadIdx.x;
+        bool keep = j < L && (j == 0 || kr[j] != kr[j - 1]);
+        unsigned bm = __ballot_sync(0xffffffffu, keep);
+        if (lane == 0) wsum[wid] = __popc(bm);
+        __syncthreads();
+        int pre = 0, tot_b = 0;
+        for (int w = 0; w < nwarp; w++) {
+            int c = wsum[w];
+            if (w < wid) pre += c;
+            tot_b += c;
+        }
+        if (keep) srt[s + out + pre + __popc(bm & lanemask_lt())] = (int32_t)(kr[j] & mask);
+        out += tot_b;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) ucnt[r] = out;
+}
+
+// deduplicated rows -> final CSR (row_ptr = exclusive scan of ucnt) + in-degrees
+__global__ void k_csr_emit(int32_t n, const int32_t* rs, const int32_t* srt, const int32_t* ucnt,
+                           const int32_t* row_ptr, int32_t* col, int32_t* indeg) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {
+        const int32_t s = rs[r], c = ucnt[r], o = row_ptr[r];
+        for (int j = lane; j < c; j += 32) {
+            int32_t v = srt[s + j];
+            col[o + j] = v;
+            atomicAdd(&indeg[v], 1);
+        }
     }
 }
 
@@ -318,11 +521,12 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     CK(cudaMemsetAsync(dag->row_ptr, 0, (nn + 1) * 4, st));
     CK(cudaMemsetAsync(dag->indeg, 0, nn * 4, st));
 
-    // ---- a1: sort (src,dst) pairs, dedup, CSR -------------------------------------------
+    // ---- a1: counting-sort CSR (bucket by source, sort + dedup rows) -----------------------
     const int b = bits_for(n > 1 ? n : 2);
     const int npass = (2 * b + 7) / 8;
     const int64_t tps = (mm + SORT_TILE - 1) / SORT_TILE;
-    size_t bytes = sort_bytes(mm, 1, npass, false) + 2 * align256(mm * 4) + align256(64);
+    size_t bytes = sort_bytes(mm, 1, npass, false) + 2 * align256(mm * 4) + 2 * align256((nn + 1) * 4) + align256(2 * (nn + 1) * 4) +
+                   align256(64) + 256 * 4;
     {
         mp_status s = ensure_ws(dag, bytes, st);
         if (s) return cleanup(s);
@@ -331,33 +535,48 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     }
     Arena ar{dag->ws, dag->ws_cap};
     SortArgs sa = carve_sort(ar, dag, mm, 1, 0, npass, false);
-    int32_t* flag = ar.take<int32_t>(mm);
-    int32_t* posb = ar.take<int32_t>(mm);
+    int32_t* tmp = ar.take<int32_t>(mm);
+    int32_t* srt = ar.take<int32_t>(mm);
+    int32_t* cnt = ar.take<int32_t>(nn + 1);   // out-degree counts, then unique counts
+    int32_t* rs = ar.take<int32_t>(nn + 1);    // bucket starts
+    int32_t* bigb = ar.take<int32_t>(2 * (nn + 1));  // long-row list | offsets
     uint64_t** kb = ar.take<uint64_t*>(2);
-    int32_t* d_scal = ar.take<int32_t>(8);  // [0]=E
+    int32_t* d_scal = ar.take<int32_t>(8);  // [0]=E, [2..3] = long rows / entries
     ALLOC(dag->col, mm);
     if (m > 0) {
-        uint64_t* hk[2] = {sa.keys[0], sa.keys[1]};
-        CK(cudaMemcpyAsync(kb, hk, sizeof(hk), cudaMemcpyHostToDevice, st));
-        MP_LAUNCH(k_pack_edges, grid_for(m), 256, 0, st, d_src, d_dst, m, n, b, sa.keys[0], dag->err);
-        sa.seg_len = m;
+        CK(cudaMemsetAsync(cnt, 0, (nn + 1) * 4, st));
+        CK(cudaMemsetAsync(d_scal, 0, 32, st));
+        MP_LAUNCH(k_csr_count, grid_for(m), 256, 0, st, d_src, d_dst, m, n, cnt, dag->err);
         {
-            mp_status s = run_sort(dag, sa, st);
+            mp_status s = scan(dag, cnt, rs, (int64_t)n + 1, nullptr, st);
             if (s) return cleanup(s);
         }
-        MP_LAUNCH(k_dedup_flags, grid_for(m), 256, 0, st, sa.plans, kb, m, flag);
+        MP_LAUNCH(k_csr_fill, grid_for(m), 256, 0, st, d_src, d_dst, m, n, rs, cnt, tmp);
+        MP_LAUNCH(k_csr_rowsort, grid_for((int64_t)n * 32, 256, (int64_t)dag->num_sms * 8), 256, 0, st, n, rs, tmp, srt, cnt, bigb, d_scal + 2,
+                                                                bigb + nn + 1);
+        int32_t h_big[2] = {0, 0};
+        CK(cudaMemcpyAsync(h_big, d_scal + 2, 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (h_big[0] > 0) {
+            uint64_t* hk[2] = {sa.keys[0], sa.keys[1]};
+            CK(cudaMemcpyAsync(kb, hk, sizeof(hk), cudaMemcpyHostToDevice, st));
+            MP_LAUNCH(k_csr_big_gather, h_big[0], 256, 0, st, bigb, bigb + nn + 1, rs, tmp, b, sa.keys[0]);
+            sa.seg_len = h_big[1];
+            {
+                mp_status s = run_sort(dag, sa, st);
+                if (s) return cleanup(s);
+            }
+            MP_LAUNCH(k_csr_big_compact, h_big[0], 1024, 0, st, bigb, sa.plans, kb, (int64_t)h_big[1], rs, b, srt,
+                                                                   cnt);
+        }
         {
-            mp_status s = scan(dag, flag, posb, m, d_scal, st);
+            mp_status s = scan(dag, cnt, dag->row_ptr, (int64_t)n + 1, d_scal, st);
             if (s) return cleanup(s);
         }
-        MP_LAUNCH(k_compact_edges, grid_for(m), 256, 0, st, sa.plans, kb, m, b, flag, posb, dag->col, dag->row_ptr,
-                                                      dag->indeg);
+        MP_LAUNCH(k_csr_emit, grid_for((int64_t)n * 32), 256, 0, st, n, rs, srt, cnt, dag->row_ptr, dag->col,
+                                                             dag->indeg);
     } else {
         CK(cudaMemsetAsync(d_scal, 0, 4, st));
-    }
-    if (n > 0) {
-        mp_status s = scan(dag, dag->row_ptr, dag->row_ptr, (int64_t)n + 1, nullptr, st);
-        if (s) return cleanup(s);
     }
 
     // ---- a2: Kahn levels ----------------------------------------------------------------

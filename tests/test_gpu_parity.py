@@ -124,6 +124,25 @@ def test_deep_chain_and_wide_star():
     compare(n, s2, d2, random_dags.dyadic_durations(n, 2, 4), np.ones(2, np.int32))
 
 
+def test_csr_row_length_boundaries():
+    """a1 ingest: rows of every length class of the counting-sort builder (warp rank sort
+    up to 256 entries, radix path above), heavy duplication, shuffled edge order."""
+    rng = np.random.default_rng(77)
+    lens = [0, 1, 2, 31, 32, 33, 63, 64, 65, 255, 256, 257, 258, 1000, 4097, 20000, 3, 129]
+    n = 30000
+    src, dst = [], []
+    for i, L in enumerate(lens):
+        u = i                                   # sources 0..17, targets above them (acyclic)
+        span = max(1, L // 3) if i % 2 else L   # odd rows: ~3 copies of every successor
+        v = rng.integers(len(lens), min(n, len(lens) + span + 1), size=L)
+        src.append(np.full(L, u, np.int32))
+        dst.append(v.astype(np.int32))
+    src, dst = np.concatenate(src), np.concatenate(dst)
+    p = rng.permutation(len(src))
+    src, dst = src[p], dst[p]
+    compare(n, src, dst, random_dags.dyadic_durations(n, 2, 12), np.ones(2, np.int32))
+
+
 def test_layered_skewed_fanin():
     n, s, d = random_dags.layered_dag([3000, 50, 20000, 7, 40000, 1], fan=40, seed=9)
     compare(n, s, d, random_dags.dyadic_durations(n, 2, 9, tiny_set=True), np.ones(2, np.int32))
