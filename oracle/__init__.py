@@ -20,6 +20,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "mp_oracle.c")
+_SIM_SRC = os.path.join(_HERE, "mp_sim_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 OK, ERR_ARG, ERR_CYCLE, ERR_DOMAIN, ERR_NOMEM = 0, 1, 2, 3, 5
@@ -38,10 +39,11 @@ SUMMARY_DTYPE = np.dtype([("count", "<i4"), ("head", "<i4"), ("brw_lo", "<u8"),
 
 def build(force: bool = False) -> str:
     """Compile the oracle (plain C, single-threaded)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    srcs = [_SRC, _SIM_SRC]
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(map(os.path.getmtime, srcs)):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math",
-                               "-fPIC", "-shared", "-o", tmp, _SRC, "-lm"])
+                               "-fPIC", "-shared", "-o", tmp, *srcs, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -65,6 +67,7 @@ def lib():
         _lib.or_perturb.argtypes = [i32, i32, P, u64, f32, i64, P]
         _lib.or_perturb.restype = None
         _lib.or_replica.argtypes = [i32, i32, P, P, P, P, P, u64, f32, i64, P, P, P, P]
+        _lib.or_simulate.argtypes = [i32, i32, P, P, P, P, P, P, i32, i32, P, P, P]
     return _lib
 
 
@@ -215,3 +218,45 @@ def score_and_queue(dag: Dag, dur, workers, kind=CRIT_BL, done=None):
     qptr, qtask, summ = build_queues(dag, key, flags, dc, done)
     return dict(bl=bl, cp=cp, gain=gain, hd=hd, flags=flags, crit=crit, crit_norm=cn, key=key,
                 qptr=qptr, qtask=qtask, summary=summ)
+
+
+# --------------------------------------------------------------------------
+# discrete-event MultiPrio simulation (mp_sim_oracle.c)
+# --------------------------------------------------------------------------
+SIM_STATS_DTYPE = np.dtype([("makespan", "<f8"), ("pops", "<i8"), ("evictions", "<i8"), ("stale", "<i8"),
+                            ("rounds", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
+SIM_ERR_STUCK = 6
+
+
+def simulate(dag: Dag, dur, workers, key, max_tries=16, eviction=True, trace=True):
+    """PUSH (Alg. 1) / POP (Alg. 2) simulation of one DAG instance.
+
+    dur: canonical durations (check_durations / perturbed), key: the a7 keys
+    that order the heaps.  Returns (stats record, start[n] or None,
+    worker[n] or None)."""
+    dur = _c(dur, np.float32)
+    n, A = dur.shape
+    key = _c(key, np.uint64).reshape(n, A)
+    st = np.zeros(1, SIM_STATS_DTYPE)
+    start = np.zeros(max(n, 1), np.float64) if trace else None
+    worker = np.zeros(max(n, 1), np.int32) if trace else None
+    indeg = _c(dag.indeg, np.int32) if n else np.zeros(1, np.int32)
+    rc = lib().or_simulate(n, A, _p(dag.row_ptr), _p(dag.col if dag.n_edges else np.zeros(1, np.int32)),
+                           _p(indeg), _p(dur), _p(_c(workers, np.int32)), _p(key), int(max_tries),
+                           int(bool(eviction)), _p(st), _p(start), _p(worker))
+    if rc:
+        raise OracleError(rc, "simulate")
+    return st[0], (start[:n] if trace else None), (worker[:n] if trace else None)
+
+
+def simulate_dag(dag: Dag, dur, workers, max_tries=16, eviction=True, kind=CRIT_BL, trace=True):
+    """Score the whole DAG (a3-a7), then simulate it (convenience for tests)."""
+    r = score_and_queue(dag, dur, workers, kind=kind)
+    dc = check_durations(dur, workers)
+    return simulate(dag, dc, workers, r["key"], max_tries, eviction, trace)
+
+
+def simulate_replica(dag: Dag, base, workers, seed, sigma, r, max_tries=16, eviction=True, trace=True):
+    """Replica r (a10 perturbation, BL criticality, ALL-mode scores), simulated."""
+    d = check_durations(perturb(base, seed, sigma, r), workers)
+    return simulate_dag(dag, d, workers, max_tries, eviction, CRIT_BL, trace)
