@@ -210,6 +210,46 @@ mp_status mp_queues_push(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, con
                          const int64_t* d_qptr_in, const int32_t* d_qtask_in, int64_t* d_qptr_out,
                          int32_t* d_qtask_out, mp_queue_summary* d_sum, void* stream);
 
+/*
+ * discrete-event simulation of MultiPrio on a platform of
+ * h_workers[a] workers of each architecture type a: PUSH (Alg. 1,
+ * P:l.133-136) of every task that becomes ready (P:l.91), POP (Alg. 2,
+ * P:l.140-160) by every idle worker with the eviction mechanism
+ * (pop_condition, §V-D, P:l.214-220; eviction = 0 disables it, Fig. 4 top)
+ * and MAX_TRIES = max_tries, and lazy removal of processed duplicates
+ * (P:l.130).  Readings s1-s9: times are binary64 ms, a task
+ * runs delta_r(t,a) (the scored duration of its arch); workers are numbered
+ * arch-major and pop in id order at each event time after the completions
+ * at that time have released their successors; get_most_local_prio_task is
+ * the heap root (no data model); pop_condition(t, a) = eviction off, or a is
+ * a best arch of t, or best_remaining_work[b] > delta(t,a) for every best
+ * arch b; a pop removes t from every heap's counters at once.
+ * Instance r in [r0, r0+R) uses delta_r of mp_replicas_run (sigma = 0: the
+ * base durations) and the ALL-mode queues that give the heap orders:
+ * d_qtask [R][n*A] and d_sum [R][A] exactly as mp_replicas_run writes them,
+ * or, for one DAG (R = 1, r0 = 0, sigma = 0), mp_build_queues' ALL-mode
+ * d_qtask / d_sum (any criticality kind).
+ * Outputs: d_stats [R]; d_start double[R][n] and d_worker int32[R][n] (the
+ * schedule; either may be NULL).  Limits: 1 <= sum of workers <= 256.
+ * A queue entry outside [0, n), a task missing from its arch's queue or a
+ * schedule that cannot complete raise MP_ERR_ARG through mp_check.
+ */
+typedef struct {
+    double makespan;   /* completion time of the last task (ms)              */
+    int64_t pops;      /* successful POPs (= n)                              */
+    int64_t evictions; /* heaps_evict_task calls                             */
+    int64_t stale;     /* processed duplicates removed at a heap root        */
+    int64_t rounds;    /* POP calls that ended on MAX_TRIES                  */
+    double busy[8];    /* sum of delta_r(t,a) over tasks run on arch a, exact */
+                       /*   sum rounded once to binary64                     */
+    int32_t ran[8];    /* tasks run on arch a                                */
+} mp_sim_stats;        /* 136 bytes */
+
+mp_status mp_simulate(mp_dag* dag, int32_t n_arch, const float* d_base_dur, const int32_t* h_workers,
+                      uint64_t seed, float sigma, int64_t r0, int32_t R, const int32_t* d_qtask,
+                      const mp_queue_summary* d_sum, int32_t max_tries, int32_t eviction,
+                      mp_sim_stats* d_stats, double* d_start, int32_t* d_worker, void* stream);
+
 /* Synchronise `stream`, then return (and clear) the handle's device error
  * flag: MP_OK or MP_ERR_DOMAIN; MP_ERR_CUDA on a pending CUDA error. */
 mp_status mp_check(mp_dag* dag, void* stream);

@@ -247,6 +247,45 @@ def queues_push(dag: Dag, key: torch.Tensor, flags: torch.Tensor, dur: torch.Ten
     return out["qptr"], out["qtask"], out["summary"]
 
 
+SIM_STATS_DTYPE = np.dtype([("makespan", "<f8"), ("pops", "<i8"), ("evictions", "<i8"), ("stale", "<i8"),
+                            ("rounds", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
+SIM_STATS_BYTES = 136
+
+
+def simulate(dag: Dag, base_dur: torch.Tensor, workers, seed: int, sigma: float, r0: int, R: int,
+             qtask: torch.Tensor, summary: torch.Tensor, max_tries: int = 16, eviction: bool = True,
+             trace: bool = False, out=None):
+    """N2 (mp_simulate): PUSH/POP simulation of R instances -> (stats bytes[R*136], start, worker).
+
+    qtask/summary: the ALL-mode queues of mp_replicas_run ([R][n*A], [R*A*32])
+    or, for one DAG (R=1, r0=0, sigma=0), of mp_build_queues."""
+    n, A = base_dur.shape
+    w, wp = _workers(workers, A)
+    dev = base_dur.device
+    if out is None:
+        out = dict(stats=torch.empty(max(R, 1) * SIM_STATS_BYTES, dtype=torch.uint8, device=dev),
+                   start=torch.empty((max(R, 1), n), dtype=torch.float64, device=dev) if trace else None,
+                   worker=torch.empty((max(R, 1), n), dtype=torch.int32, device=dev) if trace else None)
+    rc = _lib.lib().mp_simulate(dag.handle, A, _ptr(base_dur), wp, C.c_uint64(seed), C.c_float(sigma), int(r0),
+                                int(R), _ptr(qtask), _ptr(summary), int(max_tries), int(bool(eviction)),
+                                _ptr(out["stats"]), _ptr(out.get("start")), _ptr(out.get("worker")), _stream())
+    _lib.check(rc, "mp_simulate")
+    return out["stats"], out.get("start"), out.get("worker")
+
+
+def sim_stats(stats_bytes: torch.Tensor) -> np.ndarray:
+    """Host view of mp_sim_stats records."""
+    return stats_bytes.detach().cpu().numpy().view(SIM_STATS_DTYPE)
+
+
+def replicas_simulate(dag: Dag, base_dur: torch.Tensor, workers, seed: int, sigma: float, r0: int, R: int,
+                      max_tries: int = 16, eviction: bool = True, trace: bool = False):
+    """a10 queues of R replicas (mp_replicas_run), then their simulation (mp_simulate)."""
+    cp, summ, q = replicas_run(dag, base_dur, workers, seed, sigma, r0, R, want_queues=True)
+    st, start, worker = simulate(dag, base_dur, workers, seed, sigma, r0, R, q, summ, max_tries, eviction, trace)
+    return dict(cp=cp, summary=summ, qtask=q, stats=st, start=start, worker=worker)
+
+
 def summaries(summary_bytes: torch.Tensor) -> np.ndarray:
     """Host view of mp_queue_summary records."""
     return summary_bytes.detach().cpu().numpy().view(SUMMARY_DTYPE)

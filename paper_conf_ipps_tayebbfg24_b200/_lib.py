@@ -16,7 +16,7 @@ MP_CRIT_BOTTOM_LEVEL, MP_CRIT_NOD = 0, 1
 
 EXPORTS = (
     "mp_build_dag", "mp_dag_rebuild", "mp_dag_get_info", "mp_bottom_level", "mp_affinity", "mp_score",
-    "mp_build_queues", "mp_replicas_run", "mp_ready_init", "mp_queues_push", "mp_check", "mp_free", "mp_status_str",
+    "mp_build_queues", "mp_replicas_run", "mp_ready_init", "mp_queues_push", "mp_simulate", "mp_check", "mp_free", "mp_status_str",
     "mp_last_error", "mp_build_info", "mp_launch_count", "mp_prof_enable", "mp_prof_reset", "mp_prof_query", "mp_prof_names",
 )
 
@@ -58,6 +58,7 @@ def lib():
     L.mp_replicas_run.argtypes = [P, i32, P, P, u64, f32, i64, i32, P, P, P, P]
     L.mp_ready_init.argtypes = [P, P, P]
     L.mp_queues_push.argtypes = [P, i32, P, P, P, P, i32, P, P, P, P, P, P, P]
+    L.mp_simulate.argtypes = [P, i32, P, P, u64, f32, i64, i32, P, P, i32, i32, P, P, P, P]
     L.mp_check.argtypes = [P, P]
     L.mp_free.argtypes = [P]
     L.mp_free.restype = None

@@ -6,6 +6,7 @@
 
 #include "push.cuh"
 #include "rep2.cuh"
+#include "sim.cuh"
 
 static inline cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
 
@@ -77,6 +78,14 @@ mp_status mp_queues_push(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, con
                             d_qtask_out, d_sum, as_stream(stream));
 }
 
+mp_status mp_simulate(mp_dag* dag, int32_t n_arch, const float* d_base_dur, const int32_t* h_workers,
+                      uint64_t seed, float sigma, int64_t r0, int32_t R, const int32_t* d_qtask,
+                      const mp_queue_summary* d_sum, int32_t max_tries, int32_t eviction, mp_sim_stats* d_stats,
+                      double* d_start, int32_t* d_worker, void* stream) {
+    return mph::simulate(dag, n_arch, d_base_dur, h_workers, seed, sigma, r0, R, d_qtask, d_sum, max_tries, eviction,
+                         d_stats, d_start, d_worker, as_stream(stream));
+}
+
 mp_status mp_check(mp_dag* dag, void* stream) {
     if (!dag) return mph::fail(MP_ERR_ARG, "dag is NULL");
     cudaStream_t st = as_stream(stream);
@@ -88,6 +97,8 @@ mp_status mp_check(mp_dag* dag, void* stream) {
     if (e & mpk::ERR_DOMAIN_BIT)
         return mph::fail(MP_ERR_DOMAIN, "duration outside {+inf, 0} U [2^-41, 2^20), NaN, or no enabled arch");
     if (e & mpk::ERR_ARG_BIT) return mph::fail(MP_ERR_ARG, "device-detected argument error");
+    if (e & mpk::ERR_SIM_BIT)
+        return mph::fail(MP_ERR_ARG, "mp_simulate: queues do not match the DAG (ALL-mode queues required)");
     return MP_OK;
 }
 

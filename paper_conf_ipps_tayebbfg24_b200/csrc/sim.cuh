@@ -1,0 +1,470 @@
+// sim.cuh -- SURVEY §8(f) N2: discrete-event simulation of MultiPrio's PUSH
+// (Alg. 1, P:l.133-136) and POP (Alg. 2, P:l.140-160) with the eviction
+// mechanism (pop_condition, §V-D, P:l.214-220) and lazy duplicate removal
+// (P:l.130), batched over duration-perturbed replicas (a10).
+//
+// One warp simulates one instance (the event chain of one schedule is
+// sequential; instances are independent).  The heaps are not binary heaps
+// here: a heap's entries are always a subset of that arch's ALL-mode queue
+// (a8; scores are whole-DAG, reading c18), whose order is the heap order, so
+// heap a is a bitmap over queue ranks with a 32-ary summary tree on top
+// (every level-k bit says "word below is non-zero").  PUSH sets the bit at
+// rank_a(t) (atomicOr, lanes push different tasks at once); the root is the
+// first set bit -- one ballot over the top level's <= 32 words plus one
+// broadcast load per level below; a removal clears one bit and propagates
+// empty words up.  Bitmaps and the started set live in shared memory when
+// they fit the per-warp budget, else in a global per-slot scratch (same code
+// through generic pointers).  Readings s1-s9: DESIGN.md §2.
+#pragma once
+#include "handle.cuh"
+
+namespace mpk {
+
+constexpr int SIM_MAX_WORKERS = 256;
+constexpr int SIM_MAX_LEVELS = 6;
+constexpr uint32_t ERR_SIM_BIT = 8u;
+
+struct SimArgs {
+    int32_t n, A, W;
+    int32_t max_tries, eviction;
+    uint64_t seed;
+    float sigma;
+    int64_t r0;
+    int32_t R;
+    int32_t wcum[9];            // workers of archs < a (arch-major numbering, s2)
+    uint32_t emask;             // archs with workers > 0
+    const int32_t* row_ptr;
+    const int32_t* col;
+    const int32_t* indeg;
+    const float* base;          // [n][A]
+    const int32_t* qtask;       // [R][q_stride], queue a at the prefix of counts
+    int64_t q_stride;
+    const mp_queue_summary* sum;  // [R][A]
+    // bitmap layout (identical for every arch): level k at word offset lvoff[k]
+    int32_t nlev;
+    int32_t lvoff[SIM_MAX_LEVELS];
+    int32_t lvsize[SIM_MAX_LEVELS];
+    int32_t bm_words;           // words per arch
+    int32_t st_words;           // started-set words
+    int32_t smem_bits;          // 1: bitmaps + started set in shared memory
+    uint32_t* gbits;            // [slots][A*bm_words + st_words] when !smem_bits
+    int32_t* rank;              // [slots][n*A]
+    int32_t* rem;               // [slots][n]
+    mp_sim_stats* stats;        // [R]
+    double* start;              // [R][n] or null
+    int32_t* worker;            // [R][n] or null
+    uint32_t* err;
+};
+
+struct SimShared {              // per-warp counters (lane 0 writes)
+    unsigned long long brw[8][2];   // best_remaining_work, exact 128-bit
+    unsigned long long busy[8][2];
+    int32_t count[8];               // ready_tasks_count
+    int32_t ran[8];
+    uint32_t again[SIM_MAX_WORKERS / 32];
+};
+
+MP_INLINE void sub128_atomic(unsigned long long* p, uint64_t lo, uint64_t hi) {
+    // p -= (hi:lo), as the addition of the two's complement
+    uint64_t nlo = ~lo + 1ull;
+    uint64_t nhi = ~hi + (lo == 0 ? 1ull : 0ull);
+    atomic_add128(p, nlo, nhi);
+}
+
+MP_INLINE bool gt128(uint64_t alo, uint64_t ahi, uint64_t blo, uint64_t bhi) {
+    return ahi > bhi || (ahi == bhi && alo > blo);
+}
+
+// delta_r(t, a) (a10), -0 read as +0 (c20)
+MP_INLINE float sim_dur(const SimArgs& g, int64_t r, int32_t t, int32_t a) {
+    float d = g.base[(int64_t)t * g.A + a];
+    if (g.sigma != 0.0f) {
+        uint64_t c = ((uint64_t)r * (uint64_t)g.n + (uint64_t)t) * (uint64_t)g.A + (uint64_t)a + 1ull;
+        d = perturb(d, g.seed, g.sigma, c);
+    }
+    return (f2u(d) & 0x7fffffffu) == 0u ? 0.0f : d;
+}
+
+// set bit p of heap `bm` (atomic; concurrent setters allowed)
+MP_INLINE void bm_set(uint32_t* bm, const SimArgs& g, int32_t p) {
+    for (int k = 0; k < g.nlev; ++k) {
+        uint32_t old = atomicOr(bm + g.lvoff[k] + (p >> 5), 1u << (p & 31));
+        if (old != 0u) return;
+        p >>= 5;
+    }
+}
+
+// clear bit p (one lane; no concurrent access)
+MP_INLINE void bm_clear(uint32_t* bm, const SimArgs& g, int32_t p) {
+    for (int k = 0; k < g.nlev; ++k) {
+        uint32_t* w = bm + g.lvoff[k] + (p >> 5);
+        uint32_t v = *w & ~(1u << (p & 31));
+        *w = v;
+        if (v != 0u) return;
+        p >>= 5;
+    }
+}
+
+MP_INLINE bool bm_test(const uint32_t* bm, int32_t p) { return (bm[p >> 5] >> (p & 31)) & 1u; }
+
+// first set bit (the heap root's rank) or -1; whole warp, uniform result
+MP_INLINE int32_t bm_first(const uint32_t* bm, const SimArgs& g, int lane) {
+    int top = g.nlev - 1;
+    uint32_t v = lane < g.lvsize[top] ? bm[g.lvoff[top] + lane] : 0u;
+    uint32_t m = __ballot_sync(0xffffffffu, v != 0u);
+    if (m == 0u) return -1;
+    int l = __ffs(m) - 1;
+    uint32_t w = __shfl_sync(0xffffffffu, v, l);
+    int32_t idx = l * 32 + __ffs(w) - 1;
+    for (int k = top - 1; k >= 0; --k) {
+        w = bm[g.lvoff[k] + idx];
+        idx = idx * 32 + __ffs(w) - 1;
+    }
+    return idx;
+}
+
+// PUSH of task s by this lane (Alg. 1): join every enabled arch's heap;
+// ready_tasks_count and best_remaining_work updated exactly.
+MP_INLINE void sim_push(const SimArgs& g, int64_t r, int32_t s, uint32_t* bits, const int32_t* rank,
+                        SimShared& sh) {
+    float dl[8];
+    float w = __int_as_float(0x7f800000);
+#pragma unroll
+    for (int a = 0; a < 8; ++a) {
+        dl[a] = 0.0f;
+        if (a < g.A) {
+            dl[a] = sim_dur(g, r, s, a);
+            if (((g.emask >> a) & 1u) && !is_inf(dl[a]) && dl[a] < w) w = dl[a];
+        }
+    }
+#pragma unroll
+    for (int a = 0; a < 8; ++a) {
+        if (a < g.A && ((g.emask >> a) & 1u) && !is_inf(dl[a])) {
+            int32_t p = rank[(int64_t)s * g.A + a];
+            if (p < 0) {              // not in the ALL-mode queue a: invalid input
+                atomicOr(g.err, ERR_SIM_BIT);
+                continue;
+            }
+            bm_set(bits + a * g.bm_words, g, p);
+            atomicAdd(&sh.count[a], 1);
+            if (dl[a] == w) {
+                uint64_t lo, hi;
+                fixed64(dl[a], lo, hi);
+                atomic_add128(sh.brw[a], lo, hi);
+            }
+        }
+    }
+}
+
+// the successors of t that become ready (rem reaches 0) are pushed
+MP_INLINE void sim_release(const SimArgs& g, int64_t r, int32_t t, int32_t* rem, uint32_t* bits,
+                           const int32_t* rank, SimShared& sh, int lane) {
+    int32_t beg = g.row_ptr[t], end = g.row_ptr[t + 1];
+    for (int32_t j0 = beg; j0 < end; j0 += 32) {
+        int32_t j = j0 + lane;
+        if (j < end) {
+            int32_t s = g.col[j];
+            int32_t k = rem[s] - 1;
+            rem[s] = k;
+            if (k == 0) sim_push(g, r, s, bits, rank, sh);
+        }
+    }
+    __syncwarp();
+}
+
+__global__ void __launch_bounds__(32) k_sim(SimArgs g) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int lane = threadIdx.x;
+    const int32_t n = g.n, A = g.A, W = g.W;
+    SimShared& sh = *reinterpret_cast<SimShared*>(smem);
+    double* until = reinterpret_cast<double*>(smem + ((sizeof(SimShared) + 15) & ~size_t(15)));
+    int32_t* wtask = reinterpret_cast<int32_t*>(until + W);
+    uint32_t* bits = g.smem_bits ? reinterpret_cast<uint32_t*>(wtask + ((W + 3) & ~3))
+                                 : g.gbits + (size_t)blockIdx.x * (size_t)(A * g.bm_words + g.st_words);
+    uint32_t* started = bits + A * g.bm_words;
+    int32_t* rank = g.rank + (size_t)blockIdx.x * (size_t)n * A;
+    int32_t* rem = g.rem + (size_t)blockIdx.x * (size_t)n;
+
+    for (int32_t rl = blockIdx.x; rl < g.R; rl += gridDim.x) {
+        const int64_t r = g.r0 + rl;
+        const int32_t* q = g.qtask + (int64_t)rl * g.q_stride;
+        int64_t qoff[8];
+        {
+            int64_t o = 0;
+#pragma unroll
+            for (int a = 0; a < 8; ++a) {
+                qoff[a] = o;
+                if (a < A) o += g.sum[(int64_t)rl * A + a].count;
+            }
+        }
+        // ---- init: rem, ranks, empty heaps, idle workers, zero counters
+        for (int32_t t = lane; t < n; t += 32) rem[t] = g.indeg[t];
+        for (int64_t i = lane; i < (int64_t)n * A; i += 32) rank[i] = -1;
+        __syncwarp();
+        for (int a = 0; a < A; ++a) {
+            int32_t c = g.sum[(int64_t)rl * A + a].count;
+            const int32_t* qa = q + qoff[a];
+            for (int32_t p = lane; p < c; p += 32) {
+                int32_t t = qa[p];
+                if ((uint32_t)t < (uint32_t)n) rank[(int64_t)t * A + a] = p;
+                else atomicOr(g.err, ERR_SIM_BIT);
+            }
+        }
+        for (int32_t i = lane; i < A * g.bm_words + g.st_words; i += 32) bits[i] = 0u;
+        for (int32_t w = lane; w < W; w += 32) { until[w] = 0.0; wtask[w] = -1; }
+        if (lane < 8) {
+            sh.brw[lane][0] = sh.brw[lane][1] = 0ull;
+            sh.busy[lane][0] = sh.busy[lane][1] = 0ull;
+            sh.count[lane] = 0;
+            sh.ran[lane] = 0;
+        }
+        __syncwarp();
+        // ---- time 0: the sources are ready (P:l.91)
+        for (int32_t t = lane; t < n; t += 32)
+            if (g.indeg[t] == 0) sim_push(g, r, t, bits, rank, sh);
+        __syncwarp();
+
+        double T = 0.0;
+        int32_t done = 0;
+        int64_t pops = 0, evictions = 0, stale = 0, rounds = 0;
+        bool bad = false;
+        for (;;) {
+            // ---- dispatch (s2, s7): idle workers POP in id order; those whose
+            // POP ended on MAX_TRIES poll again, round-robin, at the same T
+            for (int gi = 0; gi * 32 < W; ++gi) {
+                int w = gi * 32 + lane;
+                uint32_t m = __ballot_sync(0xffffffffu, w < W && wtask[w] < 0);
+                if (lane == 0) sh.again[gi] = m;
+            }
+            __syncwarp();
+            for (bool any = true; any;) {
+                any = false;
+                for (int gi = 0; gi * 32 < W; ++gi) {
+                    uint32_t m = sh.again[gi];
+                    while (m) {
+                        int w = gi * 32 + __ffs(m) - 1;
+                        m &= m - 1;
+                        int a = 0;
+                        while (a + 1 < A && w >= g.wcum[a + 1]) ++a;
+                        uint32_t* bm = bits + a * g.bm_words;
+                        const int32_t* qa = q + qoff[a];
+                        // ---- Alg. 2 POP
+                        int tries = 0;
+                        bool hit = false;
+                        int32_t got = -1;
+                        float dgot = 0.0f;
+                        for (;;) {
+                            if (tries >= g.max_tries) { hit = true; break; }
+                            int32_t p = bm_first(bm, g, lane);
+                            if (p < 0) break;
+                            int32_t t = qa[p];
+                            if (bm_test(started, t)) {         // processed duplicate (P:l.130)
+                                if (lane == 0) bm_clear(bm, g, p);
+                                __syncwarp();
+                                ++stale;
+                                continue;
+                            }
+                            // delta_r(t, b): lane b computes arch b
+                            float mine = lane < A ? sim_dur(g, r, t, lane) : 0.0f;
+                            bool en_l = lane < A && ((g.emask >> lane) & 1u) && !is_inf(mine);
+                            float wmin = en_l ? mine : __int_as_float(0x7f800000);
+#pragma unroll
+                            for (int o = 4; o > 0; o >>= 1) wmin = fminf(wmin, __shfl_xor_sync(0xffffffffu, wmin, o));
+                            wmin = __shfl_sync(0xffffffffu, wmin, 0);
+                            bool best_l = en_l && mine == wmin;
+                            uint32_t bestm = __ballot_sync(0xffffffffu, best_l);
+                            float da = __shfl_sync(0xffffffffu, mine, a);
+                            // pop_condition (§V-D, s4)
+                            bool cond = true;
+                            if (g.eviction && !((bestm >> a) & 1u)) {
+                                uint64_t mlo, mhi;
+                                fixed64(da, mlo, mhi);
+                                bool ok = !best_l || gt128(sh.brw[lane][0], sh.brw[lane][1], mlo, mhi);
+                                cond = __all_sync(0xffffffffu, ok);
+                            }
+                            if (cond) {
+                                // heaps_pop_and_update: t leaves the counters of every heap
+                                // still holding it (s5); duplicates stay for lazy removal
+                                bool counted = false;
+                                if (en_l) counted = lane == a || bm_test(bits + lane * g.bm_words,
+                                                                         rank[(int64_t)t * A + lane]);
+                                if (counted) {
+                                    atomicSub(&sh.count[lane], 1);
+                                    if (best_l) {
+                                        uint64_t lo, hi;
+                                        fixed64(mine, lo, hi);
+                                        sub128_atomic(sh.brw[lane], lo, hi);
+                                    }
+                                }
+                                __syncwarp();
+                                if (lane == 0) {
+                                    bm_clear(bm, g, p);
+                                    started[t >> 5] |= 1u << (t & 31);
+                                }
+                                __syncwarp();
+                                ++pops;
+                                got = t;
+                                dgot = da;
+                                break;
+                            }
+                            // heaps_evict_task: t leaves this heap only (s8)
+                            if (lane == 0) {
+                                bm_clear(bm, g, p);
+                                sh.count[a] -= 1;
+                            }
+                            __syncwarp();
+                            ++evictions;
+                            ++tries;
+                        }
+                        if (hit) { ++rounds; any = true; }
+                        if (lane == 0) {
+                            if (!hit) sh.again[gi] &= ~(1u << (w & 31));
+                            if (got >= 0) {
+                                until[w] = __dadd_rn(T, (double)dgot);   // s1
+                                wtask[w] = got;
+                                uint64_t lo, hi;
+                                fixed64(dgot, lo, hi);
+                                add128(*(uint64_t*)&sh.busy[a][0], *(uint64_t*)&sh.busy[a][1], lo, hi);
+                                sh.ran[a] += 1;
+                                if (g.start) g.start[(int64_t)rl * n + got] = T;
+                                if (g.worker) g.worker[(int64_t)rl * n + got] = w;
+                            }
+                        }
+                        __syncwarp();
+                    }
+                }
+            }
+            // ---- next event: earliest completion (s2)
+            double tmin = __longlong_as_double(0x7ff0000000000000ll);
+            for (int w = lane; w < W; w += 32)
+                if (wtask[w] >= 0 && until[w] < tmin) tmin = until[w];
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                double x = __shfl_xor_sync(0xffffffffu, tmin, o);
+                tmin = x < tmin ? x : tmin;
+            }
+            if (tmin == __longlong_as_double(0x7ff0000000000000ll)) break;   // nobody busy
+            T = tmin;
+            // ---- completions at T in worker id order release successors
+            for (int gi = 0; gi * 32 < W; ++gi) {
+                int w0 = gi * 32 + lane;
+                bool fin = w0 < W && wtask[w0] >= 0 && until[w0] == T;
+                int32_t tl = fin ? wtask[w0] : -1;
+                uint32_t m = __ballot_sync(0xffffffffu, fin);
+                __syncwarp();
+                if (fin) wtask[w0] = -1;
+                __syncwarp();
+                while (m) {
+                    int l = __ffs(m) - 1;
+                    m &= m - 1;
+                    int32_t t = __shfl_sync(0xffffffffu, tl, l);
+                    ++done;
+                    sim_release(g, r, t, rem, bits, rank, sh, lane);
+                }
+            }
+        }
+        if (done != n) bad = true;
+        if (lane == 0) {
+            mp_sim_stats o;
+            o.makespan = T;
+            o.pops = pops;
+            o.evictions = evictions;
+            o.stale = stale;
+            o.rounds = rounds;
+#pragma unroll
+            for (int a = 0; a < 8; ++a) {
+                o.busy[a] = a < A ? u128_to_double_scaled(sh.busy[a][0], sh.busy[a][1]) : 0.0;
+                o.ran[a] = a < A ? sh.ran[a] : 0;
+            }
+            g.stats[rl] = o;
+            if (bad) atomicOr(g.err, ERR_SIM_BIT);
+        }
+        __syncwarp();
+    }
+}
+
+}  // namespace mpk
+
+namespace mph {
+
+inline mp_status simulate(mp_dag* dag, int32_t A, const float* d_base, const int32_t* h_workers, uint64_t seed,
+                          float sigma, int64_t r0, int32_t R, const int32_t* d_qtask, const mp_queue_summary* d_sum,
+                          int32_t max_tries, int32_t eviction, mp_sim_stats* d_stats, double* d_start,
+                          int32_t* d_worker, cudaStream_t st) {
+    if (!dag) return fail(MP_ERR_ARG, "dag is NULL");
+    if (A < 1 || A > 8) return fail(MP_ERR_ARG, "n_arch must be in [1, 8]");
+    if (!h_workers) return fail(MP_ERR_ARG, "h_workers is NULL");
+    if (R < 0 || r0 < 0) return fail(MP_ERR_ARG, "R and r0 must be >= 0");
+    if (max_tries < 1) return fail(MP_ERR_ARG, "max_tries must be >= 1");
+    if (!(sigma >= 0.0f && sigma < 1.0f)) return fail(MP_ERR_ARG, "sigma must be in [0, 1)");
+    mpk::SimArgs g{};
+    g.W = 0;
+    g.wcum[0] = 0;
+    for (int a = 0; a < A; ++a) {
+        if (h_workers[a] < 0) return fail(MP_ERR_ARG, "negative worker count");
+        g.W += h_workers[a];
+        g.wcum[a + 1] = g.W;
+    }
+    if (g.W < 1 || g.W > mpk::SIM_MAX_WORKERS) return fail(MP_ERR_ARG, "total workers must be in [1, %d]",
+                                                           mpk::SIM_MAX_WORKERS);
+    const int32_t n = dag->n;
+    if (R == 0) return MP_OK;
+    if (!d_base || !d_qtask || !d_sum || !d_stats) return fail(MP_ERR_ARG, "NULL device pointer");
+    g.n = n;
+    g.A = A;
+    g.max_tries = max_tries;
+    g.eviction = eviction ? 1 : 0;
+    g.seed = seed;
+    g.sigma = sigma;
+    g.r0 = r0;
+    g.R = R;
+    g.emask = enabled_mask(A, h_workers);
+    g.row_ptr = dag->row_ptr;
+    g.col = dag->col;
+    g.indeg = dag->indeg;
+    g.base = d_base;
+    g.qtask = d_qtask;
+    g.q_stride = (int64_t)n * A;
+    g.sum = d_sum;
+    g.stats = d_stats;
+    g.start = d_start;
+    g.worker = d_worker;
+    g.err = dag->err;
+    // summary-tree layout: level 0 = ceil(n/32) words, each level above 32x
+    // fewer, until one level has <= 32 words (searched by one ballot)
+    int32_t words = std::max<int32_t>(1, (n + 31) / 32), off = 0;
+    g.nlev = 0;
+    for (;;) {
+        if (g.nlev >= mpk::SIM_MAX_LEVELS) return fail(MP_ERR_ARG, "DAG too large for the simulator");
+        g.lvoff[g.nlev] = off;
+        g.lvsize[g.nlev] = words;
+        off += words;
+        g.nlev++;
+        if (words <= 32) break;
+        words = (words + 31) / 32;
+    }
+    g.bm_words = off;
+    g.st_words = std::max<int32_t>(1, (n + 31) / 32);
+    size_t base_smem = ((sizeof(mpk::SimShared) + 15) & ~size_t(15)) + (size_t)g.W * 8 + (size_t)((g.W + 3) & ~3) * 4;
+    size_t bits_bytes = (size_t)(A * g.bm_words + g.st_words) * 4;
+    const size_t kSmemBudget = 48 * 1024;   // per warp: >= 4 instances per SM
+    g.smem_bits = base_smem + bits_bytes <= kSmemBudget ? 1 : 0;
+    size_t smem = base_smem + (g.smem_bits ? bits_bytes : 0);
+    MP_CUDA(cudaFuncSetAttribute(mpk::k_sim, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int per_sm = 0;
+    MP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mpk::k_sim, 32, smem));
+    if (per_sm < 1) return fail(MP_ERR_ARG, "simulator does not fit on an SM");
+    int64_t slots = std::min<int64_t>(R, (int64_t)per_sm * dag->num_sms);
+    size_t need = align256((size_t)slots * n * A * 4) + align256((size_t)slots * std::max(n, 1) * 4) +
+                  (g.smem_bits ? 0 : align256((size_t)slots * bits_bytes));
+    MP_TRY(ensure_ws(dag, need, st));
+    Arena ar{dag->ws, dag->ws_cap};
+    g.rank = ar.take<int32_t>((size_t)slots * n * A);
+    g.rem = ar.take<int32_t>((size_t)slots * std::max(n, 1));
+    g.gbits = g.smem_bits ? nullptr : ar.take<uint32_t>((size_t)slots * (A * g.bm_words + g.st_words));
+    MP_LAUNCH(mpk::k_sim, (unsigned)slots, 32, smem, st, g);
+    MP_CUDA(cudaGetLastError());
+    return MP_OK;
+}
+
+}  // namespace mph
