@@ -36,6 +36,9 @@ import torch.distributed as dist  # noqa: E402
 import workloads  # noqa: E402
 
 METRIC = "DAG tasks scored+queued/sec and ms per DAG (1 GPU; replicas at 1/2/4/8 GPUs)"
+METRIC_SIM = "DAG tasks scored+queued+scheduled (simulated PUSH/POP, N2)/sec and ms per DAG"
+SIM_WORKERS = (30, 2)   # Intel-V100 node: 32 cores, 2 GPUs, one core drives each GPU
+SIM_MAX_TRIES = 16
 UNIT = "tasks/s"
 CONFIG_TEXT = {
     "c1": "tiled Cholesky DAG 4x4 tiles (20 tasks), 2 resource types CPU/GPU, fixed durations",
@@ -43,6 +46,9 @@ CONFIG_TEXT = {
     "c3": "tiled QR DAG 128x128 tiles (707,264 tasks), 3 resource types",
     "c4": "sparse-QR-like elimination-tree DAG + FMM octree DAG (depth 8), 2,156,466 tasks, skewed fan-in",
     "c5": "4096 duration-perturbed replicas of the 64x64 Cholesky DAG sharded across 1/2/4/8 B200",
+    "c5sim": "N2: 4096 duration-perturbed replicas of the 64x64 Cholesky DAG scored+queued (a1-a10) and scheduled "
+             "by the PUSH/POP simulation with eviction (MAX_TRIES 16) on 30 CPU + 2 GPU workers "
+             "(Intel-V100-like node, PAPER.md l.235)",
     "c2push": "N1 incremental READY-mode push over the whole schedule of the 64x64 Cholesky DAG "
               "(each step: sources, then one mp_queues_push per completion batch = every ready task)",
 }
@@ -60,7 +66,7 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c2push"))
+    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c5sim", "c2push"))
     p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS,
                    help="c5: replicas per GPU (weak scaling, default) or in total (--scaling strong)")
     p.add_argument("--scaling", choices=("weak", "strong"), default="weak",
@@ -140,6 +146,18 @@ def oracle_sample(cfg, w, budget_s, R):
     import oracle
     t0 = time.perf_counter()
     od = oracle.build_dag(w.n, w.src, w.dst)
+    if cfg == "c5sim":
+        k = 0
+        while True:
+            oracle.replica(od, w.dur, SIM_WORKERS, workloads.C5_SEED, workloads.C5_SIGMA, k, want_queue=True)
+            oracle.simulate_replica(od, w.dur, SIM_WORKERS, workloads.C5_SEED, workloads.C5_SIGMA, k,
+                                    SIM_MAX_TRIES, True, trace=False)
+            k += 1
+            if time.perf_counter() - t0 >= budget_s or k >= R:
+                break
+        dt = time.perf_counter() - t0
+        return k * w.n / dt, (f"1 DAG build + {k} of {R} replicas of c2: queues + simulated schedule "
+                              f"(perturbation seed {workloads.C5_SEED})"), dt
     if cfg == "c5":
         k = 0
         while True:
@@ -166,7 +184,7 @@ def run_reference(args):
     import oracle
     oracle.build()
     cfg = args.config
-    w = workloads.config("c2" if cfg == "c5" else cfg)
+    w = workloads.config("c2" if cfg in ("c5", "c5sim") else cfg)
     per_step_budget = 3.0 if cfg != "c4" else 10.0
     times, tasks = [], []
     for i in range(args.warmup + args.steps):
@@ -176,7 +194,7 @@ def run_reference(args):
             times.append(dt)
             tasks.append(v * dt)
     value = sum(tasks) / sum(times)
-    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
+    line = {"impl": "reference", "metric": METRIC_SIM if cfg == "c5sim" else METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
             "scaling": "none", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": CONFIG_TEXT[cfg], "name": cfg,
@@ -192,6 +210,7 @@ def run_reference(args):
 def kernel_alg_bytes(name, ctx):
     """Algorithmic (compulsory) HBM bytes per launch of the dominant kernel (DESIGN.md §6 table).
 
+    k_sim       : per simulated instance, queues + indeg + CSR in, statistics out
     k_rep2_sort : per replica, read bl[n] (4n) + write the A queues (4nA)
     k_rep2_bl   : per 32-replica group, read the CSR (4(n+1)+4E) and base durations (4nA);
                   per replica write bl[n] (4n)
@@ -205,6 +224,9 @@ def kernel_alg_bytes(name, ctx):
     if name.startswith("k_rep2_bl"):
         groups = (R + 31) // 32
         return groups * (4 * (n + 1) + 4 * E + 4 * n * A) + R * 4 * n
+    if name.endswith("k_sim"):
+        # per instance: its queues (4nA), indeg (4n) and the CSR (4(n+1)+4E) in, 136 B of statistics out
+        return R * (4 * n * A + 4 * n + 4 * (n + 1) + 4 * E + 136)
     if name == "k_rep_main":
         return 4 * n * A + 4 * (n + 1) + 4 * E + R * 12 * n * A
     if name == "k_sort_pass":
@@ -243,7 +265,7 @@ def run_ours(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     cfg = args.config
-    w = workloads.config("c2" if cfg in ("c5", "c2push") else cfg)
+    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c2push") else cfg)
     A = w.n_arch
     n = w.n
     src_h = torch.from_numpy(w.src).pin_memory()
@@ -256,15 +278,19 @@ def run_ours(args):
     E = dag.n_edges
     stream = torch.cuda.current_stream()
 
-    if cfg == "c5":
+    if cfg in ("c5", "c5sim"):
         # replicas are independent problems keyed by their GLOBAL id (world-size invariant results)
         R = args.replicas * world if args.scaling == "weak" else args.replicas
         r0, cnt = mpd.shard_range(R, world, rank)
         slots = mpd.shard_range(R, world, 0)[1]
-        rb = mpd.record_bytes(A)
+        sim = cfg == "c5sim"
+        workers = np.asarray(SIM_WORKERS if sim else w.workers, np.int32)
+        rb = mpd.record_bytes(A, mp.SIM_STATS_BYTES if sim else 0)
         out = dict(cp=torch.empty(max(cnt, 1), dtype=torch.float32, device=dev),
                    summary=torch.empty(max(cnt, 1) * A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev),
                    qtask=torch.empty((max(cnt, 1), n * A), dtype=torch.int32, device=dev))
+        sim_out = dict(stats=torch.empty(max(cnt, 1) * mp.SIM_STATS_BYTES, dtype=torch.uint8, device=dev),
+                       start=None, worker=None)
         local_rec = torch.zeros((slots, rb), dtype=torch.uint8, device=dev)
         gathered = torch.empty((world * slots, rb), dtype=torch.uint8, device=dev)
         result_h = torch.empty((world * slots, rb), dtype=torch.uint8).pin_memory()
@@ -272,8 +298,12 @@ def run_ours(args):
 
         def step():
             mp.dag_rebuild(dag, n, src_d, dst_d)
-            mp.replicas_run(dag, dur_d, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out=out)
-            mpd.pack_records(out["cp"], out["summary"], cnt, A, slots, out=local_rec)
+            mp.replicas_run(dag, dur_d, workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out=out)
+            if sim:
+                mp.simulate(dag, dur_d, workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out["qtask"],
+                            out["summary"], SIM_MAX_TRIES, True, out=sim_out)
+            mpd.pack_records(out["cp"], out["summary"], cnt, A, slots, out=local_rec,
+                             extra=sim_out["stats"] if sim else None)
             if world > 1:
                 mpd.gather_records(local_rec, out=gathered)
             else:
@@ -414,7 +444,7 @@ def run_ours(args):
     except Exception:
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
     ctx = dict(n=n, E=E, A=A)
-    if cfg == "c5":
+    if cfg in ("c5", "c5sim"):
         ctx["replicas_per_launch"] = cnt      # one k_rep2_bl / k_rep2_sort launch covers the rank's block
         ctx["sort_entries_per_launch"] = cnt * A * n
     else:
@@ -424,13 +454,14 @@ def run_ours(args):
     avg_ms = dom_ms / max(dom_launches, 1)
     achieved = (alg / (avg_ms * 1e-3) / 1e9) if alg else None
     traffic, traffic_src = measured_traffic(dom, cfg)
-    roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+    roof = {"kernel": dom, "bound": "hbm",
+            **({"bound_note": "latency: each warp runs one instance's sequential event chain"} if dom.endswith("k_sim") else {}), "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": (achieved / peak) if achieved else None, "traffic": traffic, "traffic_source": traffic_src,
             "alg_bytes_per_launch": alg, "avg_launch_ms": avg_ms, "launches": dom_launches,
             "share_of_step": (dom_ms / args.steps) / ms_per_step, "peak_source": peak_src,
             "per_kernel_ms_per_step": {k: round(v, 4) for k, v in sorted(step_dev_ms.items(), key=lambda x: -x[1])}}
     # whole-step algorithmic bytes (SURVEY §8(d) B_alg) as context
-    if cfg == "c5":
+    if cfg in ("c5", "c5sim"):
         b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + args.replicas * 4 * n * A / world  # CSR + dur + queues out
     else:
         b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 4 * n * A + 4 * n * A
@@ -444,25 +475,32 @@ def run_ours(args):
         v, sample, dt = oracle_sample(cfg, w, args.cpu_budget_s, args.replicas)
         cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, "seconds": round(dt, 2)}
 
-    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+    rep = cfg in ("c5", "c5sim")
+    line = {"metric": METRIC_SIM if cfg == "c5sim" else METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": args.scaling if cfg == "c5" else "none", "vs_baseline": None, "dtype": "f32",
+            "scaling": args.scaling if cfg in ("c5", "c5sim") else "none", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic",
-            "config": {"workload": (CONFIG_TEXT[cfg] if cfg != "c5" else
+            "config": {"workload": (CONFIG_TEXT[cfg] if not rep else
                                     f"{R} duration-perturbed replicas of the 64x64 Cholesky DAG ({cnt} per GPU, "
-                                    f"{args.scaling} scaling; BASELINE config 5 = 4096 in total = --scaling strong)"),
+                                    f"{args.scaling} scaling; BASELINE config 5 = 4096 in total = --scaling strong)"
+                                    + ("; each scheduled by the N2 PUSH/POP simulation with eviction on "
+                                       f"{SIM_WORKERS[0]} CPU + {SIM_WORKERS[1]} GPU workers" if cfg == "c5sim" else "")),
                        "name": cfg, "tasks_per_dag": n, "edges": E,
                        "levels": dag.n_levels, "archs": A,
-                       "replicas": R if cfg == "c5" else 1, "replicas_per_gpu": cnt,
-                       "ms_per_dag": ms_per_step / (R if cfg == "c5" else 1) * world if cfg == "c5" else ms_per_step,
+                       "replicas": R if rep else 1, "replicas_per_gpu": cnt,
+                       "ms_per_dag": ms_per_step / (R if rep else 1) * world if rep else ms_per_step,
                        "l2": f"flushed between timed steps ({L2_FLUSH_BYTES >> 20} MiB write)",
-                       "queues": "materialised in HBM for every replica" if cfg == "c5" else "materialised",
+                       "queues": "materialised in HBM for every replica" if rep else "materialised",
                        "step": ("mp_dag_rebuild + mp_replicas_run + allgather(records)" if cfg == "c5" else
+                                "mp_dag_rebuild + mp_replicas_run + mp_simulate + allgather(records + sim stats)"
+                                if cfg == "c5sim" else
                                 "mp_build_queues(sources) + mp_queues_push per completion batch (scores precomputed)"
                                 if cfg == "c2push" else
                                 "mp_dag_rebuild + bottom_level + affinity + score + build_queues"),
-                       "parallelism": f"replica shards x{world}" if cfg == "c5" else "single DAG"},
-            "ms_per_dag": ms_per_step / (R / world) if cfg == "c5" else ms_per_step,
+                       "parallelism": f"replica shards x{world}" if rep else "single DAG",
+                       **({"sim_workers": list(SIM_WORKERS), "max_tries": SIM_MAX_TRIES, "eviction": True}
+                          if cfg == "c5sim" else {})},
+            "ms_per_dag": ms_per_step / (R / world) if rep else ms_per_step,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
             "gpu_launches_per_step": launches / args.steps, "clocks": ck,
             "device": torch.cuda.get_device_name(dev)}

@@ -238,7 +238,7 @@ typedef struct {
     double makespan;   /* completion time of the last task (ms)              */
     int64_t pops;      /* successful POPs (= n)                              */
     int64_t evictions; /* heaps_evict_task calls                             */
-    int64_t stale;     /* processed duplicates removed at a heap root        */
+    int64_t dups;      /* duplicates a pop leaves in the other heaps (P:l.130) */
     int64_t rounds;    /* POP calls that ended on MAX_TRIES                  */
     double busy[8];    /* sum of delta_r(t,a) over tasks run on arch a, exact */
                        /*   sum rounded once to binary64                     */

@@ -37,7 +37,7 @@ typedef struct {             /* per simulated instance                         *
     double makespan;         /* completion time of the last task (ms)          */
     int64_t pops;            /* successful POPs (= n)                          */
     int64_t evictions;       /* heaps_evict_task calls (Alg. 2)                */
-    int64_t stale;           /* duplicates found already processed (P:l.130)   */
+    int64_t dups;            /* duplicates a pop leaves in other heaps (P:l.130) */
     int64_t rounds;          /* POP calls that ended on MAX_TRIES              */
     double busy[8];          /* sum of delta(t,a) over tasks run on arch a     */
     int32_t ran[8];          /* tasks run on arch a                            */
@@ -165,11 +165,13 @@ static int32_t pop(sched* s, int32_t a, so_stats* st, int* hit_max) {
         int32_t t = h->v[0];                       /* get_most_local_prio_task: */
         if (s->started[t]) {                       /* the heap root (s6)        */
             heap_pop_root(h);                      /* processed duplicate:      */
-            st->stale += 1;                        /* removed, not a try (s5)   */
-            continue;
+            continue;                              /* removed, not a try (s5)   */
         }
         if (pop_condition(s, t, a)) {
             heap_pop_root(h);                      /* heaps_pop_and_update      */
+            for (int32_t b = 0; b < s->A; b++)     /* "any duplicate tasks in   */
+                if (b != a && s->counted[(int64_t)t * s->A + b])   /* other     */
+                    st->dups += 1;                 /* queues will remain there" */
             uncount(s, t);
             s->started[t] = 1;
             st->pops += 1;

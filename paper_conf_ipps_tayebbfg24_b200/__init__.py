@@ -247,7 +247,7 @@ def queues_push(dag: Dag, key: torch.Tensor, flags: torch.Tensor, dur: torch.Ten
     return out["qptr"], out["qtask"], out["summary"]
 
 
-SIM_STATS_DTYPE = np.dtype([("makespan", "<f8"), ("pops", "<i8"), ("evictions", "<i8"), ("stale", "<i8"),
+SIM_STATS_DTYPE = np.dtype([("makespan", "<f8"), ("pops", "<i8"), ("evictions", "<i8"), ("dups", "<i8"),
                             ("rounds", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
 SIM_STATS_BYTES = 136
 

@@ -1,6 +1,6 @@
 // sim.cuh -- SURVEY §8(f) N2: discrete-event simulation of MultiPrio's PUSH
 // (Alg. 1, P:l.133-136) and POP (Alg. 2, P:l.140-160) with the eviction
-// mechanism (pop_condition, §V-D, P:l.214-220) and lazy duplicate removal
+// mechanism (pop_condition, §V-D, P:l.214-220) and duplicate handling
 // (P:l.130), batched over duration-perturbed replicas (a10).
 //
 // One warp simulates one instance (the event chain of one schedule is
@@ -12,9 +12,18 @@
 // rank_a(t) (atomicOr, lanes push different tasks at once); the root is the
 // first set bit -- one ballot over the top level's <= 32 words plus one
 // broadcast load per level below; a removal clears one bit and propagates
-// empty words up.  Bitmaps and the started set live in shared memory when
-// they fit the per-warp budget, else in a global per-slot scratch (same code
-// through generic pointers).  Readings s1-s9: DESIGN.md §2.
+// empty words up.  A popped task's duplicates are cleared from the other
+// heaps at once (a bitmap deletes in place; the paper's binary heaps remove
+// them lazily, P:l.130 -- a processed duplicate is skipped without counting
+// as a try, reading s5, so the schedule is the same).
+//
+// Per instance, a per-slot record array holds for each task t, in one 32-B
+// (A <= 3) sector: rem(t) (predecessors not completed), the enabled / best
+// arch masks, rank_a(t) and delta_r(t,a); a release therefore costs one
+// dependent load per successor and a POP one load after the root search.
+// Bitmaps live in shared memory when they fit the per-warp budget, else in a
+// global per-slot scratch (same code through generic pointers).
+// Readings s1-s9: DESIGN.md §2.
 #pragma once
 #include "handle.cuh"
 
@@ -25,7 +34,7 @@ constexpr int SIM_MAX_LEVELS = 6;
 constexpr uint32_t ERR_SIM_BIT = 8u;
 
 struct SimArgs {
-    int32_t n, A, W;
+    int32_t n, A, W, S;         // S = record stride in words (power of two >= 2 + 2A)
     int32_t max_tries, eviction;
     uint64_t seed;
     float sigma;
@@ -45,18 +54,20 @@ struct SimArgs {
     int32_t lvoff[SIM_MAX_LEVELS];
     int32_t lvsize[SIM_MAX_LEVELS];
     int32_t bm_words;           // words per arch
-    int32_t st_words;           // started-set words
-    int32_t smem_bits;          // 1: bitmaps + started set in shared memory
-    uint32_t* gbits;            // [slots][A*bm_words + st_words] when !smem_bits
-    int32_t* rank;              // [slots][n*A]
-    int32_t* rem;               // [slots][n]
+    int32_t smem_bits;          // 1: bitmaps in shared memory
+    uint32_t* gbits;            // [slots][A*bm_words] when !smem_bits
+    uint32_t* rec;              // [slots][n][S]
     mp_sim_stats* stats;        // [R]
     double* start;              // [R][n] or null
     int32_t* worker;            // [R][n] or null
     uint32_t* err;
 };
 
-struct SimShared {              // per-warp counters (lane 0 writes)
+// record words: [0] rem, [1] enabled mask | best mask << 8, [2, 2+A) rank_a,
+// [2+A, 2+2A) bits of delta_r(t,a)
+constexpr int REC_REM = 0, REC_MASK = 1, REC_RANK = 2;
+
+struct SimShared {              // per-warp counters
     unsigned long long brw[8][2];   // best_remaining_work, exact 128-bit
     unsigned long long busy[8][2];
     int32_t count[8];               // ready_tasks_count
@@ -94,7 +105,7 @@ MP_INLINE void bm_set(uint32_t* bm, const SimArgs& g, int32_t p) {
     }
 }
 
-// clear bit p (one lane; no concurrent access)
+// clear bit p (one lane per heap; no concurrent access to the same heap)
 MP_INLINE void bm_clear(uint32_t* bm, const SimArgs& g, int32_t p) {
     for (int k = 0; k < g.nlev; ++k) {
         uint32_t* w = bm + g.lvoff[k] + (p >> 5);
@@ -124,93 +135,66 @@ MP_INLINE int32_t bm_first(const uint32_t* bm, const SimArgs& g, int lane) {
 }
 
 // PUSH of task s by this lane (Alg. 1): join every enabled arch's heap;
-// ready_tasks_count and best_remaining_work updated exactly.
-MP_INLINE void sim_push(const SimArgs& g, int64_t r, int32_t s, uint32_t* bits, const int32_t* rank,
-                        SimShared& sh) {
-    float dl[8];
-    float w = __int_as_float(0x7f800000);
-#pragma unroll
-    for (int a = 0; a < 8; ++a) {
-        dl[a] = 0.0f;
-        if (a < g.A) {
-            dl[a] = sim_dur(g, r, s, a);
-            if (((g.emask >> a) & 1u) && !is_inf(dl[a]) && dl[a] < w) w = dl[a];
+// ready_tasks_count and best_remaining_work updated exactly.  `rc` = s's record.
+MP_INLINE void sim_push(const SimArgs& g, const uint32_t* rc, uint32_t* bits, SimShared& sh) {
+    uint32_t masks = rc[REC_MASK];
+    for (int a = 0; a < g.A; ++a) {
+        if (!((masks >> a) & 1u)) continue;
+        int32_t p = (int32_t)rc[REC_RANK + a];
+        if (p < 0) {              // not in the ALL-mode queue a: invalid input
+            atomicOr(g.err, ERR_SIM_BIT);
+            continue;
+        }
+        bm_set(bits + a * g.bm_words, g, p);
+        atomicAdd(&sh.count[a], 1);
+        if ((masks >> (8 + a)) & 1u) {
+            uint64_t lo, hi;
+            fixed64(u2f(rc[REC_RANK + g.A + a]), lo, hi);
+            atomic_add128(sh.brw[a], lo, hi);
         }
     }
-#pragma unroll
-    for (int a = 0; a < 8; ++a) {
-        if (a < g.A && ((g.emask >> a) & 1u) && !is_inf(dl[a])) {
-            int32_t p = rank[(int64_t)s * g.A + a];
-            if (p < 0) {              // not in the ALL-mode queue a: invalid input
-                atomicOr(g.err, ERR_SIM_BIT);
-                continue;
-            }
-            bm_set(bits + a * g.bm_words, g, p);
-            atomicAdd(&sh.count[a], 1);
-            if (dl[a] == w) {
-                uint64_t lo, hi;
-                fixed64(dl[a], lo, hi);
-                atomic_add128(sh.brw[a], lo, hi);
-            }
-        }
-    }
-}
-
-// the successors of t that become ready (rem reaches 0) are pushed
-MP_INLINE void sim_release(const SimArgs& g, int64_t r, int32_t t, int32_t* rem, uint32_t* bits,
-                           const int32_t* rank, SimShared& sh, int lane) {
-    int32_t beg = g.row_ptr[t], end = g.row_ptr[t + 1];
-    for (int32_t j0 = beg; j0 < end; j0 += 32) {
-        int32_t j = j0 + lane;
-        if (j < end) {
-            int32_t s = g.col[j];
-            int32_t k = rem[s] - 1;
-            rem[s] = k;
-            if (k == 0) sim_push(g, r, s, bits, rank, sh);
-        }
-    }
-    __syncwarp();
 }
 
 __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
     extern __shared__ __align__(16) unsigned char smem[];
     const int lane = threadIdx.x;
-    const int32_t n = g.n, A = g.A, W = g.W;
+    const int32_t n = g.n, A = g.A, W = g.W, S = g.S;
     SimShared& sh = *reinterpret_cast<SimShared*>(smem);
     double* until = reinterpret_cast<double*>(smem + ((sizeof(SimShared) + 15) & ~size_t(15)));
     int32_t* wtask = reinterpret_cast<int32_t*>(until + W);
     uint32_t* bits = g.smem_bits ? reinterpret_cast<uint32_t*>(wtask + ((W + 3) & ~3))
-                                 : g.gbits + (size_t)blockIdx.x * (size_t)(A * g.bm_words + g.st_words);
-    uint32_t* started = bits + A * g.bm_words;
-    int32_t* rank = g.rank + (size_t)blockIdx.x * (size_t)n * A;
-    int32_t* rem = g.rem + (size_t)blockIdx.x * (size_t)n;
+                                 : g.gbits + (size_t)blockIdx.x * (size_t)(A * g.bm_words);
+    uint32_t* rec = g.rec + (size_t)blockIdx.x * (size_t)n * S;
 
     for (int32_t rl = blockIdx.x; rl < g.R; rl += gridDim.x) {
         const int64_t r = g.r0 + rl;
         const int32_t* q = g.qtask + (int64_t)rl * g.q_stride;
-        int64_t qoff[8];
-        {
-            int64_t o = 0;
-#pragma unroll
-            for (int a = 0; a < 8; ++a) {
-                qoff[a] = o;
-                if (a < A) o += g.sum[(int64_t)rl * A + a].count;
+        // ---- init: records (rem, masks, no rank yet, delta_r), empty heaps,
+        //      idle workers, zero counters
+        for (int32_t t = lane; t < n; t += 32) {
+            uint32_t* rc = rec + (size_t)t * S;
+            float d[8];
+            float wmin = __int_as_float(0x7f800000);
+            uint32_t en = 0;
+            for (int a = 0; a < A; ++a) {
+                float x = sim_dur(g, r, t, a);
+                d[a & 7] = x;
+                if (((g.emask >> a) & 1u) && !is_inf(x)) {
+                    en |= 1u << a;
+                    if (x < wmin) wmin = x;
+                }
+            }
+            uint32_t best = 0;
+            for (int a = 0; a < A; ++a)
+                if (((en >> a) & 1u) && d[a & 7] == wmin) best |= 1u << a;   // c15
+            rc[REC_REM] = (uint32_t)g.indeg[t];
+            rc[REC_MASK] = en | (best << 8);
+            for (int a = 0; a < A; ++a) {
+                rc[REC_RANK + a] = 0xffffffffu;
+                rc[REC_RANK + A + a] = f2u(d[a & 7]);
             }
         }
-        // ---- init: rem, ranks, empty heaps, idle workers, zero counters
-        for (int32_t t = lane; t < n; t += 32) rem[t] = g.indeg[t];
-        for (int64_t i = lane; i < (int64_t)n * A; i += 32) rank[i] = -1;
-        __syncwarp();
-        for (int a = 0; a < A; ++a) {
-            int32_t c = g.sum[(int64_t)rl * A + a].count;
-            const int32_t* qa = q + qoff[a];
-            for (int32_t p = lane; p < c; p += 32) {
-                int32_t t = qa[p];
-                if ((uint32_t)t < (uint32_t)n) rank[(int64_t)t * A + a] = p;
-                else atomicOr(g.err, ERR_SIM_BIT);
-            }
-        }
-        for (int32_t i = lane; i < A * g.bm_words + g.st_words; i += 32) bits[i] = 0u;
+        for (int32_t i = lane; i < A * g.bm_words; i += 32) bits[i] = 0u;
         for (int32_t w = lane; w < W; w += 32) { until[w] = 0.0; wtask[w] = -1; }
         if (lane < 8) {
             sh.brw[lane][0] = sh.brw[lane][1] = 0ull;
@@ -219,15 +203,28 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
             sh.ran[lane] = 0;
         }
         __syncwarp();
+        {
+            int64_t o = 0;
+            for (int a = 0; a < A; ++a) {
+                int32_t c = g.sum[(int64_t)rl * A + a].count;
+                const int32_t* qa = q + o;
+                for (int32_t p = lane; p < c; p += 32) {
+                    int32_t t = qa[p];
+                    if ((uint32_t)t < (uint32_t)n) rec[(size_t)t * S + REC_RANK + a] = (uint32_t)p;
+                    else atomicOr(g.err, ERR_SIM_BIT);
+                }
+                o += c;
+            }
+        }
+        __syncwarp();
         // ---- time 0: the sources are ready (P:l.91)
         for (int32_t t = lane; t < n; t += 32)
-            if (g.indeg[t] == 0) sim_push(g, r, t, bits, rank, sh);
+            if (g.indeg[t] == 0) sim_push(g, rec + (size_t)t * S, bits, sh);
         __syncwarp();
 
         double T = 0.0;
         int32_t done = 0;
-        int64_t pops = 0, evictions = 0, stale = 0, rounds = 0;
-        bool bad = false;
+        int64_t pops = 0, evictions = 0, dups = 0, rounds = 0;
         for (;;) {
             // ---- dispatch (s2, s7): idle workers POP in id order; those whose
             // POP ended on MAX_TRIES poll again, round-robin, at the same T
@@ -247,7 +244,9 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                         int a = 0;
                         while (a + 1 < A && w >= g.wcum[a + 1]) ++a;
                         uint32_t* bm = bits + a * g.bm_words;
-                        const int32_t* qa = q + qoff[a];
+                        int64_t qoff = 0;
+                        for (int b = 0; b < a; ++b) qoff += g.sum[(int64_t)rl * A + b].count;
+                        const int32_t* qa = q + qoff;
                         // ---- Alg. 2 POP
                         int tries = 0;
                         bool hit = false;
@@ -258,37 +257,30 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                             int32_t p = bm_first(bm, g, lane);
                             if (p < 0) break;
                             int32_t t = qa[p];
-                            if (bm_test(started, t)) {         // processed duplicate (P:l.130)
-                                if (lane == 0) bm_clear(bm, g, p);
-                                __syncwarp();
-                                ++stale;
-                                continue;
-                            }
-                            // delta_r(t, b): lane b computes arch b
-                            float mine = lane < A ? sim_dur(g, r, t, lane) : 0.0f;
-                            bool en_l = lane < A && ((g.emask >> lane) & 1u) && !is_inf(mine);
-                            float wmin = en_l ? mine : __int_as_float(0x7f800000);
-#pragma unroll
-                            for (int o = 4; o > 0; o >>= 1) wmin = fminf(wmin, __shfl_xor_sync(0xffffffffu, wmin, o));
-                            wmin = __shfl_sync(0xffffffffu, wmin, 0);
-                            bool best_l = en_l && mine == wmin;
-                            uint32_t bestm = __ballot_sync(0xffffffffu, best_l);
+                            const uint32_t* rc = rec + (size_t)t * S;
+                            uint32_t masks = rc[REC_MASK];
+                            // lane b < A: arch b's rank and delta
+                            int32_t rk = lane < A ? (int32_t)rc[REC_RANK + lane] : -1;
+                            float mine = lane < A ? u2f(rc[REC_RANK + A + lane]) : 0.0f;
+                            bool best_l = lane < A && ((masks >> (8 + lane)) & 1u);
                             float da = __shfl_sync(0xffffffffu, mine, a);
                             // pop_condition (§V-D, s4)
                             bool cond = true;
-                            if (g.eviction && !((bestm >> a) & 1u)) {
+                            if (g.eviction && !((masks >> (8 + a)) & 1u)) {
                                 uint64_t mlo, mhi;
                                 fixed64(da, mlo, mhi);
                                 bool ok = !best_l || gt128(sh.brw[lane][0], sh.brw[lane][1], mlo, mhi);
                                 cond = __all_sync(0xffffffffu, ok);
                             }
                             if (cond) {
-                                // heaps_pop_and_update: t leaves the counters of every heap
-                                // still holding it (s5); duplicates stay for lazy removal
-                                bool counted = false;
-                                if (en_l) counted = lane == a || bm_test(bits + lane * g.bm_words,
-                                                                         rank[(int64_t)t * A + lane]);
-                                if (counted) {
+                                // heaps_pop_and_update: t leaves every heap that still
+                                // holds it and their counters (s5)
+                                bool held = false;
+                                if (lane < A && ((masks >> lane) & 1u))
+                                    held = lane == a || (rk >= 0 && bm_test(bits + lane * g.bm_words, rk));
+                                uint32_t hm = __ballot_sync(0xffffffffu, held);
+                                if (held) {
+                                    bm_clear(bits + lane * g.bm_words, g, lane == a ? p : rk);
                                     atomicSub(&sh.count[lane], 1);
                                     if (best_l) {
                                         uint64_t lo, hi;
@@ -297,11 +289,7 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                                     }
                                 }
                                 __syncwarp();
-                                if (lane == 0) {
-                                    bm_clear(bm, g, p);
-                                    started[t >> 5] |= 1u << (t & 31);
-                                }
-                                __syncwarp();
+                                dups += __popc(hm) - 1;
                                 ++pops;
                                 got = t;
                                 dgot = da;
@@ -345,13 +333,13 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
             }
             if (tmin == __longlong_as_double(0x7ff0000000000000ll)) break;   // nobody busy
             T = tmin;
-            // ---- completions at T in worker id order release successors
+            // ---- completions at T, in worker id order, release their
+            // successors (lanes over a task's successor row; pushes commute)
             for (int gi = 0; gi * 32 < W; ++gi) {
                 int w0 = gi * 32 + lane;
                 bool fin = w0 < W && wtask[w0] >= 0 && until[w0] == T;
                 int32_t tl = fin ? wtask[w0] : -1;
                 uint32_t m = __ballot_sync(0xffffffffu, fin);
-                __syncwarp();
                 if (fin) wtask[w0] = -1;
                 __syncwarp();
                 while (m) {
@@ -359,17 +347,26 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                     m &= m - 1;
                     int32_t t = __shfl_sync(0xffffffffu, tl, l);
                     ++done;
-                    sim_release(g, r, t, rem, bits, rank, sh, lane);
+                    int32_t beg = g.row_ptr[t], end = g.row_ptr[t + 1];
+                    for (int32_t j0 = beg; j0 < end; j0 += 32) {
+                        int32_t j = j0 + lane;
+                        if (j < end) {
+                            uint32_t* rc = rec + (size_t)g.col[j] * S;
+                            uint32_t k = rc[REC_REM] - 1u;
+                            rc[REC_REM] = k;
+                            if (k == 0u) sim_push(g, rc, bits, sh);
+                        }
+                    }
+                    __syncwarp();
                 }
             }
         }
-        if (done != n) bad = true;
         if (lane == 0) {
             mp_sim_stats o;
             o.makespan = T;
             o.pops = pops;
             o.evictions = evictions;
-            o.stale = stale;
+            o.dups = dups;
             o.rounds = rounds;
 #pragma unroll
             for (int a = 0; a < 8; ++a) {
@@ -377,7 +374,7 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                 o.ran[a] = a < A ? sh.ran[a] : 0;
             }
             g.stats[rl] = o;
-            if (bad) atomicOr(g.err, ERR_SIM_BIT);
+            if (done != n) atomicOr(g.err, ERR_SIM_BIT);
         }
         __syncwarp();
     }
@@ -412,6 +409,8 @@ inline mp_status simulate(mp_dag* dag, int32_t A, const float* d_base, const int
     if (!d_base || !d_qtask || !d_sum || !d_stats) return fail(MP_ERR_ARG, "NULL device pointer");
     g.n = n;
     g.A = A;
+    g.S = 4;
+    while (g.S < 2 + 2 * A) g.S *= 2;
     g.max_tries = max_tries;
     g.eviction = eviction ? 1 : 0;
     g.seed = seed;
@@ -444,9 +443,8 @@ inline mp_status simulate(mp_dag* dag, int32_t A, const float* d_base, const int
         words = (words + 31) / 32;
     }
     g.bm_words = off;
-    g.st_words = std::max<int32_t>(1, (n + 31) / 32);
     size_t base_smem = ((sizeof(mpk::SimShared) + 15) & ~size_t(15)) + (size_t)g.W * 8 + (size_t)((g.W + 3) & ~3) * 4;
-    size_t bits_bytes = (size_t)(A * g.bm_words + g.st_words) * 4;
+    size_t bits_bytes = (size_t)(A * g.bm_words) * 4;
     const size_t kSmemBudget = 48 * 1024;   // per warp: >= 4 instances per SM
     g.smem_bits = base_smem + bits_bytes <= kSmemBudget ? 1 : 0;
     size_t smem = base_smem + (g.smem_bits ? bits_bytes : 0);
@@ -455,13 +453,12 @@ inline mp_status simulate(mp_dag* dag, int32_t A, const float* d_base, const int
     MP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mpk::k_sim, 32, smem));
     if (per_sm < 1) return fail(MP_ERR_ARG, "simulator does not fit on an SM");
     int64_t slots = std::min<int64_t>(R, (int64_t)per_sm * dag->num_sms);
-    size_t need = align256((size_t)slots * n * A * 4) + align256((size_t)slots * std::max(n, 1) * 4) +
+    size_t need = align256((size_t)slots * std::max(n, 1) * g.S * 4) +
                   (g.smem_bits ? 0 : align256((size_t)slots * bits_bytes));
     MP_TRY(ensure_ws(dag, need, st));
     Arena ar{dag->ws, dag->ws_cap};
-    g.rank = ar.take<int32_t>((size_t)slots * n * A);
-    g.rem = ar.take<int32_t>((size_t)slots * std::max(n, 1));
-    g.gbits = g.smem_bits ? nullptr : ar.take<uint32_t>((size_t)slots * (A * g.bm_words + g.st_words));
+    g.rec = ar.take<uint32_t>((size_t)slots * std::max(n, 1) * g.S);
+    g.gbits = g.smem_bits ? nullptr : ar.take<uint32_t>((size_t)slots * A * g.bm_words);
     MP_LAUNCH(mpk::k_sim, (unsigned)slots, 32, smem, st, g);
     MP_CUDA(cudaGetLastError());
     return MP_OK;

@@ -26,19 +26,24 @@ def shard_range(R: int, world: int, rank: int) -> tuple[int, int]:
     return r0, count
 
 
-def record_bytes(n_arch: int) -> int:
-    return 4 + n_arch * SUMMARY_BYTES
+def record_bytes(n_arch: int, extra: int = 0) -> int:
+    return 4 + n_arch * SUMMARY_BYTES + extra
 
 
 def pack_records(cp: torch.Tensor, summary: torch.Tensor, count: int, n_arch: int, slots: int,
-                 out: torch.Tensor | None = None) -> torch.Tensor:
-    """[slots, 4 + A*32] uint8 records (CP float bits, then the A summaries); rows >= count are zero."""
-    rb = record_bytes(n_arch)
+                 out: torch.Tensor | None = None, extra: torch.Tensor | None = None) -> torch.Tensor:
+    """[slots, 4 + A*32 (+ k)] uint8 records (CP float bits, the A summaries, then `extra`'s k
+    bytes per replica, e.g. the N2 simulation statistics); rows >= count are zero."""
+    k = 0 if extra is None else extra.numel() // max(count, 1)
+    rb = record_bytes(n_arch, k)
     if out is None:
         out = torch.zeros((slots, rb), dtype=torch.uint8, device=cp.device)
     if count:
+        q = 4 + n_arch * SUMMARY_BYTES
         out[:count, :4].copy_(cp[:count].contiguous().view(torch.uint8).view(count, 4))
-        out[:count, 4:].copy_(summary[:count * n_arch * SUMMARY_BYTES].view(count, n_arch * SUMMARY_BYTES))
+        out[:count, 4:q].copy_(summary[:count * n_arch * SUMMARY_BYTES].view(count, n_arch * SUMMARY_BYTES))
+        if k:
+            out[:count, q:q + k].copy_(extra.reshape(-1)[:count * k].view(count, k))
     return out
 
 
@@ -51,8 +56,9 @@ def gather_records(local: torch.Tensor, group=None, out: torch.Tensor | None = N
     return out
 
 
-def unpack_records(gathered: torch.Tensor, R: int, world: int, n_arch: int):
-    """Reassemble (cp[R] float32, summary bytes[R*A*32]) ordered by global replica id."""
+def unpack_records(gathered: torch.Tensor, R: int, world: int, n_arch: int, extra: int = 0):
+    """Reassemble (cp[R] float32, summary bytes[R*A*32]) ordered by global replica id
+    (plus the extra bytes [R, extra] when extra > 0)."""
     slots = gathered.shape[0] // world
     rows = []
     for k in range(world):
@@ -60,5 +66,8 @@ def unpack_records(gathered: torch.Tensor, R: int, world: int, n_arch: int):
         rows.append(gathered[k * slots:k * slots + c])
     g = torch.cat(rows, 0) if rows else gathered[:0]
     cp = g[:, :4].contiguous().view(torch.float32).reshape(-1)
-    summ = g[:, 4:].contiguous().reshape(-1)
+    q = 4 + n_arch * SUMMARY_BYTES
+    summ = g[:, 4:q].contiguous().reshape(-1)
+    if extra:
+        return cp, summ, g[:, q:q + extra].contiguous()
     return cp, summ

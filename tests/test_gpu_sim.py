@@ -32,7 +32,7 @@ def to_dev(a, dtype=None):
 
 def _same_stats(g, o, A):
     assert g["makespan"] == o["makespan"], (g["makespan"], o["makespan"])
-    for f in ("pops", "evictions", "stale", "rounds"):
+    for f in ("pops", "evictions", "dups", "rounds"):
         assert g[f] == o[f], (f, g[f], o[f])
     assert g["busy"][:A].tobytes() == o["busy"][:A].tobytes()
     assert np.array_equal(g["ran"][:A], o["ran"][:A])

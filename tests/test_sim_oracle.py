@@ -63,7 +63,7 @@ def test_hand_worked_schedules(case):
     assert start.tolist() == case["start"]
     assert worker.tolist() == case["worker"]
     assert st["makespan"] == case["makespan"]
-    assert (st["evictions"], st["stale"], st["rounds"]) == (case["evictions"], case["stale"], case["rounds"])
+    assert (st["evictions"], st["dups"], st["rounds"]) == (case["evictions"], case["dups"], case["rounds"])
     assert st["busy"][:2].tolist() == case["busy"] and st["ran"][:2].tolist() == case["ran"]
     assert st["pops"] == len(dur)
 
@@ -135,7 +135,7 @@ def _check_trace(dag, dur, workers, st, start, worker):
         assert st["ran"][a] == int((arch == a).sum())
         assert st["busy"][a] == float(d[arch == a].sum())    # dyadic: exact
     ent = int(sum(np.sum(~np.isinf(dur[:, a])) for a in range(A) if workers[a] > 0))
-    assert st["pops"] + st["evictions"] + st["stale"] <= ent
+    assert st["pops"] + st["evictions"] + st["dups"] <= ent
     return arch, fin
 
 
@@ -172,6 +172,9 @@ def test_no_eviction_greedy_and_priority_order(seed):
     workers = rng.integers(1, 4, A).astype(np.int32)
     st, start, worker = oracle.simulate_dag(dag, dur, workers, 4, eviction=False)
     arch, fin = _check_trace(dag, dur, workers, st, start, worker)
+    # without eviction every task sits in all its enabled heaps until popped,
+    # so a pop leaves exactly (enabled archs - 1) duplicates (P:l.130)
+    assert st["dups"] == int(np.sum(np.isfinite(dur).sum(1) - 1))
     key = oracle.score_and_queue(dag, dur, workers)["key"]
     preds = _preds(dag)
     ready_at = np.array([max((fin[p] for p in ps), default=0.0) for ps in preds])
