@@ -73,6 +73,7 @@ struct SimShared {              // per-warp counters
     int32_t count[8];               // ready_tasks_count
     int32_t ran[8];
     uint32_t again[SIM_MAX_WORKERS / 32];
+    int64_t qoff[8];                // queue a's offset in the instance's queues
 };
 
 MP_INLINE void sub128_atomic(unsigned long long* p, uint64_t lo, uint64_t hi) {
@@ -207,6 +208,7 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
             int64_t o = 0;
             for (int a = 0; a < A; ++a) {
                 int32_t c = g.sum[(int64_t)rl * A + a].count;
+                if (lane == 0) sh.qoff[a] = o;
                 const int32_t* qa = q + o;
                 for (int32_t p = lane; p < c; p += 32) {
                     int32_t t = qa[p];
@@ -234,6 +236,9 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                 if (lane == 0) sh.again[gi] = m;
             }
             __syncwarp();
+            // heaps only shrink during a dispatch, so once a POP finds heap a
+            // empty every later POP on a in this dispatch returns nothing too
+            uint32_t empty = 0;
             for (bool any = true; any;) {
                 any = false;
                 for (int gi = 0; gi * 32 < W; ++gi) {
@@ -243,10 +248,13 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                         m &= m - 1;
                         int a = 0;
                         while (a + 1 < A && w >= g.wcum[a + 1]) ++a;
+                        if ((empty >> a) & 1u) {
+                            if (lane == 0) sh.again[gi] &= ~(1u << (w & 31));
+                            __syncwarp();
+                            continue;
+                        }
                         uint32_t* bm = bits + a * g.bm_words;
-                        int64_t qoff = 0;
-                        for (int b = 0; b < a; ++b) qoff += g.sum[(int64_t)rl * A + b].count;
-                        const int32_t* qa = q + qoff;
+                        const int32_t* qa = q + sh.qoff[a];
                         // ---- Alg. 2 POP
                         int tries = 0;
                         bool hit = false;
@@ -255,7 +263,7 @@ __global__ void __launch_bounds__(32) k_sim(SimArgs g) {
                         for (;;) {
                             if (tries >= g.max_tries) { hit = true; break; }
                             int32_t p = bm_first(bm, g, lane);
-                            if (p < 0) break;
+                            if (p < 0) { empty |= 1u << a; break; }
                             int32_t t = qa[p];
                             const uint32_t* rc = rec + (size_t)t * S;
                             uint32_t masks = rc[REC_MASK];
