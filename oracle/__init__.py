@@ -67,7 +67,7 @@ def lib():
         _lib.or_perturb.argtypes = [i32, i32, P, u64, f32, i64, P]
         _lib.or_perturb.restype = None
         _lib.or_replica.argtypes = [i32, i32, P, P, P, P, P, u64, f32, i64, P, P, P, P]
-        _lib.or_simulate.argtypes = [i32, i32, P, P, P, P, P, P, i32, i32, P, P, P]
+        _lib.or_simulate.argtypes = [i32, i32, P, P, P, P, P, P, P, P, P, P, P]
     return _lib
 
 
@@ -224,16 +224,34 @@ def score_and_queue(dag: Dag, dur, workers, kind=CRIT_BL, done=None):
 # discrete-event MultiPrio simulation (mp_sim_oracle.c)
 # --------------------------------------------------------------------------
 SIM_STATS_DTYPE = np.dtype([("makespan", "<f8"), ("pops", "<i8"), ("evictions", "<i8"), ("dups", "<i8"),
-                            ("rounds", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
+                            ("rounds", "<i8"), ("moved", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
 SIM_ERR_STUCK = 6
 
 
-def simulate(dag: Dag, dur, workers, key, max_tries=16, eviction=True, trace=True):
+class _SimCfg(C.Structure):
+    _fields_ = [("max_tries", C.c_int32), ("eviction", C.c_int32), ("top_n", C.c_int32), ("eps", C.c_float),
+                ("n_handles", C.c_int32), ("n_nodes", C.c_int32), ("acc_ptr", C.c_void_p), ("acc_h", C.c_void_p),
+                ("acc_mode", C.c_void_p), ("size", C.c_void_p), ("worker_node", C.c_void_p),
+                ("xfer_ms_per_byte", C.c_double)]
+
+
+@dataclass
+class DataModel:
+    """N3 data model: per-task accesses (CSR), handle sizes (bytes)."""
+    acc_ptr: np.ndarray      # int64[n+1]
+    acc_handle: np.ndarray   # int32[acc]
+    acc_mode: np.ndarray     # uint8[acc]: 1 = R, 2 = W, 3 = RW
+    size: np.ndarray         # uint64[H]
+
+
+def simulate(dag: Dag, dur, workers, key, max_tries=16, eviction=True, trace=True, gain=None, data=None,
+             top_n=1, eps=0.8, worker_node=None, xfer_ms_per_byte=0.0):
     """PUSH (Alg. 1) / POP (Alg. 2) simulation of one DAG instance.
 
     dur: canonical durations (check_durations / perturbed), key: the a7 keys
-    that order the heaps.  Returns (stats record, start[n] or None,
-    worker[n] or None)."""
+    that order the heaps, gain: eq. 1 gains (N3 epsilon filter), data: a
+    DataModel (N3 LS_SDH^2 and residency).  Returns (stats record,
+    start[n] or None, worker[n] or None)."""
     dur = _c(dur, np.float32)
     n, A = dur.shape
     key = _c(key, np.uint64).reshape(n, A)
@@ -241,22 +259,40 @@ def simulate(dag: Dag, dur, workers, key, max_tries=16, eviction=True, trace=Tru
     start = np.zeros(max(n, 1), np.float64) if trace else None
     worker = np.zeros(max(n, 1), np.int32) if trace else None
     indeg = _c(dag.indeg, np.int32) if n else np.zeros(1, np.int32)
+    keep = []
+
+    def arr(a, dt):
+        if a is None:
+            return None
+        a = _c(a, dt)
+        keep.append(a)
+        return _p(a)
+
+    cfg = _SimCfg(int(max_tries), int(bool(eviction)), int(top_n), float(eps),
+                  0 if data is None else int(len(data.size)), 0,
+                  None if data is None else arr(data.acc_ptr, np.int64),
+                  None if data is None else arr(data.acc_handle, np.int32),
+                  None if data is None else arr(data.acc_mode, np.uint8),
+                  None if data is None else arr(data.size, np.uint64),
+                  arr(worker_node, np.int32), float(xfer_ms_per_byte))
+    g = None if gain is None else _c(gain, np.float32).reshape(n, A)
     rc = lib().or_simulate(n, A, _p(dag.row_ptr), _p(dag.col if dag.n_edges else np.zeros(1, np.int32)),
-                           _p(indeg), _p(dur), _p(_c(workers, np.int32)), _p(key), int(max_tries),
-                           int(bool(eviction)), _p(st), _p(start), _p(worker))
+                           _p(indeg), _p(dur), _p(_c(workers, np.int32)), _p(key), _p(g), C.byref(cfg),
+                           _p(st), _p(start), _p(worker))
     if rc:
         raise OracleError(rc, "simulate")
     return st[0], (start[:n] if trace else None), (worker[:n] if trace else None)
 
 
-def simulate_dag(dag: Dag, dur, workers, max_tries=16, eviction=True, kind=CRIT_BL, trace=True):
-    """Score the whole DAG (a3-a7), then simulate it (convenience for tests)."""
+def simulate_dag(dag: Dag, dur, workers, max_tries=16, eviction=True, kind=CRIT_BL, trace=True, **loc):
+    """Score the whole DAG (a3-a7), then simulate it (convenience for tests).
+    loc: data / top_n / eps / worker_node / xfer_ms_per_byte (N3)."""
     r = score_and_queue(dag, dur, workers, kind=kind)
     dc = check_durations(dur, workers)
-    return simulate(dag, dc, workers, r["key"], max_tries, eviction, trace)
+    return simulate(dag, dc, workers, r["key"], max_tries, eviction, trace, gain=r["gain"], **loc)
 
 
-def simulate_replica(dag: Dag, base, workers, seed, sigma, r, max_tries=16, eviction=True, trace=True):
+def simulate_replica(dag: Dag, base, workers, seed, sigma, r, max_tries=16, eviction=True, trace=True, **loc):
     """Replica r (a10 perturbation, BL criticality, ALL-mode scores), simulated."""
     d = check_durations(perturb(base, seed, sigma, r), workers)
-    return simulate_dag(dag, d, workers, max_tries, eviction, CRIT_BL, trace)
+    return simulate_dag(dag, d, workers, max_tries, eviction, CRIT_BL, trace, **loc)

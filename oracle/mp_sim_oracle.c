@@ -14,7 +14,13 @@
  * i.e. by the a7 key ascending, ties by task id (reading c12); the CUDA path
  * uses rank bitmaps instead.
  *
- * Readings (s1-s9) are cited inline as "sN".
+ * Row N3 is the data-locality pick of POP: get_most_local_
+ * prio_task (§V-C, P:l.205-212) scores the first n heap entries whose score
+ * is within epsilon of the root's with LS_SDH^2 (eq. 3, P:l.209) on the
+ * worker's memory node, given per-task data accesses, handle sizes and a
+ * residency state that task starts update (readings l1-l6).
+ *
+ * Readings (s1-s9, l1-l6) are cited inline as "sN" / "lN".
  *
  * Pins (tests/test_oracle_pins.py, "sim" tests): hand-worked schedules of
  * Table II's tasks (P:l.180-187) with and without eviction, the closed forms
@@ -39,6 +45,7 @@ typedef struct {             /* per simulated instance                         *
     int64_t evictions;       /* heaps_evict_task calls (Alg. 2)                */
     int64_t dups;            /* duplicates a pop leaves in other heaps (P:l.130) */
     int64_t rounds;          /* POP calls that ended on MAX_TRIES              */
+    int64_t moved;           /* bytes of accessed data not resident at start   */
     double busy[8];          /* sum of delta(t,a) over tasks run on arch a     */
     int32_t ran[8];          /* tasks run on arch a                            */
 } so_stats;
@@ -105,6 +112,16 @@ typedef struct {
     int64_t count[8];        /* ready_tasks_count (Alg. 1)                     */
     u128 brw[8];             /* best_remaining_work (Alg. 1), exact            */
     int max_tries, eviction;
+    /* N3 data locality (eq. 3) */
+    const float* gain;       /* [n][A] eq. 1 gains (the heaps' first score)    */
+    int top_n;               /* n of P:l.238 (<= 1: the root)                  */
+    float eps;               /* epsilon of P:l.238                             */
+    const int64_t* acc_ptr;  /* [n+1] data accesses of each task, or NULL      */
+    const int32_t* acc_h;    /* handle                                         */
+    const uint8_t* acc_mode; /* bit0 read, bit1 write (R = 1, W = 2, RW = 3)   */
+    const uint64_t* size;    /* [H] bytes                                      */
+    int32_t H, M;            /* handles, memory nodes                          */
+    uint8_t* resident;       /* [M][H]                                         */
 } sched;
 
 static int en(const sched* s, int32_t t, int32_t a) {
@@ -154,21 +171,68 @@ static void uncount(sched* s, int32_t t) {
     }
 }
 
-/* Alg. 2 POP for a worker of arch a (memory node w_m of type a, reading
- * c13).  Returns the task, or -1; *hit_max = 1 when MAX_TRIES ended it. */
-static int32_t pop(sched* s, int32_t a, so_stats* st, int* hit_max) {
+/* eq. 3 (P:l.209): LS_SDH^2(m,t) = sum of the sizes of t's data resident on
+ * m accessed in read mode + sum of the squared sizes of those accessed in
+ * write mode (a RW access counts as write, l2). */
+static uint64_t ls_sdh2(const sched* s, int32_t m, int32_t t) {
+    uint64_t v = 0;
+    if (!s->acc_ptr) return 0;
+    for (int64_t i = s->acc_ptr[t]; i < s->acc_ptr[t + 1]; i++) {
+        int32_t hd = s->acc_h[i];
+        if (!s->resident[(int64_t)m * s->H + hd]) continue;
+        uint64_t z = s->size[hd];
+        v += (s->acc_mode[i] & 2) ? z * z : z;
+    }
+    return v;
+}
+
+/* get_most_local_prio_task (§V-C, P:l.205-212): among the first top_n live
+ * entries of heap a in priority order whose gain is within eps of the
+ * root's (l1), the one with the largest LS_SDH^2 on memory node m, ties to
+ * the higher priority (l3).  On the binary heap: pop the candidates, put
+ * back the ones not chosen.  Processed duplicates met on the way are dropped
+ * (s5).  Returns the chosen task, already removed from the heap, or -1. */
+static int32_t take_most_local(sched* s, int32_t a, int32_t m) {
     heap* h = &s->h[a];
+    int32_t cand[64];
+    int k = 0, kmax = s->top_n > 1 ? s->top_n : 1;
+    float g0 = 0.0f;
+    while (k < kmax && h->size > 0) {
+        int32_t t = h->v[0];
+        heap_pop_root(h);
+        if (s->started[t]) continue;
+        float g = s->gain ? s->gain[(int64_t)t * s->A + a] : 0.0f;
+        if (k == 0) g0 = g;
+        else {
+            float diff = g0 - g;                   /* one RN binary32 op */
+            if (!(diff <= s->eps)) { heap_insert(h, t); break; }
+        }
+        cand[k++] = t;
+    }
+    if (k == 0) return -1;
+    int b = 0;
+    if (k > 1) {
+        uint64_t bv = ls_sdh2(s, m, cand[0]);
+        for (int i = 1; i < k; i++) {
+            uint64_t v = ls_sdh2(s, m, cand[i]);
+            if (v > bv) { bv = v; b = i; }
+        }
+    }
+    for (int i = 0; i < k; i++)
+        if (i != b) heap_insert(h, cand[i]);
+    return cand[b];
+}
+
+/* Alg. 2 POP for a worker of arch a on memory node m (heaps per arch,
+ * reading c13).  Returns the task, or -1; *hit_max = 1 when MAX_TRIES ended
+ * it. */
+static int32_t pop(sched* s, int32_t a, int32_t m, so_stats* st, int* hit_max) {
     int tries = 0;
     *hit_max = 0;
     while (tries < s->max_tries) {
-        if (h->size == 0) return -1;
-        int32_t t = h->v[0];                       /* get_most_local_prio_task: */
-        if (s->started[t]) {                       /* the heap root (s6)        */
-            heap_pop_root(h);                      /* processed duplicate:      */
-            continue;                              /* removed, not a try (s5)   */
-        }
-        if (pop_condition(s, t, a)) {
-            heap_pop_root(h);                      /* heaps_pop_and_update      */
+        int32_t t = take_most_local(s, a, m);      /* already off heap a */
+        if (t < 0) return -1;
+        if (pop_condition(s, t, a)) {              /* heaps_pop_and_update      */
             for (int32_t b = 0; b < s->A; b++)     /* "any duplicate tasks in   */
                 if (b != a && s->counted[(int64_t)t * s->A + b])   /* other     */
                     st->dups += 1;                 /* queues will remain there" */
@@ -177,8 +241,7 @@ static int32_t pop(sched* s, int32_t a, so_stats* st, int* hit_max) {
             st->pops += 1;
             return t;
         }
-        heap_pop_root(h);                          /* heaps_evict_task          */
-        s->counted[(int64_t)t * s->A + a] = 0;
+        s->counted[(int64_t)t * s->A + a] = 0;    /* heaps_evict_task          */
         s->count[a] -= 1;                          /* t is not best on a        */
         st->evictions += 1;
         tries += 1;
@@ -187,17 +250,34 @@ static int32_t pop(sched* s, int32_t a, so_stats* st, int* hit_max) {
     return -1;
 }
 
+typedef struct {               /* simulation options                            */
+    int32_t max_tries;         /* MAX_TRIES (s7), >= 1                           */
+    int32_t eviction;          /* pop_condition on (1) / off (0)                 */
+    int32_t top_n;             /* N3 candidates n (P:l.238: 10); <= 1 = root     */
+    float eps;                 /* N3 epsilon (P:l.238: 0.8)                      */
+    int32_t n_handles;         /* H                                              */
+    int32_t n_nodes;           /* M (0 = default, l5)                            */
+    const int64_t* acc_ptr;    /* [n+1] or NULL = no data model                  */
+    const int32_t* acc_h;      /* [acc]                                          */
+    const uint8_t* acc_mode;   /* [acc] 1 = R, 2 = W, 3 = RW                     */
+    const uint64_t* size;      /* [H] bytes, < 2^28                              */
+    const int32_t* worker_node;/* [W] or NULL = default (l5)                     */
+    double xfer_ms_per_byte;   /* transfer time of non-resident data (l6)        */
+} so_config;
+
 /*
  * Inputs: the DAG (successor CSR, indeg), canonical durations dur[n][A]
- * (already perturbed for a replica), workers[A], the a7 keys key[n][A],
- * max_tries >= 1, eviction in {0,1}.  Workers are numbered arch-major
- * (workers[0] workers of arch 0 first, ...) (s2).  Outputs: *st, and if not
- * NULL start[n] (ms) and worker[n].
+ * (already perturbed for a replica), workers[A], the a7 keys key[n][A], the
+ * eq. 1 gains gain[n][A] (used by the N3 epsilon filter; may be NULL when
+ * top_n <= 1), options *cfg.  Workers are numbered arch-major (workers[0]
+ * workers of arch 0 first, ...) (s2).  Outputs: *st, and if not NULL
+ * start[n] (ms) and worker[n].
  */
 int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col, const int32_t* indeg,
-                const float* dur, const int32_t* workers, const uint64_t* key, int32_t max_tries,
-                int32_t eviction, so_stats* st, double* start, int32_t* worker) {
-    if (n < 0 || A < 1 || A > 8 || max_tries < 1) return SO_ERR_ARG;
+                const float* dur, const int32_t* workers, const uint64_t* key, const float* gain,
+                const so_config* cfg, so_stats* st, double* start, int32_t* worker) {
+    if (n < 0 || A < 1 || A > 8 || !cfg || cfg->max_tries < 1 || cfg->top_n > 64) return SO_ERR_ARG;
+    if (cfg->top_n > 1 && !gain) return SO_ERR_ARG;
     int32_t W = 0;
     for (int32_t a = 0; a < A; a++) W += workers[a] > 0 ? workers[a] : 0;
     if (W < 1) return SO_ERR_ARG;
@@ -205,7 +285,10 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
     sched s;
     memset(&s, 0, sizeof(s));
     s.n = n; s.A = A; s.W = W; s.row_ptr = row_ptr; s.col = col; s.dur = dur; s.workers = workers;
-    s.max_tries = max_tries; s.eviction = eviction;
+    s.max_tries = cfg->max_tries; s.eviction = cfg->eviction;
+    s.gain = gain; s.top_n = cfg->top_n; s.eps = cfg->eps;
+    s.acc_ptr = cfg->acc_ptr; s.acc_h = cfg->acc_h; s.acc_mode = cfg->acc_mode; s.size = cfg->size;
+    s.H = cfg->acc_ptr ? cfg->n_handles : 0;
     size_t nn = (size_t)n + 1;
     s.counted = (uint8_t*)calloc(nn * (size_t)A, 1);
     s.started = (uint8_t*)calloc(nn, 1);
@@ -214,6 +297,7 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
     int32_t* wtask = (int32_t*)malloc((size_t)W * sizeof(int32_t));
     double* wend = (double*)malloc((size_t)W * sizeof(double));
     uint8_t* again = (uint8_t*)malloc((size_t)W);
+    int32_t* wnode = (int32_t*)malloc((size_t)W * sizeof(int32_t));
     u128 busy[8] = {0};
     int rc = SO_ERR_NOMEM;
     for (int32_t a = 0; a < A; a++) {
@@ -221,9 +305,22 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
         s.h[a].key = key; s.h[a].A = A; s.h[a].a = a;
         if (!s.h[a].v) goto out;
     }
-    if (!s.counted || !s.started || !s.rem || !warch || !wtask || !wend || !again) goto out;
+    if (!s.counted || !s.started || !s.rem || !warch || !wtask || !wend || !again || !wnode) goto out;
     for (int32_t a = 0, w = 0; a < A; a++)
         for (int32_t k = 0; k < workers[a]; k++, w++) { warch[w] = a; wtask[w] = -1; wend[w] = 0.0; }
+    /* memory nodes (l5): given, or arch-0 workers share node 0 and every
+     * other worker has its own node */
+    s.M = 0;
+    for (int32_t w = 0; w < W; w++) {
+        wnode[w] = cfg->worker_node ? cfg->worker_node[w] : (warch[w] == 0 ? 0 : 1 + w - workers[0]);
+        if (wnode[w] < 0) { rc = SO_ERR_ARG; goto out; }
+        if (wnode[w] + 1 > s.M) s.M = wnode[w] + 1;
+    }
+    if (cfg->n_nodes > s.M) s.M = cfg->n_nodes;
+    /* every handle starts in main memory, node 0 (l4) */
+    s.resident = (uint8_t*)calloc((size_t)s.M * (size_t)(s.H > 0 ? s.H : 1), 1);
+    if (!s.resident) goto out;
+    for (int32_t hd = 0; hd < s.H; hd++) s.resident[hd] = 1;
 
     /* time 0: every task without predecessors is ready (P:l.91) */
     for (int32_t t = 0; t < n; t++) {
@@ -242,15 +339,29 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
             for (int32_t w = 0; w < W; w++) {
                 if (!again[w]) continue;
                 int hit;
-                int32_t t = pop(&s, warch[w], st, &hit);
+                int32_t t = pop(&s, warch[w], wnode[w], st, &hit);
                 again[w] = (uint8_t)hit;
                 any |= hit;
                 if (hit) st->rounds += 1;
                 if (t >= 0) {
-                    int32_t a = warch[w];
+                    int32_t a = warch[w], m = wnode[w];
                     float d = dur[(int64_t)t * A + a];
+                    /* data of t moves to node m; a write leaves m the only copy (l4) */
+                    uint64_t miss = 0;
+                    if (s.acc_ptr) {
+                        for (int64_t i = s.acc_ptr[t]; i < s.acc_ptr[t + 1]; i++)
+                            if (!s.resident[(int64_t)m * s.H + s.acc_h[i]]) miss += s.size[s.acc_h[i]];
+                        for (int64_t i = s.acc_ptr[t]; i < s.acc_ptr[t + 1]; i++) {
+                            int32_t hd = s.acc_h[i];
+                            if (s.acc_mode[i] & 2)
+                                for (int32_t m2 = 0; m2 < s.M; m2++) s.resident[(int64_t)m2 * s.H + hd] = 0;
+                            s.resident[(int64_t)m * s.H + hd] = 1;
+                        }
+                    }
+                    st->moved += (int64_t)miss;
+                    double x = (double)miss * cfg->xfer_ms_per_byte;    /* l6 */
                     wtask[w] = t;
-                    wend[w] = T + (double)d;              /* s1 */
+                    wend[w] = T + ((double)d + x);          /* s1 */
                     if (start) start[t] = T;
                     if (worker) worker[t] = w;
                     busy[a] += fx(d);
@@ -281,5 +392,6 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
 out:
     for (int32_t a = 0; a < A; a++) free(s.h[a].v);
     free(s.counted); free(s.started); free(s.rem); free(warch); free(wtask); free(wend); free(again);
+    free(wnode); free(s.resident);
     return rc;
 }

@@ -218,3 +218,123 @@ def test_sim_argument_errors():
     dur = np.ones((2, 1), np.float32)
     with pytest.raises(oracle.OracleError):
         oracle.simulate_dag(dag, dur, [1], max_tries=0)
+
+
+# ----------------------------------------------------------------------------
+# N3: data locality (LS_SDH^2, eq. 3, P:l.205-212), readings l1-l6
+# ----------------------------------------------------------------------------
+
+@pytest.mark.parametrize("case", json.load(open(os.path.join(GOLD, "sim_worked.json")))["locality_cases"],
+                         ids=lambda c: c["name"])
+def test_locality_hand_worked(case):
+    dur = np.array(case["dur_ms"], np.float32)
+    dag = _dag(len(dur), case["edges"])
+    dm = oracle.DataModel(np.array(case["acc_ptr"]), np.array(case["acc_handle"]), np.array(case["acc_mode"]),
+                          np.array(case["size"]))
+    st, start, worker = oracle.simulate_dag(dag, dur, case["workers"], data=dm, top_n=case["top_n"],
+                                            eps=case["eps"], xfer_ms_per_byte=case["xfer_ms_per_byte"])
+    assert start.tolist() == case["start"] and worker.tolist() == case["worker"]
+    assert st["makespan"] == case["makespan"] and st["moved"] == case["moved"]
+
+
+def _data(n, seed, H=12):
+    return oracle.DataModel(*random_dags.random_data_model(n, H, seed, max_size=1 << 12))
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_locality_top1_equals_plain_schedule(seed):
+    """n = 1 candidate and free transfers: the pick is the heap root, so the
+    schedule is the plain N2 one whatever the data model."""
+    n = 60
+    src, dst = random_dags.random_dag(n, 1.5, seed)
+    dag = oracle.build_dag(n, src, dst)
+    dur = random_dags.dyadic_durations(n, 2, seed, p_inf=0.2)
+    a = oracle.simulate_dag(dag, dur, [2, 1], 3, bool(seed % 2))
+    b = oracle.simulate_dag(dag, dur, [2, 1], 3, bool(seed % 2), data=_data(n, seed), top_n=1)
+    assert np.array_equal(a[1], b[1]) and np.array_equal(a[2], b[2])
+    assert a[0]["makespan"] == b[0]["makespan"]
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_locality_replay(seed):
+    """Replay the schedule independently of the heaps (eviction off, so heap a
+    holds exactly the ready, unstarted tasks enabled on a): at every start, in
+    (time, worker) order, the task must be the max-LS_SDH^2 candidate among
+    the first n in (key, id) order whose gain is within eps of the first
+    (ties to the earlier), on the worker's node (arch-0 workers node 0, the
+    others one node each); residency follows reads (copy) and writes (only
+    copy); finish = start + (delta + missing bytes x cost)."""
+    rng = np.random.default_rng(900 + seed)
+    n = int(rng.integers(20, 90))
+    A = int(rng.integers(1, 4))
+    src, dst = random_dags.random_dag(n, float(rng.uniform(0.5, 2.5)), seed)
+    dag = oracle.build_dag(n, src, dst)
+    dur = random_dags.dyadic_durations(n, A, seed, p_inf=0.25, tiny_set=bool(seed % 3 == 0))
+    workers = rng.integers(1, 3, A).astype(np.int32)
+    H = int(rng.integers(2, 10))
+    dm = _data(n, seed, H)
+    top_n = int(rng.integers(2, 8))
+    eps = float(np.float32(rng.choice([0.0, 0.25, 0.8, 1.0])))
+    cost = float(rng.choice([0.0, 2.0 ** -10]))
+    st, start, worker = oracle.simulate_dag(dag, dur, workers, 4, False, data=dm, top_n=top_n, eps=eps,
+                                            xfer_ms_per_byte=cost)
+    r = oracle.score_and_queue(dag, dur, workers)
+    key, gain = r["key"], r["gain"]
+    wa = np.repeat(np.arange(A), workers)
+    W0 = int(workers[0])
+    node = np.array([0 if wa[w] == 0 else 1 + w - W0 for w in range(len(wa))])
+    M = int(node.max()) + 1
+    res = np.zeros((M, H), bool)
+    res[0] = True
+    preds = _preds(dag)
+    fin = np.full(n, np.inf)
+    started = np.zeros(n, bool)
+    moved = 0
+    for t in sorted(range(n), key=lambda t: (start[t], worker[t])):
+        w, T = int(worker[t]), start[t]
+        a, m = int(wa[w]), int(node[w])
+        ready = [u for u in range(n) if not started[u] and np.isfinite(dur[u, a])
+                 and all(fin[p] <= T for p in preds[u])]
+        ready.sort(key=lambda u: (int(key[u, a]), u))
+        cand = []
+        for u in ready[:top_n]:
+            if cand and not (np.float32(gain[cand[0], a]) - np.float32(gain[u, a]) <= np.float32(eps)):
+                break
+            cand.append(u)
+
+        def ls(u):
+            v = 0
+            for i in range(dm.acc_ptr[u], dm.acc_ptr[u + 1]):
+                h = int(dm.acc_handle[i])
+                if res[m, h]:
+                    z = int(dm.size[h])
+                    v += z * z if dm.acc_mode[i] & 2 else z
+            return v
+
+        best = max(cand, key=lambda u: (ls(u), -cand.index(u)))
+        assert t == best, (t, cand)
+        miss = 0
+        for i in range(dm.acc_ptr[t], dm.acc_ptr[t + 1]):
+            h = int(dm.acc_handle[i])
+            if not res[m, h]:
+                miss += int(dm.size[h])
+        for i in range(dm.acc_ptr[t], dm.acc_ptr[t + 1]):
+            h = int(dm.acc_handle[i])
+            if dm.acc_mode[i] & 2:
+                res[:, h] = False
+            res[m, h] = True
+        moved += miss
+        started[t] = True
+        fin[t] = T + (float(dur[t, a]) + miss * cost)
+    assert st["moved"] == moved and st["makespan"] == fin.max()
+
+
+def test_locality_reduces_transfers_cholesky():
+    """The point of §V-C: with n = 10, eps = 0.8 (P:l.238) the pick moves
+    fewer tiles than the heap root on a tiled Cholesky (2 GPUs, 30 CPUs)."""
+    w = workloads.cholesky(16)
+    dag = oracle.build_dag(w.n, w.src, w.dst)
+    dm = oracle.DataModel(w.acc_ptr, w.acc_handle, w.acc_mode, w.handle_size)
+    root = oracle.simulate_dag(dag, w.dur, [30, 2], data=dm, top_n=1, trace=False)[0]
+    loc = oracle.simulate_dag(dag, w.dur, [30, 2], data=dm, top_n=10, eps=0.8, trace=False)[0]
+    assert loc["moved"] < root["moved"]

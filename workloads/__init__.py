@@ -70,6 +70,11 @@ class Workload:
     workers: np.ndarray      # int32[A], >0 enables the arch
     kind: np.ndarray | None = None
     meta: dict = field(default_factory=dict)
+    # N3 data model (STF workloads): accesses per task and handle sizes in bytes
+    acc_ptr: np.ndarray | None = None
+    acc_handle: np.ndarray | None = None
+    acc_mode: np.ndarray | None = None
+    handle_size: np.ndarray | None = None
 
     @property
     def n_arch(self) -> int:
@@ -85,12 +90,19 @@ def _table(kind: np.ndarray, model: dict) -> np.ndarray:
     return np.ascontiguousarray(tab[kind])
 
 
+# tile of the paper's Chameleon runs: 960 x 960 doubles
+TILE_BYTES = 960 * 960 * 8
+
+
 def _from_stf(name, s: STFRecorder, model, arch_names, **meta) -> Workload:
     src, dst = s.edges()
     kind = s.kinds()
     dur = _table(kind, model)
+    ap, ah, am = s.accesses()
+    H = int(ah.max()) + 1 if len(ah) else 0
     return Workload(name, s.n, src, dst, dur, arch_names,
-                    np.ones(dur.shape[1], np.int32), kind, dict(meta))
+                    np.ones(dur.shape[1], np.int32), kind, dict(meta),
+                    ap, ah, am, np.full(H, TILE_BYTES, np.uint64))
 
 
 def cholesky(N: int) -> Workload:

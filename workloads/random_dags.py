@@ -75,3 +75,23 @@ def dyadic_durations(n: int, A: int, seed: int, denom: int = 64, hi: int = 64,
         mask[np.arange(n), keep] = False
         d[mask] = np.inf
     return d.astype(np.float32)
+
+
+def random_data_model(n: int, H: int, seed: int, max_acc: int = 3, max_size: int = 1 << 20):
+    """Random N3 data model: each task accesses 0..max_acc distinct handles of
+    [0, H) in mode R (1), W (2) or RW (3); sizes are integers in [1, max_size].
+    Returns (acc_ptr int64[n+1], acc_handle int32[], acc_mode uint8[], size uint64[H])."""
+    rng = np.random.default_rng(seed)
+    k = rng.integers(0, max_acc + 1, n)
+    ptr = np.zeros(n + 1, np.int64)
+    ptr[1:] = np.cumsum(k)
+    hs, ms = [], []
+    for t in range(n):
+        h = rng.choice(H, size=min(int(k[t]), H), replace=False)
+        hs.append(h)
+        ms.append(rng.integers(1, 4, len(h)))
+    ptr[1:] = np.cumsum([len(h) for h in hs])
+    acc_h = np.concatenate(hs).astype(np.int32) if n else np.zeros(0, np.int32)
+    acc_m = np.concatenate(ms).astype(np.uint8) if n else np.zeros(0, np.uint8)
+    size = rng.integers(1, max_size + 1, H).astype(np.uint64)
+    return ptr, acc_h, acc_m, size

@@ -20,7 +20,7 @@ import numpy as np
 
 
 class STFRecorder:
-    __slots__ = ("n", "kind", "_src", "_dst", "_last_writer", "_readers")
+    __slots__ = ("n", "kind", "_src", "_dst", "_last_writer", "_readers", "_acc_h", "_acc_m", "_acc_ptr")
 
     def __init__(self) -> None:
         self.n = 0
@@ -29,6 +29,9 @@ class STFRecorder:
         self._dst: list[int] = []
         self._last_writer: dict = {}
         self._readers: dict = {}
+        self._acc_h: list[int] = []        # data accesses of every task
+        self._acc_m: list[int] = []        # 1 = R, 3 = RW
+        self._acc_ptr: list[int] = [0]
 
     def submit(self, kind: int, reads=(), writes=()) -> int:
         """Submit one task.  `reads` are R handles, `writes` are RW handles."""
@@ -40,6 +43,8 @@ class STFRecorder:
         src = self._src
         dst = self._dst
         for h in reads:
+            self._acc_h.append(h)
+            self._acc_m.append(1)
             lw = lw_map.get(h)
             if lw is not None:
                 src.append(lw)
@@ -50,6 +55,8 @@ class STFRecorder:
             else:
                 lst.append(t)
         for h in writes:
+            self._acc_h.append(h)
+            self._acc_m.append(3)
             lw = lw_map.get(h)
             if lw is not None:
                 src.append(lw)
@@ -62,6 +69,7 @@ class STFRecorder:
                         dst.append(t)
                 rd_map[h] = []
             lw_map[h] = t
+        self._acc_ptr.append(len(self._acc_h))
         return t
 
     def edges(self) -> tuple[np.ndarray, np.ndarray]:
@@ -70,3 +78,8 @@ class STFRecorder:
 
     def kinds(self) -> np.ndarray:
         return np.asarray(self.kind, dtype=np.int32)
+
+    def accesses(self) -> tuple[np.ndarray, np.ndarray, np.ndarray]:
+        """(acc_ptr int64[n+1], handle int32[acc], mode uint8[acc]; 1 = R, 3 = RW)."""
+        return (np.asarray(self._acc_ptr, dtype=np.int64), np.asarray(self._acc_h, dtype=np.int32),
+                np.asarray(self._acc_m, dtype=np.uint8))
