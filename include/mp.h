@@ -240,15 +240,55 @@ typedef struct {
     int64_t evictions; /* heaps_evict_task calls                             */
     int64_t dups;      /* duplicates a pop leaves in the other heaps (P:l.130) */
     int64_t rounds;    /* POP calls that ended on MAX_TRIES                  */
+    int64_t moved;     /* bytes of accessed data not resident at task starts */
     double busy[8];    /* sum of delta_r(t,a) over tasks run on arch a, exact */
                        /*   sum rounded once to binary64                     */
     int32_t ran[8];    /* tasks run on arch a                                */
-} mp_sim_stats;        /* 136 bytes */
+} mp_sim_stats;        /* 144 bytes */
 
 mp_status mp_simulate(mp_dag* dag, int32_t n_arch, const float* d_base_dur, const int32_t* h_workers,
                       uint64_t seed, float sigma, int64_t r0, int32_t R, const int32_t* d_qtask,
                       const mp_queue_summary* d_sum, int32_t max_tries, int32_t eviction,
                       mp_sim_stats* d_stats, double* d_start, int32_t* d_worker, void* stream);
+
+/*
+ * the same simulation with POP's data-locality pick,
+ * get_most_local_prio_task (§V-C, P:l.205-212): among the first top_n heap
+ * entries (priority order) whose gain is within eps of the root's
+ * (gain(root) - gain(t) <= eps, one binary32 subtraction; reading l1), the
+ * task with the largest LS_SDH^2(m, t) (eq. 3, P:l.209) on the popping
+ * worker's memory node m, ties to the higher priority (l3):
+ *   LS_SDH^2(m,t) = sum over t's accesses of data resident on m of
+ *                   size (mode R) or size^2 (mode W or RW, l2), exact uint64.
+ * Data model: d_acc_ptr int64[n+1], d_acc_handle int32[], d_acc_mode uint8[]
+ * (1 = R, 2 = W, 3 = RW) per task, d_size uint64[n_handles] bytes (< 2^28).
+ * Every handle starts resident on node 0 only; a task started on node m
+ * makes its data resident on m, and a write leaves m the only copy (l4).
+ * Memory nodes: h_worker_node[W] (NULL: arch-0 workers share node 0, every
+ * other worker has its own node 1, 2, ...; l5).  A task runs
+ * delta_r(t,a) (+) missing bytes x xfer_ms_per_byte (l6).
+ * top_n <= 1 and d_acc_ptr = NULL give mp_simulate; top_n <= 32; eps >= 0.
+ * The P:l.238 setting is top_n = 10, eps = 0.8.
+ */
+typedef struct {
+    int32_t max_tries;           /* MAX_TRIES (>= 1)                          */
+    int32_t eviction;            /* pop_condition on (1) / off (0)            */
+    int32_t top_n;               /* n of §V-C (<= 1: the heap root)           */
+    float eps;                   /* epsilon of §V-C                           */
+    int32_t n_handles;           /* data handles                              */
+    int32_t n_nodes;             /* memory nodes (0: from h_worker_node)      */
+    const int64_t* d_acc_ptr;    /* [n+1], or NULL: no data model             */
+    const int32_t* d_acc_handle; /* [acc]                                     */
+    const uint8_t* d_acc_mode;   /* [acc]                                     */
+    const uint64_t* d_size;      /* [n_handles]                               */
+    const int32_t* h_worker_node;/* [W] host, or NULL                         */
+    double xfer_ms_per_byte;     /* >= 0                                      */
+} mp_sim_config;
+
+mp_status mp_simulate_cfg(mp_dag* dag, int32_t n_arch, const float* d_base_dur, const int32_t* h_workers,
+                          uint64_t seed, float sigma, int64_t r0, int32_t R, const int32_t* d_qtask,
+                          const mp_queue_summary* d_sum, const mp_sim_config* cfg, mp_sim_stats* d_stats,
+                          double* d_start, int32_t* d_worker, void* stream);
 
 /* Synchronise `stream`, then return (and clear) the handle's device error
  * flag: MP_OK or MP_ERR_DOMAIN; MP_ERR_CUDA on a pending CUDA error. */

@@ -194,7 +194,7 @@ static uint64_t ls_sdh2(const sched* s, int32_t m, int32_t t) {
  * (s5).  Returns the chosen task, already removed from the heap, or -1. */
 static int32_t take_most_local(sched* s, int32_t a, int32_t m) {
     heap* h = &s->h[a];
-    int32_t cand[64];
+    int32_t cand[32];
     int k = 0, kmax = s->top_n > 1 ? s->top_n : 1;
     float g0 = 0.0f;
     while (k < kmax && h->size > 0) {
@@ -276,7 +276,7 @@ typedef struct {               /* simulation options                            
 int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col, const int32_t* indeg,
                 const float* dur, const int32_t* workers, const uint64_t* key, const float* gain,
                 const so_config* cfg, so_stats* st, double* start, int32_t* worker) {
-    if (n < 0 || A < 1 || A > 8 || !cfg || cfg->max_tries < 1 || cfg->top_n > 64) return SO_ERR_ARG;
+    if (n < 0 || A < 1 || A > 8 || !cfg || cfg->max_tries < 1 || cfg->top_n > 32) return SO_ERR_ARG;
     if (cfg->top_n > 1 && !gain) return SO_ERR_ARG;
     int32_t W = 0;
     for (int32_t a = 0; a < A; a++) W += workers[a] > 0 ? workers[a] : 0;

@@ -248,17 +248,30 @@ def queues_push(dag: Dag, key: torch.Tensor, flags: torch.Tensor, dur: torch.Ten
 
 
 SIM_STATS_DTYPE = np.dtype([("makespan", "<f8"), ("pops", "<i8"), ("evictions", "<i8"), ("dups", "<i8"),
-                            ("rounds", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
-SIM_STATS_BYTES = 136
+                            ("rounds", "<i8"), ("moved", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
+SIM_STATS_BYTES = 144
+
+
+class DataModel:
+    """N3 data model on the device: per-task accesses (CSR) and handle sizes (bytes)."""
+
+    def __init__(self, acc_ptr, acc_handle, acc_mode, size, device="cuda"):
+        self.acc_ptr = torch.as_tensor(np.asarray(acc_ptr, np.int64)).to(device)
+        self.acc_handle = torch.as_tensor(np.asarray(acc_handle, np.int32)).to(device)
+        self.acc_mode = torch.as_tensor(np.asarray(acc_mode, np.uint8)).to(device)
+        self.size = torch.as_tensor(np.asarray(size, np.uint64).view(np.int64)).to(device)
+        self.n_handles = int(self.size.numel())
 
 
 def simulate(dag: Dag, base_dur: torch.Tensor, workers, seed: int, sigma: float, r0: int, R: int,
              qtask: torch.Tensor, summary: torch.Tensor, max_tries: int = 16, eviction: bool = True,
-             trace: bool = False, out=None):
-    """N2 (mp_simulate): PUSH/POP simulation of R instances -> (stats bytes[R*136], start, worker).
+             trace: bool = False, out=None, data: DataModel | None = None, top_n: int = 1, eps: float = 0.8,
+             worker_node=None, xfer_ms_per_byte: float = 0.0):
+    """N2/N3 (mp_simulate_cfg): PUSH/POP simulation of R instances -> (stats bytes[R*144], start, worker).
 
     qtask/summary: the ALL-mode queues of mp_replicas_run ([R][n*A], [R*A*32])
-    or, for one DAG (R=1, r0=0, sigma=0), of mp_build_queues."""
+    or, for one DAG (R=1, r0=0, sigma=0), of mp_build_queues.  data/top_n/eps/
+    worker_node/xfer_ms_per_byte: N3 data locality (P:l.205-212, l.238)."""
     n, A = base_dur.shape
     w, wp = _workers(workers, A)
     dev = base_dur.device
@@ -266,10 +279,18 @@ def simulate(dag: Dag, base_dur: torch.Tensor, workers, seed: int, sigma: float,
         out = dict(stats=torch.empty(max(R, 1) * SIM_STATS_BYTES, dtype=torch.uint8, device=dev),
                    start=torch.empty((max(R, 1), n), dtype=torch.float64, device=dev) if trace else None,
                    worker=torch.empty((max(R, 1), n), dtype=torch.int32, device=dev) if trace else None)
-    rc = _lib.lib().mp_simulate(dag.handle, A, _ptr(base_dur), wp, C.c_uint64(seed), C.c_float(sigma), int(r0),
-                                int(R), _ptr(qtask), _ptr(summary), int(max_tries), int(bool(eviction)),
-                                _ptr(out["stats"]), _ptr(out.get("start")), _ptr(out.get("worker")), _stream())
-    _lib.check(rc, "mp_simulate")
+    wn = None if worker_node is None else np.ascontiguousarray(np.asarray(worker_node, np.int32))
+    cfg = _lib.mp_sim_config(int(max_tries), int(bool(eviction)), int(top_n), float(eps),
+                             0 if data is None else data.n_handles, 0,
+                             None if data is None else _ptr(data.acc_ptr),
+                             None if data is None or data.acc_handle.numel() == 0 else _ptr(data.acc_handle),
+                             None if data is None or data.acc_mode.numel() == 0 else _ptr(data.acc_mode),
+                             None if data is None or data.n_handles == 0 else _ptr(data.size),
+                             None if wn is None else wn.ctypes.data_as(C.c_void_p), float(xfer_ms_per_byte))
+    rc = _lib.lib().mp_simulate_cfg(dag.handle, A, _ptr(base_dur), wp, C.c_uint64(seed), C.c_float(sigma),
+                                    int(r0), int(R), _ptr(qtask), _ptr(summary), C.byref(cfg), _ptr(out["stats"]),
+                                    _ptr(out.get("start")), _ptr(out.get("worker")), _stream())
+    _lib.check(rc, "mp_simulate_cfg")
     return out["stats"], out.get("start"), out.get("worker")
 
 
@@ -279,10 +300,12 @@ def sim_stats(stats_bytes: torch.Tensor) -> np.ndarray:
 
 
 def replicas_simulate(dag: Dag, base_dur: torch.Tensor, workers, seed: int, sigma: float, r0: int, R: int,
-                      max_tries: int = 16, eviction: bool = True, trace: bool = False):
-    """a10 queues of R replicas (mp_replicas_run), then their simulation (mp_simulate)."""
+                      max_tries: int = 16, eviction: bool = True, trace: bool = False, **loc):
+    """a10 queues of R replicas (mp_replicas_run), then their simulation (mp_simulate_cfg).
+    loc: data / top_n / eps / worker_node / xfer_ms_per_byte (N3)."""
     cp, summ, q = replicas_run(dag, base_dur, workers, seed, sigma, r0, R, want_queues=True)
-    st, start, worker = simulate(dag, base_dur, workers, seed, sigma, r0, R, q, summ, max_tries, eviction, trace)
+    st, start, worker = simulate(dag, base_dur, workers, seed, sigma, r0, R, q, summ, max_tries, eviction, trace,
+                                 **loc)
     return dict(cp=cp, summary=summ, qtask=q, stats=st, start=start, worker=worker)
 
 

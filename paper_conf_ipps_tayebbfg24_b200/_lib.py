@@ -16,8 +16,8 @@ MP_CRIT_BOTTOM_LEVEL, MP_CRIT_NOD = 0, 1
 
 EXPORTS = (
     "mp_build_dag", "mp_dag_rebuild", "mp_dag_get_info", "mp_bottom_level", "mp_affinity", "mp_score",
-    "mp_build_queues", "mp_replicas_run", "mp_ready_init", "mp_queues_push", "mp_simulate", "mp_check", "mp_free", "mp_status_str",
-    "mp_last_error", "mp_build_info", "mp_launch_count", "mp_prof_enable", "mp_prof_reset", "mp_prof_query", "mp_prof_names",
+    "mp_build_queues", "mp_replicas_run", "mp_ready_init", "mp_queues_push", "mp_simulate", "mp_simulate_cfg",
+    "mp_check", "mp_free", "mp_status_str", "mp_last_error", "mp_build_info", "mp_launch_count", "mp_prof_enable", "mp_prof_reset", "mp_prof_query", "mp_prof_names",
 )
 
 
@@ -34,6 +34,13 @@ class mp_dag_info(C.Structure):
                 ("max_width", C.c_int32), ("d_row_ptr", C.c_void_p), ("d_col", C.c_void_p),
                 ("d_indeg", C.c_void_p), ("d_level", C.c_void_p), ("d_level_ptr", C.c_void_p),
                 ("d_level_order", C.c_void_p)]
+
+
+class mp_sim_config(C.Structure):
+    _fields_ = [("max_tries", C.c_int32), ("eviction", C.c_int32), ("top_n", C.c_int32), ("eps", C.c_float),
+                ("n_handles", C.c_int32), ("n_nodes", C.c_int32), ("d_acc_ptr", C.c_void_p),
+                ("d_acc_handle", C.c_void_p), ("d_acc_mode", C.c_void_p), ("d_size", C.c_void_p),
+                ("h_worker_node", C.c_void_p), ("xfer_ms_per_byte", C.c_double)]
 
 
 _lib = None
@@ -59,6 +66,7 @@ def lib():
     L.mp_ready_init.argtypes = [P, P, P]
     L.mp_queues_push.argtypes = [P, i32, P, P, P, P, i32, P, P, P, P, P, P, P]
     L.mp_simulate.argtypes = [P, i32, P, P, u64, f32, i64, i32, P, P, i32, i32, P, P, P, P]
+    L.mp_simulate_cfg.argtypes = [P, i32, P, P, u64, f32, i64, i32, P, P, C.POINTER(mp_sim_config), P, P, P, P]
     L.mp_check.argtypes = [P, P]
     L.mp_free.argtypes = [P]
     L.mp_free.restype = None

@@ -82,8 +82,21 @@ mp_status mp_simulate(mp_dag* dag, int32_t n_arch, const float* d_base_dur, cons
                       uint64_t seed, float sigma, int64_t r0, int32_t R, const int32_t* d_qtask,
                       const mp_queue_summary* d_sum, int32_t max_tries, int32_t eviction, mp_sim_stats* d_stats,
                       double* d_start, int32_t* d_worker, void* stream) {
-    return mph::simulate(dag, n_arch, d_base_dur, h_workers, seed, sigma, r0, R, d_qtask, d_sum, max_tries, eviction,
-                         d_stats, d_start, d_worker, as_stream(stream));
+    mp_sim_config cfg{};
+    cfg.max_tries = max_tries;
+    cfg.eviction = eviction;
+    cfg.top_n = 1;
+    cfg.eps = 0.0f;
+    return mph::simulate(dag, n_arch, d_base_dur, h_workers, seed, sigma, r0, R, d_qtask, d_sum, &cfg, d_stats,
+                         d_start, d_worker, as_stream(stream));
+}
+
+mp_status mp_simulate_cfg(mp_dag* dag, int32_t n_arch, const float* d_base_dur, const int32_t* h_workers,
+                          uint64_t seed, float sigma, int64_t r0, int32_t R, const int32_t* d_qtask,
+                          const mp_queue_summary* d_sum, const mp_sim_config* cfg, mp_sim_stats* d_stats,
+                          double* d_start, int32_t* d_worker, void* stream) {
+    return mph::simulate(dag, n_arch, d_base_dur, h_workers, seed, sigma, r0, R, d_qtask, d_sum, cfg, d_stats,
+                         d_start, d_worker, as_stream(stream));
 }
 
 mp_status mp_check(mp_dag* dag, void* stream) {

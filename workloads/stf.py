@@ -80,6 +80,10 @@ class STFRecorder:
         return np.asarray(self.kind, dtype=np.int32)
 
     def accesses(self) -> tuple[np.ndarray, np.ndarray, np.ndarray]:
-        """(acc_ptr int64[n+1], handle int32[acc], mode uint8[acc]; 1 = R, 3 = RW)."""
-        return (np.asarray(self._acc_ptr, dtype=np.int64), np.asarray(self._acc_h, dtype=np.int32),
+        """(acc_ptr int64[n+1], handle int32[acc], mode uint8[acc]; 1 = R, 3 = RW).
+        Handle keys are renumbered densely 0..H-1 in increasing key order."""
+        h = np.asarray(self._acc_h, dtype=np.int64)
+        if len(h) and (h.min() < 0 or h.max() >= len(h)):
+            _, h = np.unique(h, return_inverse=True)
+        return (np.asarray(self._acc_ptr, dtype=np.int64), h.astype(np.int32),
                 np.asarray(self._acc_m, dtype=np.uint8))
