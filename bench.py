@@ -39,6 +39,7 @@ METRIC = "DAG tasks scored+queued/sec and ms per DAG (1 GPU; replicas at 1/2/4/8
 METRIC_SIM = "DAG tasks scored+queued+scheduled (simulated PUSH/POP, N2)/sec and ms per DAG"
 SIM_WORKERS = (30, 2)   # Intel-V100 node: 32 cores, 2 GPUs, one core drives each GPU
 SIM_MAX_TRIES = 16
+LOC = dict(top_n=10, eps=0.8, xfer_ms_per_byte=2.0 ** -24)   # N3 (c5loc)
 UNIT = "tasks/s"
 CONFIG_TEXT = {
     "c1": "tiled Cholesky DAG 4x4 tiles (20 tasks), 2 resource types CPU/GPU, fixed durations",
@@ -49,6 +50,8 @@ CONFIG_TEXT = {
     "c5sim": "N2: 4096 duration-perturbed replicas of the 64x64 Cholesky DAG scored+queued (a1-a10) and scheduled "
              "by the PUSH/POP simulation with eviction (MAX_TRIES 16) on 30 CPU + 2 GPU workers "
              "(Intel-V100-like node, PAPER.md l.235)",
+    "c5loc": "N3: as c5sim with POP's data-locality pick (LS_SDH^2, n = 10, eps = 0.8, PAPER.md l.238) on "
+             "960x960-double tiles, per-node residency, transfers at 2^-24 ms/byte (~16.8 GB/s)",
     "c2push": "N1 incremental READY-mode push over the whole schedule of the 64x64 Cholesky DAG "
               "(each step: sources, then one mp_queues_push per completion batch = every ready task)",
 }
@@ -66,7 +69,7 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c5sim", "c2push"))
+    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c5sim", "c5loc", "c2push"))
     p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS,
                    help="c5: replicas per GPU (weak scaling, default) or in total (--scaling strong)")
     p.add_argument("--scaling", choices=("weak", "strong"), default="weak",
@@ -146,12 +149,15 @@ def oracle_sample(cfg, w, budget_s, R):
     import oracle
     t0 = time.perf_counter()
     od = oracle.build_dag(w.n, w.src, w.dst)
-    if cfg == "c5sim":
+    if cfg in ("c5sim", "c5loc"):
+        loc = {}
+        if cfg == "c5loc":
+            loc = dict(LOC, data=oracle.DataModel(w.acc_ptr, w.acc_handle, w.acc_mode, w.handle_size))
         k = 0
         while True:
             oracle.replica(od, w.dur, SIM_WORKERS, workloads.C5_SEED, workloads.C5_SIGMA, k, want_queue=True)
             oracle.simulate_replica(od, w.dur, SIM_WORKERS, workloads.C5_SEED, workloads.C5_SIGMA, k,
-                                    SIM_MAX_TRIES, True, trace=False)
+                                    SIM_MAX_TRIES, True, trace=False, **loc)
             k += 1
             if time.perf_counter() - t0 >= budget_s or k >= R:
                 break
@@ -184,7 +190,7 @@ def run_reference(args):
     import oracle
     oracle.build()
     cfg = args.config
-    w = workloads.config("c2" if cfg in ("c5", "c5sim") else cfg)
+    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc") else cfg)
     per_step_budget = 3.0 if cfg != "c4" else 10.0
     times, tasks = [], []
     for i in range(args.warmup + args.steps):
@@ -194,7 +200,7 @@ def run_reference(args):
             times.append(dt)
             tasks.append(v * dt)
     value = sum(tasks) / sum(times)
-    line = {"impl": "reference", "metric": METRIC_SIM if cfg == "c5sim" else METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
+    line = {"impl": "reference", "metric": METRIC_SIM if cfg in ("c5sim", "c5loc") else METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
             "scaling": "none", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": CONFIG_TEXT[cfg], "name": cfg,
@@ -265,7 +271,8 @@ def run_ours(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     cfg = args.config
-    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c2push") else cfg)
+    sim = cfg in ("c5sim", "c5loc")
+    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc", "c2push") else cfg)
     A = w.n_arch
     n = w.n
     src_h = torch.from_numpy(w.src).pin_memory()
@@ -278,12 +285,14 @@ def run_ours(args):
     E = dag.n_edges
     stream = torch.cuda.current_stream()
 
-    if cfg in ("c5", "c5sim"):
+    if cfg in ("c5", "c5sim", "c5loc"):
         # replicas are independent problems keyed by their GLOBAL id (world-size invariant results)
         R = args.replicas * world if args.scaling == "weak" else args.replicas
         r0, cnt = mpd.shard_range(R, world, rank)
         slots = mpd.shard_range(R, world, 0)[1]
-        sim = cfg == "c5sim"
+        loc = {}
+        if cfg == "c5loc":
+            loc = dict(LOC, data=mp.DataModel(w.acc_ptr, w.acc_handle, w.acc_mode, w.handle_size, device=dev))
         workers = np.asarray(SIM_WORKERS if sim else w.workers, np.int32)
         rb = mpd.record_bytes(A, mp.SIM_STATS_BYTES if sim else 0)
         out = dict(cp=torch.empty(max(cnt, 1), dtype=torch.float32, device=dev),
@@ -301,7 +310,7 @@ def run_ours(args):
             mp.replicas_run(dag, dur_d, workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out=out)
             if sim:
                 mp.simulate(dag, dur_d, workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out["qtask"],
-                            out["summary"], SIM_MAX_TRIES, True, out=sim_out)
+                            out["summary"], SIM_MAX_TRIES, True, out=sim_out, **loc)
             mpd.pack_records(out["cp"], out["summary"], cnt, A, slots, out=local_rec,
                              extra=sim_out["stats"] if sim else None)
             if world > 1:
@@ -444,7 +453,7 @@ def run_ours(args):
     except Exception:
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
     ctx = dict(n=n, E=E, A=A)
-    if cfg in ("c5", "c5sim"):
+    if cfg in ("c5", "c5sim", "c5loc"):
         ctx["replicas_per_launch"] = cnt      # one k_rep2_bl / k_rep2_sort launch covers the rank's block
         ctx["sort_entries_per_launch"] = cnt * A * n
     else:
@@ -461,7 +470,7 @@ def run_ours(args):
             "share_of_step": (dom_ms / args.steps) / ms_per_step, "peak_source": peak_src,
             "per_kernel_ms_per_step": {k: round(v, 4) for k, v in sorted(step_dev_ms.items(), key=lambda x: -x[1])}}
     # whole-step algorithmic bytes (SURVEY §8(d) B_alg) as context
-    if cfg in ("c5", "c5sim"):
+    if cfg in ("c5", "c5sim", "c5loc"):
         b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + args.replicas * 4 * n * A / world  # CSR + dur + queues out
     else:
         b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 4 * n * A + 4 * n * A
@@ -476,15 +485,17 @@ def run_ours(args):
         cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, "seconds": round(dt, 2)}
 
     rep = cfg in ("c5", "c5sim")
-    line = {"metric": METRIC_SIM if cfg == "c5sim" else METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+    line = {"metric": METRIC_SIM if cfg in ("c5sim", "c5loc") else METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": args.scaling if cfg in ("c5", "c5sim") else "none", "vs_baseline": None, "dtype": "f32",
+            "scaling": args.scaling if rep else "none", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic",
             "config": {"workload": (CONFIG_TEXT[cfg] if not rep else
                                     f"{R} duration-perturbed replicas of the 64x64 Cholesky DAG ({cnt} per GPU, "
                                     f"{args.scaling} scaling; BASELINE config 5 = 4096 in total = --scaling strong)"
                                     + ("; each scheduled by the N2 PUSH/POP simulation with eviction on "
-                                       f"{SIM_WORKERS[0]} CPU + {SIM_WORKERS[1]} GPU workers" if cfg == "c5sim" else "")),
+                                       f"{SIM_WORKERS[0]} CPU + {SIM_WORKERS[1]} GPU workers" if sim else "")
+                                    + ("; POP with the LS_SDH^2 locality pick (n = 10, eps = 0.8) on 960x960 tiles, "
+                                       "transfers at 2^-24 ms/byte" if cfg == "c5loc" else "")),
                        "name": cfg, "tasks_per_dag": n, "edges": E,
                        "levels": dag.n_levels, "archs": A,
                        "replicas": R if rep else 1, "replicas_per_gpu": cnt,
@@ -493,13 +504,15 @@ def run_ours(args):
                        "queues": "materialised in HBM for every replica" if rep else "materialised",
                        "step": ("mp_dag_rebuild + mp_replicas_run + allgather(records)" if cfg == "c5" else
                                 "mp_dag_rebuild + mp_replicas_run + mp_simulate + allgather(records + sim stats)"
-                                if cfg == "c5sim" else
+                                if sim else
                                 "mp_build_queues(sources) + mp_queues_push per completion batch (scores precomputed)"
                                 if cfg == "c2push" else
                                 "mp_dag_rebuild + bottom_level + affinity + score + build_queues"),
                        "parallelism": f"replica shards x{world}" if rep else "single DAG",
                        **({"sim_workers": list(SIM_WORKERS), "max_tries": SIM_MAX_TRIES, "eviction": True}
-                          if cfg == "c5sim" else {})},
+                          if sim else {}),
+                       **({"locality": {"top_n": LOC["top_n"], "eps": LOC["eps"],
+                                        "xfer_ms_per_byte": LOC["xfer_ms_per_byte"]}} if cfg == "c5loc" else {})},
             "ms_per_dag": ms_per_step / (R / world) if rep else ms_per_step,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
             "gpu_launches_per_step": launches / args.steps, "clocks": ck,
