@@ -67,6 +67,9 @@ def lib():
         _lib.or_perturb.argtypes = [i32, i32, P, u64, f32, i64, P]
         _lib.or_perturb.restype = None
         _lib.or_replica.argtypes = [i32, i32, P, P, P, P, P, u64, f32, i64, P, P, P, P]
+        _lib.or_bottom_level_w.argtypes = [i32, i32, P, P, P, P, P, i32, P, P]
+        _lib.or_nod_remaining.argtypes = [i32, i32, P, P, P, P, P, P]
+        _lib.or_affinity_prefix.argtypes = [i32, i32, P, P, P, P, P, P]
         _lib.or_simulate.argtypes = [i32, i32, P, P, P, P, P, P, P, P, P, P, P]
     return _lib
 
@@ -132,6 +135,48 @@ def bottom_level(dag: Dag, dur, workers):
     if rc:
         raise OracleError(rc, "bottom_level")
     return bl[:n], cp[0]
+
+
+WEIGHT_MIN, WEIGHT_MEAN = 0, 1
+
+
+def bottom_level_w(dag: Dag, dur, workers, wkind=WEIGHT_MIN):
+    """N4: bottom-level with node weight min (c2) or HEFT mean cost (v1)."""
+    dur = _c(dur, np.float32)
+    n, A = dur.shape
+    bl = np.zeros(max(n, 1), np.float32)
+    cp = np.zeros(1, np.float32)
+    rc = lib().or_bottom_level_w(n, A, _p(dag.row_ptr), _p(dag.col if dag.n_edges else np.zeros(1, np.int32)),
+                                 _p(dag.level_order), _p(dur), _p(_c(workers, np.int32)), int(wkind), _p(bl), _p(cp))
+    if rc:
+        raise OracleError(rc, "bottom_level_w")
+    return bl[:n], cp[0]
+
+
+def nod_remaining(dag: Dag, dur, workers, done):
+    """N4: NOD against the remaining graph (done tasks removed, v3)."""
+    dur = _c(dur, np.float32)
+    n, A = dur.shape
+    out = np.zeros((max(n, 1), A), np.float32)
+    rc = lib().or_nod_remaining(n, A, _p(dag.row_ptr), _p(dag.col if dag.n_edges else np.zeros(1, np.int32)),
+                                _p(dur), _p(_c(workers, np.int32)), _p(_c(done, np.uint8)), _p(out))
+    if rc:
+        raise OracleError(rc, "nod_remaining")
+    return out[:n]
+
+
+def affinity_prefix(dur, workers, order=None):
+    """N4: gains with hd(a) as the running max along the push order (v2)."""
+    dur = _c(dur, np.float32)
+    n, A = dur.shape
+    gain = np.zeros((max(n, 1), A), np.float32)
+    hd = np.zeros(A, np.float32)
+    flags = np.zeros((max(n, 1), A), np.uint8)
+    o = None if order is None else _c(order, np.int32)
+    rc = lib().or_affinity_prefix(n, A, _p(dur), _p(_c(workers, np.int32)), _p(o), _p(gain), _p(hd), _p(flags))
+    if rc:
+        raise OracleError(rc, "affinity_prefix")
+    return gain[:n], hd, flags[:n]
 
 
 def nod(dag: Dag, dur, workers):

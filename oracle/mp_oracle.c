@@ -153,9 +153,41 @@ static float weight(const float* dur, const int32_t* workers, int32_t A, int32_t
 /* a4: bottom-level (north_star): bl(v) = w(v) + max_{s in succ(v)} bl(s),  */
 /* bl(v) = w(v) when v has no successor; CP = max_v bl(v).                 */
 /* --------------------------------------------------------------------- */
+/* N4: HEFT-style mean cost as the node weight (reading v1):
+ * w(t) = (sum over enabled a, in arch order, of W_a * delta(t,a)) / sum of
+ * W_a, each op one RN binary64 op, rounded once to binary32. */
+static float weight_mean(const float* dur, const int32_t* workers, int32_t A, int32_t t) {
+    double num = 0.0;
+    int64_t den = 0;
+    for (int32_t a = 0; a < A; a++)
+        if (enabled(dur, workers, A, t, a)) {
+            num = num + (double)workers[a] * (double)dur[(int64_t)t * A + a];
+            den += workers[a];
+        }
+    return (float)(num / (double)den);
+}
+
+static int bottom_level_kind(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
+                             const int32_t* level_order, const float* dur_in, const int32_t* workers,
+                             int32_t wkind, float* bl, float* cp);
+
 int or_bottom_level(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
                     const int32_t* level_order, const float* dur_in, const int32_t* workers,
                     float* bl, float* cp) {
+    return bottom_level_kind(n, A, row_ptr, col, level_order, dur_in, workers, 0, bl, cp);
+}
+
+/* wkind 0: w = min over enabled archs (c2); 1: mean cost (v1) */
+int or_bottom_level_w(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
+                      const int32_t* level_order, const float* dur_in, const int32_t* workers,
+                      int32_t wkind, float* bl, float* cp) {
+    if (wkind < 0 || wkind > 1) return OR_ERR_ARG;
+    return bottom_level_kind(n, A, row_ptr, col, level_order, dur_in, workers, wkind, bl, cp);
+}
+
+static int bottom_level_kind(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
+                             const int32_t* level_order, const float* dur_in, const int32_t* workers,
+                             int32_t wkind, float* bl, float* cp) {
     float* dur = (float*)malloc((size_t)((int64_t)n * A + 1) * sizeof(float));
     if (!dur) return OR_ERR_NOMEM;
     int rc = or_check_durations(n, A, dur_in, workers, dur);
@@ -163,7 +195,7 @@ int or_bottom_level(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t*
     float best = 0.0f;
     for (int32_t i = n - 1; i >= 0; i--) {                /* reverse topological order */
         int32_t v = level_order[i];
-        float w = weight(dur, workers, A, v);
+        float w = wkind ? weight_mean(dur, workers, A, v) : weight(dur, workers, A, v);
         if (row_ptr[v] == row_ptr[v + 1]) {
             bl[v] = w;
         } else {
@@ -187,8 +219,24 @@ int or_bottom_level(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t*
 /* converted once to binary32 and scaled by 2^-32.  nod = 0 when (t,a) is  */
 /* not enabled.                                                            */
 /* --------------------------------------------------------------------- */
+static int nod_done(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
+                    const float* dur_in, const int32_t* workers, const uint8_t* done, float* nod);
+
 int or_nod(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
            const float* dur_in, const int32_t* workers, float* nod) {
+    return nod_done(n, A, row_ptr, col, dur_in, workers, NULL, nod);
+}
+
+/* N4: NOD against the REMAINING graph (reading v3): completed tasks (done)
+ * leave lambda-; successors that are done and done tasks themselves score 0.
+ * With done = all-zero this is or_nod. */
+int or_nod_remaining(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
+                     const float* dur_in, const int32_t* workers, const uint8_t* done, float* nod) {
+    return nod_done(n, A, row_ptr, col, dur_in, workers, done, nod);
+}
+
+static int nod_done(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
+                    const float* dur_in, const int32_t* workers, const uint8_t* done, float* nod) {
     float* dur = (float*)malloc((size_t)((int64_t)n * A + 1) * sizeof(float));
     int32_t* ind = (int32_t*)calloc((size_t)n + 1, sizeof(int32_t));
     if (!dur || !ind) { free(dur); free(ind); return OR_ERR_NOMEM; }
@@ -197,15 +245,16 @@ int or_nod(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col,
     for (int32_t a = 0; a < A; a++) {
         for (int32_t s = 0; s < n; s++) ind[s] = 0;
         for (int32_t p = 0; p < n; p++)                        /* |lambda-(s, P_a)| */
-            if (enabled(dur, workers, A, p, a))
+            if (enabled(dur, workers, A, p, a) && !(done && done[p]))
                 for (int32_t e = row_ptr[p]; e < row_ptr[p + 1]; e++) ind[col[e]]++;
         for (int32_t t = 0; t < n; t++) {
             float v = 0.0f;
-            if (enabled(dur, workers, A, t, a)) {
+            if (enabled(dur, workers, A, t, a) && !(done && done[t])) {
                 uint64_t acc = 0;
                 for (int32_t e = row_ptr[t]; e < row_ptr[t + 1]; e++) {
                     int32_t s = col[e];
-                    if (enabled(dur, workers, A, s, a)) acc += (uint64_t)(4294967296ull / (uint64_t)ind[s]);
+                    if (enabled(dur, workers, A, s, a) && !(done && done[s]))
+                        acc += (uint64_t)(4294967296ull / (uint64_t)ind[s]);
                 }
                 v = (float)acc * 0x1p-32f;
             }
@@ -277,6 +326,57 @@ int or_affinity(int32_t n, int32_t A, const float* dur_in, const int32_t* worker
 /* kind 0: crit = bl[n] (crit_norm[n]); kind 1: crit = nod[n][A]           */
 /* normalised per arch over enabled tasks (crit_norm[n][A]).               */
 /* --------------------------------------------------------------------- */
+/* --------------------------------------------------------------------- */
+/* N4: hd(a) "recorded so far" read literally (P:l.176, reading v2): tasks  */
+/* are pushed in the given order (NULL = id order) and each task's gain     */
+/* uses the running max of |d| over the tasks pushed up to and including   */
+/* it; hd[] returns the final max (= or_affinity's hd).                     */
+/* --------------------------------------------------------------------- */
+int or_affinity_prefix(int32_t n, int32_t A, const float* dur_in, const int32_t* workers,
+                       const int32_t* order, float* gain, float* hd, uint8_t* flags) {
+    float* dur = (float*)malloc((size_t)((int64_t)n * A + 1) * sizeof(float));
+    if (!dur) return OR_ERR_NOMEM;
+    int rc = or_check_durations(n, A, dur_in, workers, dur);
+    if (rc) { free(dur); return rc; }
+    float run[8] = {0};
+    for (int32_t i = 0; i < n; i++) {
+        int32_t t = order ? order[i] : i;
+        if (t < 0 || t >= n) { free(dur); return OR_ERR_ARG; }
+        int k = 0;
+        for (int32_t a = 0; a < A; a++) k += enabled(dur, workers, A, t, a);
+        float w = weight(dur, workers, A, t);
+        float dd[8];
+        for (int32_t a = 0; a < A; a++) {
+            dd[a] = 0.0f;
+            if (!enabled(dur, workers, A, t, a)) continue;
+            float ref = INFINITY;
+            for (int32_t b = 0; b < A; b++)
+                if (b != a && enabled(dur, workers, A, t, b) && dur[(int64_t)t * A + b] < ref)
+                    ref = dur[(int64_t)t * A + b];
+            if (k >= 2) {
+                dd[a] = ref - dur[(int64_t)t * A + a];
+                if (fabsf(dd[a]) > run[a]) run[a] = fabsf(dd[a]);      /* pushed: recorded */
+            }
+        }
+        for (int32_t a = 0; a < A; a++) {
+            int64_t j = (int64_t)t * A + a;
+            float g = 0.0f;
+            uint8_t f = 0;
+            if (enabled(dur, workers, A, t, a)) {
+                f = 1 | (dur[j] == w ? 2 : 0);
+                if (k == 1) g = 1.0f;
+                else if (run[a] == 0.0f) g = 0.5f;
+                else g = (dd[a] + run[a]) / (run[a] + run[a]);
+            }
+            gain[j] = g;
+            flags[j] = f;
+        }
+    }
+    for (int32_t a = 0; a < A; a++) hd[a] = run[a];
+    free(dur);
+    return OR_OK;
+}
+
 static uint32_t f2u(float x) { uint32_t u; memcpy(&u, &x, 4); return u; }
 
 int or_score(int32_t n, int32_t A, int32_t kind, const float* crit, const float* gain,
