@@ -290,6 +290,37 @@ mp_status mp_simulate_cfg(mp_dag* dag, int32_t n_arch, const float* d_base_dur, 
                           const mp_queue_summary* d_sum, const mp_sim_config* cfg, mp_sim_stats* d_stats,
                           double* d_start, int32_t* d_worker, void* stream);
 
+/*
+ * variants (ablations of readings c2, c4, c10).
+ *
+ * mp_bottom_level_w: bottom-level (a4) with a choice of node weight:
+ *   MP_WEIGHT_MIN  = min over enabled archs (reading c2, = mp_bottom_level);
+ *   MP_WEIGHT_MEAN = HEFT's mean cost over the platform's processors
+ *     (reading v1): w(t) = (sum over enabled a, in arch order, of
+ *     h_workers[a] * delta(t,a)) / sum of h_workers[a], each op one RN
+ *     binary64 op, rounded once to binary32.
+ *
+ * mp_affinity_prefix: eq. 1 gains with hd(a) read as "the highest execution
+ *   time difference recorded SO FAR" (P:l.176, reading v2): tasks are pushed
+ *   in the order d_order (int32[n], a permutation of [0,n); NULL = id order)
+ *   and task t's gains use the running max of |d(u,a)| over the tasks u
+ *   pushed up to and including t.  d_hd receives the final max (= mp_affinity's
+ *   hd); d_flags as mp_affinity.  An id outside [0,n) raises MP_ERR_ARG via
+ *   mp_check.
+ *
+ * mp_nod_remaining: NOD (eq. 2) on the remaining graph (reading v3): tasks
+ *   with d_done[t] != 0 are removed from lambda^- and lambda^+; done tasks
+ *   score 0.  d_done = all-zero gives mp_bottom_level's d_nod.
+ */
+typedef enum { MP_WEIGHT_MIN = 0, MP_WEIGHT_MEAN = 1 } mp_weight;
+
+mp_status mp_bottom_level_w(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers,
+                            mp_weight kind, float* d_bl, float* d_cp, void* stream);
+mp_status mp_affinity_prefix(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers,
+                             const int32_t* d_order, float* d_gain, float* d_hd, uint8_t* d_flags, void* stream);
+mp_status mp_nod_remaining(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers,
+                           const uint8_t* d_done, float* d_nod, void* stream);
+
 /* Synchronise `stream`, then return (and clear) the handle's device error
  * flag: MP_OK or MP_ERR_DOMAIN; MP_ERR_CUDA on a pending CUDA error. */
 mp_status mp_check(mp_dag* dag, void* stream);

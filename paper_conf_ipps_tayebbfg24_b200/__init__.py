@@ -18,7 +18,7 @@ import torch
 
 from . import _lib
 from ._lib import (MP_CRIT_BOTTOM_LEVEL, MP_CRIT_NOD, MP_ERR_ARG, MP_ERR_CUDA, MP_ERR_CYCLE,  # noqa: F401
-                   MP_ERR_DOMAIN, MP_ERR_NOMEM, MP_OK, MPError)
+                   MP_ERR_DOMAIN, MP_ERR_NOMEM, MP_OK, MP_WEIGHT_MEAN, MP_WEIGHT_MIN, MPError)
 
 SUMMARY_DTYPE = np.dtype([("count", "<i4"), ("head", "<i4"), ("brw_lo", "<u8"), ("brw_hi", "<i8"),
                           ("brw", "<f8")])
@@ -158,6 +158,48 @@ def bottom_level(dag: Dag, dur: torch.Tensor, workers, nod: bool = False, out=No
                                     _ptr(out["nod"]) if out.get("nod") is not None else None, _stream())
     _lib.check(rc, "mp_bottom_level")
     return out["bl"], out["cp"], out.get("nod")
+
+
+def bottom_level_w(dag: Dag, dur: torch.Tensor, workers, kind: int = MP_WEIGHT_MIN, out=None):
+    """N4 (mp_bottom_level_w): bottom-level with node weight min (c2) or HEFT mean cost (v1) -> (bl, cp)."""
+    n, A = dur.shape
+    w, wp = _workers(workers, A)
+    dev = dur.device
+    if out is None:
+        out = dict(bl=torch.empty(n, dtype=torch.float32, device=dev),
+                   cp=torch.empty(1, dtype=torch.float32, device=dev))
+    rc = _lib.lib().mp_bottom_level_w(dag.handle, A, _ptr(dur), wp, int(kind), _ptr(out["bl"]), _ptr(out["cp"]),
+                                      _stream())
+    _lib.check(rc, "mp_bottom_level_w")
+    return out["bl"], out["cp"]
+
+
+def affinity_prefix(dag: Dag, dur: torch.Tensor, workers, order: torch.Tensor | None = None, out=None):
+    """N4 (mp_affinity_prefix): gains with hd as a running max along the push order -> (gain, hd, flags)."""
+    n, A = dur.shape
+    w, wp = _workers(workers, A)
+    dev = dur.device
+    if out is None:
+        out = dict(gain=torch.empty((n, A), dtype=torch.float32, device=dev),
+                   hd=torch.empty(A, dtype=torch.float32, device=dev),
+                   flags=torch.empty((n, A), dtype=torch.uint8, device=dev))
+    o = None if order is None else order.to(torch.int32).contiguous()
+    rc = _lib.lib().mp_affinity_prefix(dag.handle, A, _ptr(dur), wp, _ptr(o), _ptr(out["gain"]), _ptr(out["hd"]),
+                                       _ptr(out["flags"]), _stream())
+    _lib.check(rc, "mp_affinity_prefix")
+    return out["gain"], out["hd"], out["flags"]
+
+
+def nod_remaining(dag: Dag, dur: torch.Tensor, workers, done: torch.Tensor, out=None):
+    """N4 (mp_nod_remaining): NOD on the remaining graph (done tasks removed) -> nod[n][A]."""
+    n, A = dur.shape
+    w, wp = _workers(workers, A)
+    if out is None:
+        out = torch.empty((n, A), dtype=torch.float32, device=dur.device)
+    rc = _lib.lib().mp_nod_remaining(dag.handle, A, _ptr(dur), wp, _ptr(done.to(torch.uint8).contiguous()),
+                                     _ptr(out), _stream())
+    _lib.check(rc, "mp_nod_remaining")
+    return out
 
 
 def affinity(dag: Dag, dur: torch.Tensor, workers, out=None):

@@ -7,6 +7,7 @@
 #include "push.cuh"
 #include "rep2.cuh"
 #include "sim.cuh"
+#include "variants.cuh"
 
 static inline cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
 
@@ -97,6 +98,21 @@ mp_status mp_simulate_cfg(mp_dag* dag, int32_t n_arch, const float* d_base_dur, 
                           double* d_start, int32_t* d_worker, void* stream) {
     return mph::simulate(dag, n_arch, d_base_dur, h_workers, seed, sigma, r0, R, d_qtask, d_sum, cfg, d_stats,
                          d_start, d_worker, as_stream(stream));
+}
+
+mp_status mp_bottom_level_w(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers, mp_weight kind,
+                            float* d_bl, float* d_cp, void* stream) {
+    return mph::bottom_level(dag, n_arch, d_dur, h_workers, d_bl, d_cp, nullptr, as_stream(stream), (int32_t)kind);
+}
+
+mp_status mp_affinity_prefix(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers,
+                             const int32_t* d_order, float* d_gain, float* d_hd, uint8_t* d_flags, void* stream) {
+    return mph::affinity_prefix(dag, n_arch, d_dur, h_workers, d_order, d_gain, d_hd, d_flags, as_stream(stream));
+}
+
+mp_status mp_nod_remaining(mp_dag* dag, int32_t n_arch, const float* d_dur, const int32_t* h_workers,
+                           const uint8_t* d_done, float* d_nod, void* stream) {
+    return mph::nod_remaining(dag, n_arch, d_dur, h_workers, d_done, d_nod, as_stream(stream));
 }
 
 mp_status mp_check(mp_dag* dag, void* stream) {

@@ -12,21 +12,32 @@ struct DurView {          // read-only duration table + enabled archs
     const float* dur;     // [n][A]
     int32_t A;
     uint32_t emask;
+    int32_t wkind;        // node weight: 0 = min (c2), 1 = mean cost (N4, v1)
+    int32_t W[MAX_ARCH];  // worker counts (mean cost only)
 };
 
 // w(v) = min over enabled a of delta(v,a) (reading c2), with the domain check
 // (reading c20).  Sets `bad` on a domain violation or no enabled arch.
+// N4 (v1): w(v) = (sum_a W_a delta(v,a)) / sum_a W_a over enabled a, in arch
+// order, each op one RN binary64 op, rounded once to binary32.
 MP_INLINE float task_weight(const DurView& d, int32_t v, bool& bad) {
     float w = __uint_as_float(0x7f800000u);
     bool any = false;
+    double num = 0.0;
+    int64_t den = 0;
     for (int a = 0; a < d.A; a++) {
         float x = canon_dur(__ldg(d.dur + (int64_t)v * d.A + a), bad);
         if (((d.emask >> a) & 1u) && !is_inf(x)) {
             any = true;
             w = x < w ? x : w;
+            if (d.wkind) {
+                num = __dadd_rn(num, __dmul_rn((double)d.W[a], (double)x));
+                den += d.W[a];
+            }
         }
     }
     if (!any) bad = true;
+    if (any && d.wkind) w = __double2float_rn(__ddiv_rn(num, (double)den));
     return any ? w : 0.0f;
 }
 
@@ -128,9 +139,11 @@ __global__ void __launch_bounds__(FLOW_THREADS) k_bl_flow(int32_t nchunks, const
 
 // ---- a5: NOD (eq. 2) -----------------------------------------------------------------
 // indeg_a(s) = |{p in lambda^-(s) : p enabled on a}|
+// (N4, v3: with `done`, completed predecessors leave lambda^-)
 __global__ void k_nod_indeg(int32_t n, const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                            DurView d, int32_t* inda) {
+                            DurView d, const uint8_t* __restrict__ done, int32_t* inda) {
     for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
+        if (done && done[u]) continue;
         uint32_t en = 0;
         for (int a = 0; a < d.A; a++)
             if (((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + u * d.A + a))) en |= 1u << a;
@@ -145,16 +158,18 @@ __global__ void k_nod_indeg(int32_t n, const int32_t* __restrict__ row_ptr, cons
 
 // NOD_a(t) = sum over enabled successors s of floor(2^32 / indeg_a(s)) (exact uint64),
 // converted once (RN) and scaled by 2^-32 (exact); 0 where (t,a) is not enabled.
+// (N4, v3: with `done`, completed tasks and successors score / count 0)
 __global__ void k_nod_sum(int32_t n, const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                          DurView d, const int32_t* __restrict__ inda, float* nod) {
+                          DurView d, const uint8_t* __restrict__ done, const int32_t* __restrict__ inda, float* nod) {
     for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+        const bool tdone = done && done[t];
         for (int a = 0; a < d.A; a++) {
             float out = 0.0f;
-            if (((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + t * d.A + a))) {
+            if (!tdone && ((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + t * d.A + a))) {
                 uint64_t acc = 0;
                 for (int32_t e = row_ptr[t]; e < row_ptr[t + 1]; e++) {
                     int32_t s = col[e];
-                    if (((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + (int64_t)s * d.A + a)))
+                    if (((d.emask >> a) & 1u) && !is_inf(__ldg(d.dur + (int64_t)s * d.A + a)) && !(done && done[s]))
                         acc += 4294967296ull / (uint64_t)inda[(int64_t)s * d.A + a];
                 }
                 out = __fmul_rn(__ull2float_rn(acc), 0x1p-32f);
@@ -387,12 +402,15 @@ inline mp_status check_arch(int32_t A, const int32_t* h_workers) {
 }
 
 inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const int32_t* h_workers, float* bl,
-                              float* cp, float* nod, cudaStream_t st) {
+                              float* cp, float* nod, cudaStream_t st, int32_t wkind = 0) {
     using namespace mpk;
     if (!dag) return fail(MP_ERR_ARG, "dag is NULL");
     MP_TRY(check_arch(A, h_workers));
+    if (wkind != 0 && wkind != 1) return fail(MP_ERR_ARG, "unknown weight kind %d", wkind);
     if (!cp || (dag->n > 0 && (!dur || !bl))) return fail(MP_ERR_ARG, "NULL buffer");
     DurView d{dur, A, enabled_mask(A, h_workers)};
+    d.wkind = wkind;
+    for (int a = 0; a < A; a++) d.W[a] = h_workers[a] > 0 ? h_workers[a] : 0;
     MP_CUDA(cudaMemsetAsync(cp, 0, 4, st));
     const int32_t n = dag->n;
     if (n == 0) return MP_OK;
@@ -429,8 +447,8 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
         MP_TRY(ensure_ws(dag, need, st));
         int32_t* inda = (int32_t*)dag->ws;
         MP_CUDA(cudaMemsetAsync(inda, 0, (size_t)n * A * 4, st));
-        MP_LAUNCH(k_nod_indeg, grid_for(n), 256, 0, st, n, dag->row_ptr, dag->col, d, inda);
-        MP_LAUNCH(k_nod_sum, grid_for(n), 256, 0, st, n, dag->row_ptr, dag->col, d, inda, nod);
+        MP_LAUNCH(k_nod_indeg, grid_for(n), 256, 0, st, n, dag->row_ptr, dag->col, d, nullptr, inda);
+        MP_LAUNCH(k_nod_sum, grid_for(n), 256, 0, st, n, dag->row_ptr, dag->col, d, nullptr, inda, nod);
         MP_CUDA(cudaGetLastError());
     }
     return MP_OK;
