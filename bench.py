@@ -52,6 +52,10 @@ CONFIG_TEXT = {
              "(Intel-V100-like node, PAPER.md l.235)",
     "c5loc": "N3: as c5sim with POP's data-locality pick (LS_SDH^2, n = 10, eps = 0.8, PAPER.md l.238) on "
              "960x960-double tiles, per-node residency, transfers at 2^-24 ms/byte (~16.8 GB/s)",
+    "lu64": "N4 workload: tiled LU without pivoting 64x64 tiles (getrf, PAPER.md l.251; 89,440 tasks), 2 resource types",
+    "c2n4": "N4 variants on the 64x64 Cholesky DAG: mean-cost (HEFT) bottom-level, hd as a running max along the "
+            "push order (id order), NOD on the remaining graph (first half of the level order completed), "
+            "score + queues",
     "c2push": "N1 incremental READY-mode push over the whole schedule of the 64x64 Cholesky DAG "
               "(each step: sources, then one mp_queues_push per completion batch = every ready task)",
 }
@@ -69,7 +73,7 @@ def parse():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c5sim", "c5loc", "c2push"))
+    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c5sim", "c5loc", "c2push", "lu64", "c2n4"))
     p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS,
                    help="c5: replicas per GPU (weak scaling, default) or in total (--scaling strong)")
     p.add_argument("--scaling", choices=("weak", "strong"), default="weak",
@@ -174,8 +178,18 @@ def oracle_sample(cfg, w, budget_s, R):
         dt = time.perf_counter() - t0
         return k * w.n / dt, f"1 DAG build + {k} of {R} replicas of c2 (perturbation seed {workloads.C5_SEED})", dt
     reps = 0
+    if cfg == "c2n4":
+        done = np.zeros(w.n, np.uint8)
+        done[od.level_order[: w.n // 2]] = 1
     while True:
-        oracle.score_and_queue(od, w.dur, w.workers)
+        if cfg == "c2n4":
+            bl, cp = oracle.bottom_level_w(od, w.dur, w.workers, oracle.WEIGHT_MEAN)
+            gain, hd, flags = oracle.affinity_prefix(w.dur, w.workers)
+            oracle.nod_remaining(od, w.dur, w.workers, done)
+            cn, key = oracle.score(oracle.CRIT_BL, bl, gain, flags)
+            oracle.build_queues(od, key, flags, oracle.check_durations(w.dur, w.workers))
+        else:
+            oracle.score_and_queue(od, w.dur, w.workers)
         reps += 1
         if time.perf_counter() - t0 >= budget_s:
             break
@@ -190,7 +204,7 @@ def run_reference(args):
     import oracle
     oracle.build()
     cfg = args.config
-    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc") else cfg)
+    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc", "c2n4") else cfg)
     per_step_budget = 3.0 if cfg != "c4" else 10.0
     times, tasks = [], []
     for i in range(args.warmup + args.steps):
@@ -272,7 +286,7 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=dev)
     cfg = args.config
     sim = cfg in ("c5sim", "c5loc")
-    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc", "c2push") else cfg)
+    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc", "c2push", "c2n4") else cfg)
     A = w.n_arch
     n = w.n
     src_h = torch.from_numpy(w.src).pin_memory()
@@ -344,6 +358,33 @@ def run_ours(args):
                 mp.queues_push(dag, key_d, flags_d, dur_d, batch, rem, bufs[cur]["qptr"], bufs[cur]["qtask"],
                                out=bufs[cur ^ 1])
                 cur ^= 1
+    elif cfg == "c2n4":
+        R, cnt = 1, 1
+        tasks_per_step = n
+        done_h = np.zeros(n, np.uint8)
+        done_h[dag.arrays()["level_order"].cpu().numpy()[: n // 2]] = 1
+        done_d = torch.from_numpy(done_h).to(dev)
+        o = dict(bl=dict(bl=torch.empty(n, dtype=torch.float32, device=dev),
+                         cp=torch.empty(1, dtype=torch.float32, device=dev)),
+                 aff=dict(gain=torch.empty((n, A), dtype=torch.float32, device=dev),
+                          hd=torch.empty(A, dtype=torch.float32, device=dev),
+                          flags=torch.empty((n, A), dtype=torch.uint8, device=dev)),
+                 nod=torch.empty((n, A), dtype=torch.float32, device=dev),
+                 sc=dict(crit_norm=torch.empty(n, dtype=torch.float32, device=dev),
+                         key=torch.empty((n, A), dtype=torch.int64, device=dev)),
+                 q=dict(qptr=torch.empty(A + 1, dtype=torch.int64, device=dev),
+                        qtask=torch.empty(n * A, dtype=torch.int32, device=dev),
+                        summary=torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev)))
+        result_h = torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8).pin_memory()
+
+        def step():
+            mp.dag_rebuild(dag, n, src_d, dst_d)
+            bl, cp = mp.bottom_level_w(dag, dur_d, w.workers, mp.MP_WEIGHT_MEAN, out=o["bl"])
+            gain, hd, flags = mp.affinity_prefix(dag, dur_d, w.workers, None, out=o["aff"])
+            mp.nod_remaining(dag, dur_d, w.workers, done_d, out=o["nod"])
+            cn, key = mp.score(dag, 0, bl, gain, flags, out=o["sc"])
+            qptr, qtask, summ = mp.build_queues(dag, key, flags, dur_d, out=o["q"])
+            return summ
     else:
         R, cnt = 1, 1
         outs = {}
@@ -507,6 +548,8 @@ def run_ours(args):
                                 if sim else
                                 "mp_build_queues(sources) + mp_queues_push per completion batch (scores precomputed)"
                                 if cfg == "c2push" else
+                                "mp_dag_rebuild + bottom_level_w(mean) + affinity_prefix + nod_remaining + score + "
+                                "build_queues" if cfg == "c2n4" else
                                 "mp_dag_rebuild + bottom_level + affinity + score + build_queues"),
                        "parallelism": f"replica shards x{world}" if rep else "single DAG",
                        **({"sim_workers": list(SIM_WORKERS), "max_tries": SIM_MAX_TRIES, "eviction": True}
