@@ -6,8 +6,11 @@ O=gpurun_out/meas
 mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,clocks.mem,power.draw --format=csv > $O/gpu.txt
 timeout 600 python bench.py > $O/bench_c5.json 2> $O/bench_c5.err; echo "c5 rc=$?"
-for c in c2 c3 c4; do
+for c in c2 c3 c4 lu64 c2n4 c2push; do
   timeout 600 python bench.py --config $c --steps 10 --warmup 3 --cpu-budget-s 8 > $O/bench_$c.json 2> $O/bench_$c.err; echo "$c rc=$?"
+done
+for c in c5sim c5loc; do
+  timeout 600 python bench.py --config $c --steps 5 --warmup 3 --cpu-budget-s 8 > $O/bench_$c.json 2> $O/bench_$c.err; echo "$c rc=$?"
 done
 timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > $O/bench_ref_c5.json 2> $O/bench_ref.err; echo "ref rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_c5.csv \
@@ -16,3 +19,5 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_re
    python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e > $O/full_c5.log 2>&1; echo "full c5 rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_bl_flow|k_kahn|k_sort_pass" -c 4 -o $O/full_c4 \
    python bench.py --config c4 --steps 1 --warmup 0 --no-cpu-baseline --no-e2e > $O/full_c4.log 2>&1; echo "full c4 rc=$?"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_sim -c 1 -o $O/full_c5sim \
+   python bench.py --config c5sim --replicas 2048 --steps 1 --warmup 0 --no-cpu-baseline --no-e2e > $O/full_c5sim.log 2>&1; echo "full c5sim rc=$?"
