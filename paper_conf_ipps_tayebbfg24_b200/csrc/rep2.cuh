@@ -765,6 +765,34 @@ MP_INLINE void r2_gains_from_D(uint32_t D, float hd, uint32_t& G0, uint32_t& G1)
     G1 = ONE_BITS - f2u(g1);
 }
 
+// Do the sorted neighbours Da, Db have equal gain keys on arch 0 (s0) / arch 1 (s1)?
+// Same as comparing r2_gains_from_D's keys, without most divisions: for two-arch
+// tasks gain = RN(x / den) with x = RN(+-d + hd) in [0, den] (hd >= |d|), so
+// the quotients lie in [0, 1], where every rounding interval is at most 2^-24
+// wide; numerators further apart than den * 2^-24 (exact in binary64: both are
+// floats) therefore give different gains, equal numerators equal gains, and
+// only the remaining near-ties are divided.
+MP_INLINE void r2_same_gains(uint32_t Da, uint32_t Db, float hd, bool& s0, bool& s1) {
+    if (Da == Db) { s0 = s1 = true; return; }
+    if (Da == 0u || Da == 0xFFFFFFFFu || Db == 0u || Db == 0xFFFFFFFFu || hd == 0.0f) {
+        uint32_t A0, A1, B0, B1;
+        r2_gains_from_D(Da, hd, A0, A1);
+        r2_gains_from_D(Db, hd, B0, B1);
+        s0 = A0 == B0;
+        s1 = A1 == B1;
+        return;
+    }
+    const float da = u2f((Da & 0x80000000u) ? (Da & 0x7FFFFFFFu) : ~Da);
+    const float db = u2f((Db & 0x80000000u) ? (Db & 0x7FFFFFFFu) : ~Db);
+    const float den = __fadd_rn(hd, hd);
+    const double lim = (double)den * 0x1p-24;
+    const float xa = __fadd_rn(da, hd), xb = __fadd_rn(db, hd);
+    s0 = xa == xb || (fabs((double)xb - (double)xa) <= lim && __fdiv_rn(xa, den) == __fdiv_rn(xb, den));
+    const float ya = __fadd_rn(__fsub_rn(0.0f, da), hd), yb = __fadd_rn(__fsub_rn(0.0f, db), hd);
+    s1 = ya == yb || (fabs((double)yb - (double)ya) <= lim && __fdiv_rn(ya, den) == __fdiv_rn(yb, den));
+}
+
+
 template <int A>
 __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     extern __shared__ __align__(16) unsigned char r3s[];
@@ -943,22 +971,14 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         const int32_t wb = wb0 + h * R2_THREADS;
                         if (wb >= a.n) break;
                         const int32_t p = wb + lane;
-                        uint32_t G0 = 0xFFFFFFFFu, G1 = 0xFFFFFFFFu;
                         const uint32_t DD = DDv[h];
-                        if (p < a.n) r2_gains_from_D(DD, h2, G0, G1);
-                        uint32_t N0 = __shfl_down_sync(0xffffffffu, G0, 1);
-                        uint32_t N1 = __shfl_down_sync(0xffffffffu, G1, 1);
                         uint32_t ND = __shfl_down_sync(0xffffffffu, DD, 1);
-                        if (lane == 31) {
-                            N0 = 0xFFFFFFFEu; N1 = 0xFFFFFFFEu; ND = ~DD;
-                            if (p + 1 < a.n) {
-                                ND = NDv[h];
-                                r2_gains_from_D(ND, h2, N0, N1);
-                            }
-                        }
+                        if (lane == 31) ND = p + 1 < a.n ? NDv[h] : ~DD;
                         const bool ok = p + 1 < a.n;
-                        const uint32_t b0 = __ballot_sync(0xffffffffu, ok && G0 == N0);
-                        const uint32_t b1 = __ballot_sync(0xffffffffu, ok && G1 == N1);
+                        bool same0 = false, same1 = false;
+                        if (ok) r2_same_gains(DD, ND, h2, same0, same1);
+                        const uint32_t b0 = __ballot_sync(0xffffffffu, same0);
+                        const uint32_t b1 = __ballot_sync(0xffffffffu, same1);
                         const uint32_t bD = __ballot_sync(0xffffffffu, ok && DD == ND);
                         if (lane == 0) {
                             e0[wb >> 5] = b0;
