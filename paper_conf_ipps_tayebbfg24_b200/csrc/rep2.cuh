@@ -241,7 +241,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
         }
     }
     if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(a.err, ERR_DOMAIN_BIT);
-    // ---- transpose bl32 [q][32] -> blT [r][t] ----
+    // ---- transpose bl32 [q][32] -> blT [r][t] (two archs: K2 reads bl32 directly, and
+    //      only for equal-gain runs) ----
+    if (A == 2) return;
     float* tile = reinterpret_cast<float*>(r2_smem) + w0 * 32 * 33;
     const int32_t nchunks = (a.n + 31) / 32;
     for (int32_t c = w; c < nchunks; c += WG) {
@@ -942,9 +944,10 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             int32_t* q0 = a.qtask ? a.qtask + rl * (int64_t)a.n * 2 : nullptr;
             int32_t* q1 = q0 ? q0 + cC : nullptr;
             const float h2 = hdv[0];   // hd(0) == hd(1) for two archs
-            const float* blr = a.blT + rl * a.n;
+            // bl of this replica in K1's [group][q][32] layout (no transpose for two archs)
+            const float* blr = a.bl32 + (rl >> 5) * (int64_t)a.n * 32 + (rl & 31);
             auto critc_of = [&](uint32_t t) -> uint32_t {
-                const float c = CP > 0.0f ? __fdiv_rn(__ldcg(blr + t), CP) : 0.0f;
+                const float c = CP > 0.0f ? __fdiv_rn(__ldcg(blr + (int64_t)__ldg(a.qof + t) * 32), CP) : 0.0f;
                 return ONE_BITS - f2u(c);
             };
             // sorted order into shared memory (the sort's buffers are free now) + neighbour-equality
@@ -1070,7 +1073,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
 #pragma unroll
             for (int b = 0; b < A; b++) { fmn[b] = ~0ull; fmx[b] = 0ull; }
             for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
-                const float c = CP > 0.0f ? __fdiv_rn(__ldcg(a.blT + rl * a.n + t), CP) : 0.0f;
+                const float c = CP > 0.0f ? __fdiv_rn(__ldcg(a.bl32 + (rl >> 5) * (int64_t)a.n * 32 +
+                                                              (int64_t)__ldg(a.qof + t) * 32 + (rl & 31)), CP)
+                                          : 0.0f;
                 const uint32_t cc = ONE_BITS - f2u(c);
                 critc[t] = cc;
                 uint32_t G[2];
@@ -1137,7 +1142,8 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const int32_t n = dag->n;
     const int64_t groups = (R + 31) / 32;
     const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
-    size_t bytes = align256((size_t)groups * n * 32 * 4) + align256((size_t)R * n * 4) + align256((size_t)R * A * 4) * 2 +
+    const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
+    size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
                    align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 3)) + align256((size_t)grid2 * ((n + 15) & ~15) * 4);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
@@ -1157,7 +1163,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.seed = seed;
     a.sigma = sigma;
     a.bl32 = ar.take<float>((size_t)groups * n * 32);
-    a.blT = ar.take<float>((size_t)R * n);
+    a.blT = ar.take<float>(blT_elems);
     a.cp = cp;
     a.hd = ar.take<uint32_t>((size_t)R * A);
     a.counts = ar.take<int32_t>((size_t)R * A);
