@@ -177,6 +177,24 @@ def oracle_sample(cfg, w, budget_s, R):
                 break
         dt = time.perf_counter() - t0
         return k * w.n / dt, f"1 DAG build + {k} of {R} replicas of c2 (perturbation seed {workloads.C5_SEED})", dt
+    if cfg == "c2push":
+        r = oracle.score_and_queue(od, w.dur, w.workers)
+        dc = oracle.check_durations(w.dur, w.workers)
+        reps = 0
+        while True:
+            done = np.zeros(w.n, np.uint8)
+            while True:                            # READY-mode rebuild after every completion batch
+                qp, q, _ = oracle.build_queues(od, r["key"], r["flags"], dc, done)
+                m = int(qp[1] - qp[0])
+                if m == 0:
+                    break
+                done[q[:m]] = 1
+            reps += 1
+            if time.perf_counter() - t0 >= budget_s:
+                break
+        dt = time.perf_counter() - t0
+        return reps * w.n / dt, (f"1 DAG build + scores + {reps} whole c2 schedules, READY-mode queues rebuilt "
+                                 f"after every completion batch"), dt
     reps = 0
     if cfg == "c2n4":
         done = np.zeros(w.n, np.uint8)
@@ -335,10 +353,12 @@ def run_ours(args):
     elif cfg == "c2push":
         R, cnt = 1, 1
         tasks_per_step = n
-        full = mp.score_and_queue(dag, dur_d, w.workers)
-        key_d, flags_d = full["key"], full["flags"]
-        zeros = torch.zeros(n, dtype=torch.uint8, device=dev)
+        full = mp.score_and_queue(dag, dur_d, w.workers)            # whole-DAG scores + ALL-mode queues
+        flags_d = full["flags"]
+        qptr_all, qtask_all = full["qptr"], full["qtask"]
         rem = torch.empty(n, dtype=torch.int32, device=dev)
+        done = torch.empty(n, dtype=torch.uint8, device=dev)
+        empty = torch.zeros(0, dtype=torch.int32, device=dev)
         bufs = [dict(qptr=torch.empty(A + 1, dtype=torch.int64, device=dev),
                      qtask=torch.empty(n * A, dtype=torch.int32, device=dev),
                      summary=torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev)) for _ in range(2)]
@@ -346,8 +366,9 @@ def run_ours(args):
         result_h = torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8).pin_memory()
 
         def step():
-            mp.build_queues(dag, key_d, flags_d, dur_d, done=zeros, out=bufs[0])
             mp.ready_init(dag, rem)
+            done.zero_()
+            mp.queues_push_all(dag, qptr_all, qtask_all, flags_d, dur_d, empty, rem, done, out=bufs[0])
             cur = 0
             while True:
                 qhost.copy_(bufs[cur]["qptr"])          # the scheduler reads the ready count
@@ -355,8 +376,7 @@ def run_ours(args):
                 if m == 0:
                     return bufs[cur]["summary"]
                 batch = bufs[cur]["qtask"][:m]
-                mp.queues_push(dag, key_d, flags_d, dur_d, batch, rem, bufs[cur]["qptr"], bufs[cur]["qtask"],
-                               out=bufs[cur ^ 1])
+                mp.queues_push_all(dag, qptr_all, qtask_all, flags_d, dur_d, batch, rem, done, out=bufs[cur ^ 1])
                 cur ^= 1
     elif cfg == "c2n4":
         R, cnt = 1, 1
@@ -546,7 +566,8 @@ def run_ours(args):
                        "step": ("mp_dag_rebuild + mp_replicas_run + allgather(records)" if cfg == "c5" else
                                 "mp_dag_rebuild + mp_replicas_run + mp_simulate + allgather(records + sim stats)"
                                 if sim else
-                                "mp_build_queues(sources) + mp_queues_push per completion batch (scores precomputed)"
+                                "mp_ready_init + mp_queues_push_all per completion batch (scores and ALL-mode queues "
+                                "precomputed)"
                                 if cfg == "c2push" else
                                 "mp_dag_rebuild + bottom_level_w(mean) + affinity_prefix + nod_remaining + score + "
                                 "build_queues" if cfg == "c2n4" else

@@ -211,6 +211,24 @@ mp_status mp_queues_push(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, con
                          int32_t* d_qtask_out, mp_queue_summary* d_sum, void* stream);
 
 /*
+ * N1, static-order variant.  Because the scores are whole-DAG (reading c18),
+ * every READY-mode queue is the ALL-mode queue restricted to the ready tasks,
+ * in the same order.  The caller keeps the ALL-mode queues (d_qptr_all,
+ * d_qtask_all from mp_build_queues with d_done = NULL), d_rem (mp_ready_init)
+ * and a done mask d_done (uint8[n], zeroed by the caller before the first
+ * push); a push marks the batch done, releases successors and compacts the
+ * ALL-mode queues into d_qptr_out / d_qtask_out (capacity n*A) with the
+ * summaries -- the same queues mp_queues_push produces, with no sort or merge.
+ * Pushing the empty batch (m = 0) yields the sources' queues.  A batch task
+ * that is not ready, completed twice, or outside [0,n) raises MP_ERR_ARG
+ * (mp_check).
+ */
+mp_status mp_queues_push_all(mp_dag* dag, int32_t n_arch, const int64_t* d_qptr_all, const int32_t* d_qtask_all,
+                             const uint8_t* d_flags, const float* d_dur, const int32_t* d_batch, int32_t m,
+                             int32_t* d_rem, uint8_t* d_done, int64_t* d_qptr_out, int32_t* d_qtask_out,
+                             mp_queue_summary* d_sum, void* stream);
+
+/*
  * discrete-event simulation of MultiPrio on a platform of
  * h_workers[a] workers of each architecture type a: PUSH (Alg. 1,
  * P:l.133-136) of every task that becomes ready (P:l.91), POP (Alg. 2,

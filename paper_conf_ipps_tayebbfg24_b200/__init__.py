@@ -351,6 +351,26 @@ def replicas_simulate(dag: Dag, base_dur: torch.Tensor, workers, seed: int, sigm
     return dict(cp=cp, summary=summ, qtask=q, stats=st, start=start, worker=worker)
 
 
+def queues_push_all(dag: Dag, qptr_all: torch.Tensor, qtask_all: torch.Tensor, flags: torch.Tensor,
+                    dur: torch.Tensor, batch: torch.Tensor, rem: torch.Tensor, done: torch.Tensor, out=None):
+    """mp_queues_push_all (N1, static order): complete `batch`, compact the ALL-mode queues
+    to the READY-mode queues -> (qptr, qtask, summary).  `rem` (mp_ready_init) and `done`
+    (uint8[n], zero at the start) are updated in place."""
+    n, A = flags.shape
+    dev = flags.device
+    batch = batch.to(torch.int32).contiguous()
+    if out is None:
+        out = dict(qptr=torch.empty(A + 1, dtype=torch.int64, device=dev),
+                   qtask=torch.empty(max(n * A, 1), dtype=torch.int32, device=dev),
+                   summary=torch.empty(A * SUMMARY_BYTES, dtype=torch.uint8, device=dev))
+    m = batch.numel()
+    rc = _lib.lib().mp_queues_push_all(dag.handle, A, _ptr(qptr_all), _ptr(qtask_all), _ptr(flags), _ptr(dur),
+                                       _ptr(batch) if m else None, m, _ptr(rem), _ptr(done), _ptr(out["qptr"]),
+                                       _ptr(out["qtask"]), _ptr(out["summary"]), _stream())
+    _lib.check(rc, "mp_queues_push_all")
+    return out["qptr"], out["qtask"], out["summary"]
+
+
 def summaries(summary_bytes: torch.Tensor) -> np.ndarray:
     """Host view of mp_queue_summary records."""
     return summary_bytes.detach().cpu().numpy().view(SUMMARY_DTYPE)

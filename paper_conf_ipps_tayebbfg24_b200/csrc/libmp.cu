@@ -115,6 +115,14 @@ mp_status mp_nod_remaining(mp_dag* dag, int32_t n_arch, const float* d_dur, cons
     return mph::nod_remaining(dag, n_arch, d_dur, h_workers, d_done, d_nod, as_stream(stream));
 }
 
+mp_status mp_queues_push_all(mp_dag* dag, int32_t n_arch, const int64_t* d_qptr_all, const int32_t* d_qtask_all,
+                             const uint8_t* d_flags, const float* d_dur, const int32_t* d_batch, int32_t m,
+                             int32_t* d_rem, uint8_t* d_done, int64_t* d_qptr_out, int32_t* d_qtask_out,
+                             mp_queue_summary* d_sum, void* stream) {
+    return mph::queues_push_all(dag, n_arch, d_qptr_all, d_qtask_all, d_flags, d_dur, d_batch, m, d_rem, d_done,
+                                d_qptr_out, d_qtask_out, d_sum, as_stream(stream));
+}
+
 mp_status mp_check(mp_dag* dag, void* stream) {
     if (!dag) return mph::fail(MP_ERR_ARG, "dag is NULL");
     cudaStream_t st = as_stream(stream);

@@ -7,6 +7,8 @@
 // newly ready (P:l.91) and joins every queue whose arch can run it (P:l.104,
 // Alg. 1), (c) merges the newly ready run, sorted by (key, id), into each
 // queue with merge-path partitions, and (d) recomputes the queue summaries.
+// mp_queues_push_all is the static-order variant: it keeps the ALL-mode queues
+// and a done mask instead of the current queues and needs no sort or merge.
 #pragma once
 #include "path.cuh"
 
@@ -193,9 +195,129 @@ __global__ void k_push_finish(int32_t A, const int64_t* qptr, const int32_t* q, 
     sum[a] = s;
 }
 
+// ---- static-order push (mp_queues_push_all) ------------------------------------------
+// Scores are whole-DAG (reading c18), so every READY-mode queue is the ALL-mode
+// queue restricted to the ready tasks, in the same order: a push is a release
+// followed by one stream compaction of the ALL-mode queues.
+
+// completed tasks: done[t] = 1, successors' counters decremented
+__global__ void k_pushall_release(const int32_t* batch, int32_t m, int32_t n, const int32_t* row_ptr,
+                                  const int32_t* col, int32_t* rem, uint8_t* done, uint32_t* err) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t u = batch[i];
+        if (u < 0 || u >= n) {
+            atomicOr(err, ERR_ARG_BIT);
+            continue;
+        }
+        if (rem[u] != 0 || done[u]) {          // not ready, or completed twice
+            atomicOr(err, ERR_ARG_BIT);
+            continue;
+        }
+        done[u] = 1;
+        for (int32_t e = row_ptr[u]; e < row_ptr[u + 1]; e++)
+            if (atomicSub(&rem[col[e]], 1) <= 0) atomicOr(err, ERR_ARG_BIT);
+    }
+}
+
+// keep[i] = 1 iff the task at ALL-mode position i is ready (not done, no pending predecessor)
+__global__ void k_pushall_flag(int64_t cap, int32_t A, const int64_t* qptr_all, const int32_t* qall,
+                               const int32_t* rem, const uint8_t* done, int32_t* keep) {
+    const int64_t Q = qptr_all[A];
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cap; i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t k = 0;
+        if (i < Q) {
+            const int32_t t = qall[i];
+            k = (!done[t] && rem[t] == 0) ? 1 : 0;
+        }
+        keep[i] = k;
+    }
+}
+
+// scatter the kept entries (global exclusive scan = output position, arch segments
+// stay contiguous) and sum best_remaining_work per arch
+__global__ void k_pushall_scatter(int32_t A, const int64_t* qptr_all, const int32_t* qall, const int32_t* keep,
+                                  const int32_t* pos, const uint8_t* flags, const float* dur, int32_t* qout,
+                                  unsigned long long* brw) {
+    const int a = blockIdx.y;
+    const int64_t b = qptr_all[a], e = qptr_all[a + 1];
+    uint64_t lo = 0, hi = 0;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t rounds = (e - b + stride - 1) / stride;
+    for (int64_t it = 0; it < rounds; it++) {
+        const int64_t i = b + it * stride + blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+        if (i < e && keep[i]) {
+            const int32_t t = qall[i];
+            qout[pos[i]] = t;
+            if (flags[(int64_t)t * A + a] & 2) {
+                bool dummy = false;
+                uint64_t l, h;
+                fixed64(canon_dur(dur[(int64_t)t * A + a], dummy), l, h);
+                add128(lo, hi, l, h);
+            }
+        }
+    }
+    warp_sum128(lo, hi);
+    if ((threadIdx.x & 31) == 0) atomic_add128(brw + 2 * a, lo, hi);
+}
+
+// qptr_out[a] = kept entries before arch a's segment; summaries
+__global__ void k_pushall_finish(int32_t A, int64_t cap, const int64_t* qptr_all, const int32_t* pos,
+                                 const int32_t* total, const int32_t* qout, const unsigned long long* brw,
+                                 int64_t* qptr_out, mp_queue_summary* sum) {
+    if (threadIdx.x > A) return;
+    const int a = threadIdx.x;
+    const int64_t s = qptr_all[a];
+    const int64_t o = s < cap ? (int64_t)pos[s] : (int64_t)*total;
+    qptr_out[a] = o;
+    if (a == A) return;
+    const int64_t s1 = qptr_all[a + 1];
+    const int64_t o1 = s1 < cap ? (int64_t)pos[s1] : (int64_t)*total;
+    mp_queue_summary r;
+    r.count = (int32_t)(o1 - o);
+    r.head = r.count > 0 ? qout[o] : -1;
+    r.brw_lo = brw[2 * a];
+    r.brw_hi = (int64_t)brw[2 * a + 1];
+    r.brw = u128_to_double_scaled(brw[2 * a], brw[2 * a + 1]);
+    sum[a] = r;
+}
+
 }  // namespace mpk
 
 namespace mph {
+
+inline mp_status queues_push_all(mp_dag* dag, int32_t A, const int64_t* qptr_all, const int32_t* qall,
+                                 const uint8_t* flags, const float* dur, const int32_t* batch, int32_t m,
+                                 int32_t* rem, uint8_t* done, int64_t* qptr_out, int32_t* qout,
+                                 mp_queue_summary* sum, cudaStream_t st) {
+    using namespace mpk;
+    if (!dag) return fail(MP_ERR_ARG, "dag is NULL");
+    if (A < 1 || A > MAX_ARCH) return fail(MP_ERR_ARG, "n_arch %d outside [1, 8]", A);
+    if (m < 0 || (m > 0 && !batch)) return fail(MP_ERR_ARG, "bad batch");
+    if (!qptr_all || !qptr_out || !sum || (dag->n > 0 && (!qall || !flags || !dur || !rem || !done || !qout)))
+        return fail(MP_ERR_ARG, "NULL buffer");
+    if (qall == qout) return fail(MP_ERR_ARG, "qtask_all and qtask_out must not alias");
+    const int32_t n = dag->n;
+    const int64_t cap = (int64_t)n * A > 0 ? (int64_t)n * A : 1;
+    MP_TRY(ensure_ws(dag, 2 * align256((size_t)cap * 4) + align256(64) + align256(16 * MAX_ARCH), st));
+    Arena ar{dag->ws, dag->ws_cap};
+    int32_t* keep = ar.take<int32_t>((size_t)cap);
+    int32_t* pos = ar.take<int32_t>((size_t)cap);
+    int32_t* total = ar.take<int32_t>(16);
+    unsigned long long* brw = ar.take<unsigned long long>(2 * MAX_ARCH);
+    MP_CUDA(cudaMemsetAsync(brw, 0, 16 * MAX_ARCH, st));
+    MP_CUDA(cudaMemsetAsync(total, 0, 4, st));
+    if (m > 0)
+        MP_LAUNCH(k_pushall_release, grid_for(m), 256, 0, st, batch, m, n, dag->row_ptr, dag->col, rem, done,
+                  dag->err);
+    // the ALL-mode queues hold at most n*A entries; their true length is qptr_all[A] (device)
+    MP_LAUNCH(k_pushall_flag, grid_for(cap), 256, 0, st, cap, A, qptr_all, qall, rem, done, keep);
+    MP_TRY(scan(dag, keep, pos, cap, total, st));
+    dim3 g(grid_for(cap, 256, 148 * 4), A);
+    MP_LAUNCH(k_pushall_scatter, g, 256, 0, st, A, qptr_all, qall, keep, pos, flags, dur, qout, brw);
+    MP_LAUNCH(k_pushall_finish, 1, 32, 0, st, A, cap, qptr_all, pos, total, qout, brw, qptr_out, sum);
+    MP_CUDA(cudaGetLastError());
+    return MP_OK;
+}
 
 inline mp_status ready_init(mp_dag* dag, int32_t* rem, cudaStream_t st) {
     using namespace mpk;

@@ -344,8 +344,8 @@ def test_ready_push_sequence_equals_ready_rebuild(name, A, steps):
     full = mp.score_and_queue(dag, dur, w.workers)
     key, flags = full["key"], full["flags"]
     od = oracle.build_dag(w.n, w.src, w.dst)
-    okey = key.cpu().numpy().view(np.uint64)
-    oflags = flags.cpu().numpy()
+    ofull = oracle.score_and_queue(od, w.dur, w.workers)      # oracle inputs come from the oracle
+    okey, oflags = ofull["key"], ofull["flags"]
     done = np.zeros(w.n, np.uint8)
     qptr, qtask, summ = mp.build_queues(dag, key, flags, dur, done=to_dev(done))
     rem = mp.ready_init(dag)
@@ -365,6 +365,51 @@ def test_ready_push_sequence_equals_ready_rebuild(name, A, steps):
         assert np.array_equal(qptr.cpu().numpy(), oq_ptr), step
         assert np.array_equal(qtask.cpu().numpy()[:oq_ptr[-1]], oq), step
         assert summ.cpu().numpy().tobytes() == osum.tobytes(), step
+
+
+@pytest.mark.parametrize("name,A", [("c1", 2), ("c2", 2), ("qr", 3)])
+def test_push_all_sequence_equals_ready_rebuild(name, A):
+    """N1 static-order push (mp_queues_push_all): after every batch the queues equal
+    the oracle's READY-mode rebuild, and the old merge push gives the same bytes."""
+    w = workloads.qr(10) if name == "qr" else workloads.config(name)
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    dur = to_dev(w.dur)
+    full = mp.score_and_queue(dag, dur, w.workers)            # ALL-mode queues
+    key, flags = full["key"], full["flags"]
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    ofull = oracle.score_and_queue(od, w.dur, w.workers)
+    okey, oflags = ofull["key"], ofull["flags"]
+    done_h = np.zeros(w.n, np.uint8)
+    done_d = torch.zeros(w.n, dtype=torch.uint8, device=DEV)
+    rem = mp.ready_init(dag)
+    rem2 = mp.ready_init(dag)
+    qptr, qtask, summ = mp.queues_push_all(dag, full["qptr"], full["qtask"], flags, dur,
+                                           torch.zeros(0, dtype=torch.int32, device=DEV), rem, done_d)
+    q2ptr, q2task, _ = mp.build_queues(dag, key, flags, dur, done=to_dev(done_h))
+    rng = np.random.default_rng(11)
+    steps = 0
+    while True:
+        mp.check(dag)
+        oq_ptr, oq, osum = oracle.build_queues(od, okey, oflags, w.dur, done_h)
+        assert np.array_equal(qptr.cpu().numpy(), oq_ptr), steps
+        assert np.array_equal(qtask.cpu().numpy()[:oq_ptr[-1]], oq), steps
+        assert summ.cpu().numpy().tobytes() == osum.tobytes(), steps
+        assert np.array_equal(q2task.cpu().numpy()[:oq_ptr[-1]], oq), steps
+        ready = np.unique(oq)
+        if len(ready) == 0:
+            break
+        k = int(rng.integers(1, min(len(ready), 300) + 1))
+        batch = rng.choice(ready, k, replace=False).astype(np.int32)
+        done_h[batch] = 1
+        qptr, qtask, summ = mp.queues_push_all(dag, full["qptr"], full["qtask"], flags, dur, to_dev(batch), rem,
+                                               done_d)
+        q2ptr, q2task, _ = mp.queues_push(dag, key, flags, dur, to_dev(batch), rem2, q2ptr, q2task)
+        steps += 1
+    assert done_h.all() and steps > 0
+    # a task completed twice is an argument error
+    mp.queues_push_all(dag, full["qptr"], full["qtask"], flags, dur, to_dev(np.array([0], np.int32)), rem, done_d)
+    with pytest.raises(mp.MPError):
+        mp.check(dag)
 
 
 # ----------------------------------------------------------------------------
