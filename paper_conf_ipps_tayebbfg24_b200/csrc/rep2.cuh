@@ -805,7 +805,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     S.clog = reinterpret_cast<uint8_t*>(S.coff + R3_NC + 64);
     S.sc = reinterpret_cast<uint32_t*>(S.clog + R3_NC + 64);
     S.misc = S.sc + 96;
-    __shared__ uint32_t s_tick, s_head, s_flag, s_h0, s_h1;
+    __shared__ uint32_t s_tick, s_head, s_flag, s_h0, s_h1, s_mtot;
     __shared__ unsigned long long s_min[A + 1], s_max[A + 1];
     const int64_t npad = ((int64_t)a.n + 15) & ~15ll;   // 16-entry aligned scratch rows
     uint32_t* critc = a.s_key + (int64_t)blockIdx.x * npad * (A + 3);
@@ -992,6 +992,88 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 }
             }
             __syncthreads();
+            // members of equal-gain runs (rare): their critc is gathered once, all loads in
+            // flight together, into shared memory (the sort's bin counters are free now):
+            // mw = member bits per 32 positions, mp = exclusive prefix of their popcounts,
+            // crs[mp[w] + rank in word] = critc of the task at that position
+            uint32_t* mw = S.starts;
+            uint32_t* mp = mw + nw;
+            uint32_t* crs = mp + nw;
+            const uint32_t ccap = (uint32_t)(R3_NF + 64) - 2u * (uint32_t)nw;
+            auto lt = [&](int32_t wb, int32_t x) -> uint32_t {   // bits i with wb + i < x
+                const int32_t c = x - wb;
+                return c <= 0 ? 0u : (c >= 32 ? 0xFFFFFFFFu : ((1u << c) - 1u));
+            };
+            uint32_t mloc[2], pre = 0;
+            {
+                uint32_t cnt = 0;
+#pragma unroll
+                for (int h = 0; h < 2; h++) {
+                    const int32_t w = 2 * (int32_t)threadIdx.x + h;
+                    uint32_t m = 0;
+                    if (w < nw) {
+                        const int32_t wb = w * 32;
+                        const uint32_t E1 = e1[w], E0 = e0[w];
+                        const uint32_t P1 = (E1 << 1) | (w > 0 ? e1[w - 1] >> 31 : 0u);   // bit(e1, p-1)
+                        const uint32_t P0 = (E0 << 1) | (w > 0 ? e0[w - 1] >> 31 : 0u);
+                        const uint32_t m1 = (P1 | (E1 & lt(wb, cG - 1))) & lt(wb, cG);
+                        const uint32_t ge0 = ~lt(wb, n1only), ge1 = ~lt(wb, n1only + 1);
+                        const uint32_t m0 = (P0 & ge1) | (E0 & ge0);
+                        m = (m0 | m1) & lt(wb, a.n);
+                    }
+                    mloc[h] = m;
+                    cnt += __popc(m);
+                }
+                uint32_t tot;
+                pre = r3_scan(cnt, S.sc, tot);
+                if (threadIdx.x == 0) s_mtot = tot;
+            }
+#pragma unroll
+            for (int h = 0; h < 2; h++) {
+                const int32_t w = 2 * (int32_t)threadIdx.x + h;
+                if (w < nw) {
+                    mw[w] = mloc[h];
+                    mp[w] = pre;
+                }
+                pre += __popc(mloc[h]);
+            }
+            __syncthreads();
+            const bool mfit = s_mtot <= ccap;
+            if (mfit) {
+#pragma unroll
+                for (int h = 0; h < 2; h++) {
+                    const int32_t w = 2 * (int32_t)threadIdx.x + h;
+                    if (w >= nw) continue;
+                    uint32_t m = mloc[h];
+                    uint32_t idx = mp[w];
+                    while (m) {   // up to 4 gathers in flight per thread
+                        uint32_t tq[4], ix[4];
+                        int c = 0;
+#pragma unroll
+                        for (int u = 0; u < 4; u++) {
+                            if (m) {
+                                const int b = __ffs(m) - 1;
+                                m &= m - 1u;
+                                tq[u] = __ldg(a.qof + Ps[w * 32 + b]);
+                                ix[u] = idx++;
+                                c = u + 1;
+                            }
+                        }
+                        float bv[4];
+#pragma unroll
+                        for (int u = 0; u < 4; u++) bv[u] = u < c ? __ldcg(blr + (int64_t)tq[u] * 32) : 0.0f;
+#pragma unroll
+                        for (int u = 0; u < 4; u++)
+                            if (u < c) crs[ix[u]] = ONE_BITS - f2u(CP > 0.0f ? __fdiv_rn(bv[u], CP) : 0.0f);
+                    }
+                }
+            }
+            __syncthreads();
+            auto crit_at = [&](int32_t i) -> uint32_t {   // critc of the task at sorted position i
+                if (!mfit) return critc_of(Ps[i]);
+                const uint32_t m = mw[i >> 5];
+                return crs[mp[i >> 5] + __popc(m & ((1u << (i & 31)) - 1u))];
+            };
             auto bit = [&](const uint32_t* e, int32_t i) -> bool { return (e[i >> 5] >> (i & 31)) & 1u; };
             for (int32_t p = threadIdx.x; p < a.n; p += R2_THREADS) {
                 const uint32_t t = Ps[p];
@@ -1006,11 +1088,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         while (hi + 1 < cG && hi - p < 64 && bit(e1, hi)) hi++;
                         if ((lo > 0 && bit(e1, lo - 1)) || (hi + 1 < cG && bit(e1, hi))) s_flag = 1;
                         {   // the sort ordered the run by (d, id): rank it by (critc, id)
-                            const uint64_t me = ((uint64_t)critc_of(t) << 16) | t;
+                            const uint64_t me = ((uint64_t)crit_at(p) << 16) | t;
                             int32_t rk = 0;
                             for (int32_t i = lo; i <= hi; i++) {
                                 const uint32_t ti = Ps[i];
-                                rk += (((uint64_t)critc_of(ti) << 16) | ti) < me ? 1 : 0;
+                                rk += (((uint64_t)crit_at(i) << 16) | ti) < me ? 1 : 0;
                             }
                             pos = lo + rk;
                         }
@@ -1030,11 +1112,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         if ((lo > n1only && bit(e0, lo - 1)) || (hi + 1 < a.n && bit(e0, hi))) s_flag = 1;
                         const int32_t base = a.n - 1 - hi;   // the run's block in queue 0
                         {   // the sort ordered the run by (d, id): rank it by (critc, id)
-                            const uint64_t me = ((uint64_t)critc_of(t) << 16) | t;
+                            const uint64_t me = ((uint64_t)crit_at(p) << 16) | t;
                             int32_t rk = 0;
                             for (int32_t i = lo; i <= hi; i++) {
                                 const uint32_t ti = Ps[i];
-                                rk += (((uint64_t)critc_of(ti) << 16) | ti) < me ? 1 : 0;
+                                rk += (((uint64_t)crit_at(i) << 16) | ti) < me ? 1 : 0;
                             }
                             pos = base + rk;
                         }
