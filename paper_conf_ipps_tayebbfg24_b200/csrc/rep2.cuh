@@ -502,7 +502,12 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
         const uint32_t s0 = (f == b0 ? base : S.starts[f - 1]) - base;
         const uint32_t s1 = S.starts[f] - base;
         uint32_t rank = 0;
-        for (uint32_t i = s0; i < s1; i++) rank += r3_less<KT>(bk[i], bv[i], k, v) ? 1u : 0u;
+        uint32_t i = s0;
+        for (; i + 4 <= s1; i += 4) {   // 4 independent compares per trip
+#pragma unroll
+            for (int u = 0; u < 4; u++) rank += r3_less<KT>(bk[i + u], bv[i + u], k, v) ? 1u : 0u;
+        }
+        for (; i < s1; i++) rank += r3_less<KT>(bk[i], bv[i], k, v) ? 1u : 0u;
         out.put(ob + (int32_t)(s0 + rank), v, k64);
     }
     __syncthreads();
