@@ -207,4 +207,15 @@ int64_t mp_prof_names(char* buf, int64_t len) {
     return (int64_t)all.size();
 }
 
+#ifdef MP_PHASES
+// debug build only (tools/k2_phases.py): accumulated K2 phase cycles (thread 0 of every CTA)
+int mp_debug_k2_phases(unsigned long long* h_out32, int reset) {
+    if (cudaMemcpyFromSymbol(h_out32, mpk::g_k2_phase, 32 * sizeof(unsigned long long)) != cudaSuccess) return 1;
+    if (reset) {
+        static const unsigned long long z[32] = {};
+        if (cudaMemcpyToSymbol(mpk::g_k2_phase, z, sizeof(z)) != cudaSuccess) return 1;
+    }
+    return 0;
+}
+#endif
 }  // extern "C"

@@ -26,6 +26,24 @@ constexpr int R2_WARPS = 32;
 constexpr int R2_CAP = 16384;
 constexpr int R2_NBINS = 4096;
 
+// Optional per-phase cycle accounting of K2 (build with -DMP_PHASES; tools/k2_phases.py).
+#ifdef MP_PHASES
+__device__ unsigned long long g_k2_phase[32];
+MP_INLINE void k2_phase(int i) {
+    __shared__ long long s_t;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const long long t = clock64();
+        if (i > 0) atomicAdd(&g_k2_phase[i], (unsigned long long)(t - s_t));
+        s_t = t;
+    }
+    __syncthreads();
+}
+#define K2_PHASE(i) k2_phase(i)
+#else
+#define K2_PHASE(i) ((void)0)
+#endif
+
 struct Rep2Args {
     int32_t n, A, L, R;
     int64_t r0;                  // global id of replica 0 of this call
@@ -46,8 +64,9 @@ struct Rep2Args {
     unsigned long long* brw;     // [R][A][2]
     uint32_t* err;
     // K2
-    uint32_t* s_key;             // [grid][n]   per-CTA scratch keys
-    uint16_t* s_pi;              // [grid][n]   per-CTA crit order
+    uint32_t* s_key;             // [grid][2][npad] per-CTA hot scratch: D in id order, D in sorted order
+    uint16_t* s_pi;              // [grid][2][npad] per-CTA hot scratch: fine-bin ids, sorted positions
+    uint32_t* s_cold;            // [grid][A+1][npad] general path only: critc, gainc per arch
     int32_t* qtask;              // [R][n*A] or null
     mp_queue_summary* sum;       // [R][A]
     uint32_t* ticket;
@@ -587,6 +606,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
             }
         }
         __syncthreads();
+        K2_PHASE(2);
         // ---- sub-bins per coarse bin: 2^ceil(log2(c / T)) with T doubling until they fit ----
         constexpr int CPER = R3_NC / R2_THREADS;  // 4
         uint32_t cc[CPER];
@@ -631,6 +651,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         for (int w = 0; w < R2_WARPS; w++) need = max(need, S.sc[40 + w]);
         need = g.cs - need;   // fine bins use key bits >= need
         const uint32_t nfb = ftot;
+        K2_PHASE(3);
         // ---- pass 2: fine histogram ----
         for (int32_t c0 = threadIdx.x * 8; c0 < n; c0 += 8 * R2_THREADS) {
             uint32_t hv[8], fv[8];
@@ -666,6 +687,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
             }
         }
         __syncthreads();
+        K2_PHASE(4);
         // ---- prefixes over fine bins (12 per thread) + group boundaries ----
         constexpr int PER = R3_NF / R2_THREADS;  // 12
         const uint32_t H = CAPK - R3_MID;        // a multi-bin group never exceeds H + MID = CAP
@@ -711,6 +733,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
                 }
         }
         __syncthreads();
+        K2_PHASE(5);
         for (uint32_t gi = 0; gi < ng; gi++) {
             const uint32_t b0 = grp[gi * 3], e0 = grp[gi * 3 + 1], kind = grp[gi * 3 + 2];
             const uint32_t b1 = gi + 1 < ng ? grp[(gi + 1) * 3] : nfb;
@@ -791,12 +814,15 @@ MP_INLINE void r2_same_gains(uint32_t Da, uint32_t Db, float hd, bool& s0, bool&
     }
     const float da = u2f((Da & 0x80000000u) ? (Da & 0x7FFFFFFFu) : ~Da);
     const float db = u2f((Db & 0x80000000u) ? (Db & 0x7FFFFFFFu) : ~Db);
+    // screen in float: lim = den * 2^-24 is exact (den >= 2^-40 for a nonzero hd in the
+    // domain), and RN is monotone, so a true |xb - xa| <= lim never rounds above lim;
+    // a rounded difference above lim is a true difference above lim (different gains)
     const float den = __fadd_rn(hd, hd);
-    const double lim = (double)den * 0x1p-24;
+    const float lim = __fmul_rn(den, 0x1p-24f);
     const float xa = __fadd_rn(da, hd), xb = __fadd_rn(db, hd);
-    s0 = xa == xb || (fabs((double)xb - (double)xa) <= lim && __fdiv_rn(xa, den) == __fdiv_rn(xb, den));
+    s0 = xa == xb || (fabsf(__fsub_rn(xb, xa)) <= lim && __fdiv_rn(xa, den) == __fdiv_rn(xb, den));
     const float ya = __fadd_rn(__fsub_rn(0.0f, da), hd), yb = __fadd_rn(__fsub_rn(0.0f, db), hd);
-    s1 = ya == yb || (fabs((double)yb - (double)ya) <= lim && __fdiv_rn(ya, den) == __fdiv_rn(yb, den));
+    s1 = ya == yb || (fabsf(__fsub_rn(yb, ya)) <= lim && __fdiv_rn(ya, den) == __fdiv_rn(yb, den));
 }
 
 
@@ -813,9 +839,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     __shared__ uint32_t s_tick, s_head, s_flag, s_h0, s_h1, s_mtot;
     __shared__ unsigned long long s_min[A + 1], s_max[A + 1];
     const int64_t npad = ((int64_t)a.n + 15) & ~15ll;   // 16-entry aligned scratch rows
-    uint32_t* critc = a.s_key + (int64_t)blockIdx.x * npad * (A + 3);
+    uint32_t* critc = a.s_cold + (int64_t)blockIdx.x * npad * (A + 1);
     uint32_t* gainc = critc + npad;   // [A][npad]
-    uint32_t* dkey = gainc + (int64_t)A * npad;
+    uint32_t* dkey = a.s_key + (int64_t)blockIdx.x * npad * 2;
     uint16_t* fbuf = a.s_pi + (int64_t)blockIdx.x * npad * 2;
     uint16_t* ppos = fbuf + npad;
     uint32_t* dsorted = dkey + npad;   // (A == 2) D in sorted order (gains are recomputed from it)
@@ -830,6 +856,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         const int64_t rl = s_tick;
         __syncthreads();
         if (rl >= a.R) break;
+        K2_PHASE(0);
         const int64_t r = a.r0 + rl;
         const float CP = a.cp[rl];
         float hdv[A];
@@ -941,7 +968,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         bool done = false;
         if constexpr (A == 2) {
             // one sort by (D, critc, t) -> P; then both queues in one pass (runs of equal gain fixed up)
+            K2_PHASE(1);
             r3_sort<uint32_t>(R3Keys{dkey, nullptr, fbuf}, R3PosOut{ppos, dsorted}, a.n, s_min[A] & ~0xFFFFFFFFull, s_max[A] & ~0xFFFFFFFFull, S);
+            K2_PHASE(7);
             if (threadIdx.x == 0) { s_flag = 0; s_h0 = 0xffffffffu; s_h1 = 0xffffffffu; }
             __syncthreads();
             const int32_t cC = a.counts[rl * 2 + 0], cG = a.counts[rl * 2 + 1];
@@ -956,42 +985,64 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 return ONE_BITS - f2u(c);
             };
             // sorted order into shared memory (the sort's buffers are free now) + neighbour-equality
-            // bits: e0/e1 = same gain as the next position (arch 0 / arch 1), eD = same D
+            // bits: e0/e1 = same gain as the next position (arch 0 / arch 1)
             uint16_t* Ps = reinterpret_cast<uint16_t*>(S.bkraw);
             const int32_t nw = (a.n + 31) / 32;
             uint32_t* e0 = reinterpret_cast<uint32_t*>(Ps + ((a.n + 63) & ~63));
             uint32_t* e1 = e0 + nw;
-            uint32_t* eD = e1 + nw;
-            for (int32_t i = threadIdx.x; i < a.n; i += R2_THREADS) Ps[i] = ppos[i];
-            __syncthreads();
+            {   // 16-byte copies (ppos and Ps are 32-byte aligned)
+                const int32_t n8 = a.n >> 3;
+                for (int32_t i = threadIdx.x; i < n8; i += R2_THREADS)
+                    reinterpret_cast<uint4*>(Ps)[i] = __ldcg(reinterpret_cast<const uint4*>(ppos) + i);
+                for (int32_t i = (n8 << 3) + threadIdx.x; i < a.n; i += R2_THREADS) Ps[i] = ppos[i];
+            }
             {
+                K2_PHASE(8);
+                // 4 consecutive positions per lane (one 16-byte load), 128 per warp and chunk,
+                // two chunks in flight; nibbles of 8 lanes OR-ed into one bit word
                 const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-                for (int32_t wb0 = w * 32; wb0 < a.n; wb0 += 2 * R2_THREADS) {
-                    uint32_t DDv[2], NDv[2];
+                constexpr int32_t CH = 128, STEP = CH * R2_WARPS;
+                for (int32_t cb0 = w * CH; cb0 < a.n; cb0 += 2 * STEP) {
+                    uint32_t Dv[2][4], nx[2];
 #pragma unroll
-                    for (int h = 0; h < 2; h++) {      // loads of both chunks first
-                        const int32_t p = wb0 + h * R2_THREADS + lane;
-                        DDv[h] = p < a.n ? __ldcg(dsorted + p) : 0u;
-                        NDv[h] = (lane == 31 && p + 1 < a.n) ? __ldcg(dsorted + p + 1) : 0u;
+                    for (int h = 0; h < 2; h++) {
+                        const int32_t p4 = cb0 + h * STEP + lane * 4;
+                        if (p4 + 4 <= a.n) {
+                            const uint4 v = __ldcg(reinterpret_cast<const uint4*>(dsorted + p4));
+                            Dv[h][0] = v.x; Dv[h][1] = v.y; Dv[h][2] = v.z; Dv[h][3] = v.w;
+                        } else {
+#pragma unroll
+                            for (int j = 0; j < 4; j++) Dv[h][j] = p4 + j < a.n ? __ldcg(dsorted + p4 + j) : 0u;
+                        }
+                        nx[h] = (lane == 31 && p4 + 4 < a.n) ? __ldcg(dsorted + p4 + 4) : 0u;
                     }
 #pragma unroll
                     for (int h = 0; h < 2; h++) {
-                        const int32_t wb = wb0 + h * R2_THREADS;
-                        if (wb >= a.n) break;
-                        const int32_t p = wb + lane;
-                        const uint32_t DD = DDv[h];
-                        uint32_t ND = __shfl_down_sync(0xffffffffu, DD, 1);
-                        if (lane == 31) ND = p + 1 < a.n ? NDv[h] : ~DD;
-                        const bool ok = p + 1 < a.n;
-                        bool same0 = false, same1 = false;
-                        if (ok) r2_same_gains(DD, ND, h2, same0, same1);
-                        const uint32_t b0 = __ballot_sync(0xffffffffu, same0);
-                        const uint32_t b1 = __ballot_sync(0xffffffffu, same1);
-                        const uint32_t bD = __ballot_sync(0xffffffffu, ok && DD == ND);
-                        if (lane == 0) {
-                            e0[wb >> 5] = b0;
-                            e1[wb >> 5] = b1;
-                            eD[wb >> 5] = bD;
+                        const int32_t cb = cb0 + h * STEP;
+                        if (cb >= a.n) break;
+                        const int32_t p4 = cb + lane * 4;
+                        uint32_t nxt = __shfl_down_sync(0xffffffffu, Dv[h][0], 1);
+                        if (lane == 31) nxt = nx[h];
+                        uint32_t n0 = 0, n1 = 0;
+#pragma unroll
+                        for (int j = 0; j < 4; j++) {
+                            if (p4 + j + 1 < a.n) {
+                                bool s0, s1;
+                                r2_same_gains(Dv[h][j], j < 3 ? Dv[h][j + 1] : nxt, h2, s0, s1);
+                                n0 |= (uint32_t)s0 << j;
+                                n1 |= (uint32_t)s1 << j;
+                            }
+                        }
+                        n0 <<= (lane & 7) * 4;
+                        n1 <<= (lane & 7) * 4;
+#pragma unroll
+                        for (int o = 1; o < 8; o <<= 1) {
+                            n0 |= __shfl_xor_sync(0xffffffffu, n0, o);
+                            n1 |= __shfl_xor_sync(0xffffffffu, n1, o);
+                        }
+                        if ((lane & 7) == 0 && p4 < a.n) {
+                            e0[(cb >> 5) + (lane >> 3)] = n0;
+                            e1[(cb >> 5) + (lane >> 3)] = n1;
                         }
                     }
                 }
@@ -1001,10 +1052,12 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             // flight together, into shared memory (the sort's bin counters are free now):
             // mw = member bits per 32 positions, mp = exclusive prefix of their popcounts,
             // crs[mp[w] + rank in word] = critc of the task at that position
+            K2_PHASE(9);
             uint32_t* mw = S.starts;
             uint32_t* mp = mw + nw;
             uint32_t* crs = mp + nw;
-            const uint32_t ccap = (uint32_t)(R3_NF + 64) - 2u * (uint32_t)nw;
+            const uint32_t ccap = ((uint32_t)(R3_NF + 64) - 2u * (uint32_t)nw) * 4u / 6u;
+            uint16_t* mpos = reinterpret_cast<uint16_t*>(crs + ccap);   // position of member #i
             auto lt = [&](int32_t wb, int32_t x) -> uint32_t {   // bits i with wb + i < x
                 const int32_t c = x - wb;
                 return c <= 0 ? 0u : (c >= 32 ? 0xFFFFFFFFu : ((1u << c) - 1u));
@@ -1060,6 +1113,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                                 const int b = __ffs(m) - 1;
                                 m &= m - 1u;
                                 tq[u] = __ldg(a.qof + Ps[w * 32 + b]);
+                                mpos[idx] = (uint16_t)(w * 32 + b);
                                 ix[u] = idx++;
                                 c = u + 1;
                             }
@@ -1074,13 +1128,31 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 }
             }
             __syncthreads();
+            K2_PHASE(10);
             auto crit_at = [&](int32_t i) -> uint32_t {   // critc of the task at sorted position i
                 if (!mfit) return critc_of(Ps[i]);
                 const uint32_t m = mw[i >> 5];
                 return crs[mp[i >> 5] + __popc(m & ((1u << (i & 31)) - 1u))];
             };
             auto bit = [&](const uint32_t* e, int32_t i) -> bool { return (e[i >> 5] >> (i & 31)) & 1u; };
-            for (int32_t p = threadIdx.x; p < a.n; p += R2_THREADS) {
+            if (mfit) {   // positions in no equal-gain run go straight to both queues (coalesced)
+                for (int32_t p = threadIdx.x; p < a.n; p += R2_THREADS) {
+                    if ((mw[p >> 5] >> (p & 31)) & 1u) continue;
+                    const uint32_t t = Ps[p];
+                    if (p < cG) {
+                        if (p == 0) s_h1 = t;
+                        if (q1) __stcs(q1 + p, (int32_t)t);
+                    }
+                    if (p >= n1only) {
+                        if (p == a.n - 1) s_h0 = t;
+                        if (q0) __stcs(q0 + (a.n - 1 - p), (int32_t)t);
+                    }
+                }
+            }
+            // members (all positions when they did not fit): rank inside their runs
+            const int32_t nslow = mfit ? (int32_t)s_mtot : a.n;
+            for (int32_t ii = threadIdx.x; ii < nslow; ii += R2_THREADS) {
+                const int32_t p = mfit ? (int32_t)mpos[ii] : ii;
                 const uint32_t t = Ps[p];
                 // arch 1 (forward order), positions [0, cG); p and p+1 in one run iff bit(e1, p)
                 if (p < cG) {
@@ -1131,6 +1203,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 }
             }
             __syncthreads();
+            K2_PHASE(11);
             if (!s_flag) {
                 done = true;
                 if (threadIdx.x < 2) {
@@ -1148,6 +1221,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             }
             __syncthreads();
         }
+        K2_PHASE(12);
         if (done) continue;
         if constexpr (A == 2) {
             // fallback for this replica: materialise both archs' gain keys and ranges
@@ -1222,6 +1296,40 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
 
 namespace mph {
 
+// L2 persisting carve-out for K2's scratch (opt-in: MP_L2_PERSIST=1; set once per process)
+inline size_t l2_persist_bytes() {
+    static size_t v = [] {
+        const char* e = getenv("MP_L2_PERSIST");   // opt-in: measured no gain on c5, K1 slower
+        if (!e || atoi(e) == 0) return (size_t)0;
+        int dev = 0, mx = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess) return (size_t)0;
+        if (cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev) != cudaSuccess || mx <= 0) {
+            cudaGetLastError();
+            return (size_t)0;
+        }
+        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)mx) != cudaSuccess) {
+            cudaGetLastError();
+            return (size_t)0;
+        }
+        size_t got = 0;
+        cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize);
+        return got;
+    }();
+    return v;
+}
+inline size_t l2_window_max() {
+    static size_t v = [] {
+        int dev = 0, mx = 0;
+        cudaGetDevice(&dev);
+        if (cudaDeviceGetAttribute(&mx, cudaDevAttrMaxAccessPolicyWindowSize, dev) != cudaSuccess) {
+            cudaGetLastError();
+            return (size_t)0;
+        }
+        return (size_t)mx;
+    }();
+    return v;
+}
+
 template <int A>
 inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uint64_t seed, float sigma, int64_t r0,
                              int32_t R, float* cp, mp_queue_summary* sum, int32_t* qtask, cudaStream_t st) {
@@ -1231,7 +1339,8 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
     const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
-                   align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 3)) + align256((size_t)grid2 * ((n + 15) & ~15) * 4);
+                   align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 8) +
+                   align256((size_t)grid2 * ((n + 15) & ~15) * 4);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
     Rep2Args a{};
@@ -1256,8 +1365,10 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.counts = ar.take<int32_t>((size_t)R * A);
     a.brw = ar.take<unsigned long long>((size_t)R * A * 2);
     a.err = dag->err;
-    a.s_key = ar.take<uint32_t>((size_t)grid2 * ((n + 15) & ~15) * (A + 3));
-    a.s_pi = ar.take<uint16_t>((size_t)grid2 * ((n + 15) & ~15) * 2);
+    const size_t npad = (size_t)((n + 15) & ~15);
+    a.s_cold = ar.take<uint32_t>((size_t)grid2 * npad * (A + 1));
+    a.s_key = ar.take<uint32_t>((size_t)grid2 * npad * 2);   // hot scratch: s_key and s_pi adjacent
+    a.s_pi = ar.take<uint16_t>((size_t)grid2 * npad * 2);
     a.qtask = qtask;
     a.sum = sum;
     a.ticket = dag->tickets + 56;
@@ -1306,7 +1417,35 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         if (cs == 1) return fail(MP_ERR_CUDA, "k_rep2_bl launch: %s", cudaGetErrorString(e));
     }
     MP_CUDA(cudaMemsetAsync(a.ticket, 0, 4, st));
-    MP_LAUNCH(k_rep2_sort<A>, (unsigned)grid2, R2_THREADS, smem2, st, a);
+    {
+        // K2's hot per-CTA scratch (~12 B per task per CTA: 81 MB for c2 on 148 SMs) is
+        // re-read by every pass of the in-CTA sort: keep it L2-resident (persisting
+        // access-policy window; the queue stores stream past it with evict-first)
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)grid2);
+        cfg.blockDim = dim3(R2_THREADS);
+        cfg.dynamicSmemBytes = (size_t)smem2;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        int na = 0;
+        const size_t hot = (size_t)(reinterpret_cast<char*>(a.s_pi + (size_t)grid2 * npad * 2) -
+                                    reinterpret_cast<char*>(a.s_key));
+        const size_t persist = l2_persist_bytes();
+        if (persist > 0) {
+            at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+            at[0].val.accessPolicyWindow.base_ptr = a.s_key;
+            at[0].val.accessPolicyWindow.num_bytes = std::min(hot, l2_window_max());
+            at[0].val.accessPolicyWindow.hitRatio =
+                (float)std::min(1.0, (double)persist / (double)at[0].val.accessPolicyWindow.num_bytes);
+            at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+            at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+            na = 1;
+        }
+        cfg.attrs = at;
+        cfg.numAttrs = na;
+        mph::ProfScope ps("k_rep2_sort<A>", st);
+        MP_CUDA(cudaLaunchKernelEx(&cfg, k_rep2_sort<A>, a));
+    }
     MP_CUDA(cudaGetLastError());
     return MP_OK;
 }

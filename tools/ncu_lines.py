@@ -33,16 +33,23 @@ for r in rows[2:]:
 base = int(data[0][0], 16)
 col = "Warp Stall Sampling (All Samples)"
 agg = collections.Counter()
+reasons = collections.defaultdict(collections.Counter)
+rcols = [k for k in h if k.startswith("stall_") and "Not Issued" not in k]
 for r in data:
-    agg[fmap.get(int(r[0], 16) - base)] += int(r[I[col]] or 0)
+    key = fmap.get(int(r[0], 16) - base)
+    agg[key] += int(r[I[col]] or 0)
+    for k in rcols:
+        reasons[key][k[6:]] += int(r[I[k]] or 0)
 tot = sum(agg.values()) or 1
 srcs = {}
 for (k, c) in agg.most_common(top):
     if k is None:
         print(f"{100*c/tot:5.1f}%  ?"); continue
     f, ln = k
+    k = (f, ln)
     if f not in srcs:
         p = os.path.join(os.path.dirname(lib), "csrc", f)
         srcs[f] = open(p).read().split("\n") if os.path.exists(p) else []
     txt = srcs[f][ln - 1].strip() if ln - 1 < len(srcs[f]) else ""
-    print(f"{100*c/tot:5.1f}%  {f}:{ln}  {txt[:100]}")
+    rs = " ".join(f"{k}:{v}" for k, v in reasons[k].most_common(3) if v) if os.environ.get("REASONS") else ""
+    print(f"{100*c/tot:5.1f}%  {f}:{ln}  {txt[:90]}  {rs}")
