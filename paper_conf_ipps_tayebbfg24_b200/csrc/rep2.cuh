@@ -513,6 +513,7 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
         bv[slot] = (uint16_t)t;
     }
     __syncthreads();
+    K2_PHASE(13);
     for (uint32_t j = threadIdx.x; j < cnt; j += R2_THREADS) {
         const KT k = bk[j];
         const uint16_t v = bv[j];
@@ -530,6 +531,7 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
         out.put(ob + (int32_t)(s0 + rank), v, k64);
     }
     __syncthreads();
+    K2_PHASE(14);
 }
 
 MP_INLINE uint32_t r3_clog2(uint32_t x) { return x <= 1 ? 0u : 32u - __clz(x - 1); }   // ceil(log2 x)
@@ -826,6 +828,11 @@ MP_INLINE void r2_same_gains(uint32_t Da, uint32_t Db, float hd, bool& s0, bool&
 }
 
 
+// RN(xa / den) == RN(xb / den) for numerators in [0, den] (see r2_same_gains)
+MP_INLINE bool r2_same_q(float xa, float xb, float den, float lim) {
+    return xa == xb || (fabsf(__fsub_rn(xb, xa)) <= lim && __fdiv_rn(xa, den) == __fdiv_rn(xb, den));
+}
+
 template <int A>
 __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     extern __shared__ __align__(16) unsigned char r3s[];
@@ -868,13 +875,21 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
 #pragma unroll
         for (int b = 0; b <= A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
         if constexpr (A == 2) {
-            // two archs: only the orderable d is needed to sort (crit is read for equal-gain runs)
-            for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
-                float x[A];
-                uint32_t en;
-                int k;
-                float wt;
-                r2_durs<A>(a, r, t, x, en, k, wt, bad);
+            // two archs: only the orderable d is needed to sort (crit is read for equal-gain runs).
+            // 4 tasks per thread and trip (t, t+1 | t+2048, t+2049): both 16-byte base loads
+            // are issued before the hashing
+            uint32_t dmn = ~0u, dmx = 0u;
+            auto one = [&](int32_t t, float b0v, float b1v) {
+                const float bb[2] = {b0v, b1v};
+                const uint64_t c0 = ((uint64_t)r * (uint64_t)a.n + (uint64_t)t) * 2u + 1u;
+                uint32_t en = 0;
+                float x[2];
+#pragma unroll
+                for (int b = 0; b < 2; b++) {
+                    x[b] = canon_dur(perturb(bb[b], a.seed, a.sigma, c0 + b), bad);
+                    if (((a.emask >> b) & 1u) && !is_inf(x[b])) en |= 1u << b;
+                }
+                if (!en) bad = true;
                 uint32_t D;
                 if (en == 3u) {
                     const uint32_t db = f2u(__fsub_rn(x[1], x[0]));
@@ -883,10 +898,27 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                     D = en == 1u ? 0xFFFFFFFFu : 0u;
                 }
                 dkey[t] = D;
-                const unsigned long long full = (unsigned long long)D << 32;
-                mn[A] = full < mn[A] ? full : mn[A];
-                mx[A] = full > mx[A] ? full : mx[A];
+                dmn = min(dmn, D);
+                dmx = max(dmx, D);
+            };
+            const bool al = (reinterpret_cast<uintptr_t>(a.base) & 15u) == 0;
+            const int32_t n2 = al ? (a.n & ~1) : 0;
+            for (int32_t t0 = 2 * threadIdx.x; t0 < n2; t0 += 4 * R2_THREADS) {
+                const int32_t t1 = t0 + 2 * R2_THREADS;
+                const float4 v0 = __ldg(reinterpret_cast<const float4*>(a.base) + (t0 >> 1));
+                float4 v1 = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (t1 < n2) v1 = __ldg(reinterpret_cast<const float4*>(a.base) + (t1 >> 1));
+                one(t0, v0.x, v0.y);
+                one(t0 + 1, v0.z, v0.w);
+                if (t1 < n2) {
+                    one(t1, v1.x, v1.y);
+                    one(t1 + 1, v1.z, v1.w);
+                }
             }
+            for (int32_t t = n2 + threadIdx.x; t < a.n; t += R2_THREADS)
+                one(t, __ldg(a.base + 2 * (int64_t)t), __ldg(a.base + 2 * (int64_t)t + 1));
+            mn[A] = (unsigned long long)dmn << 32;
+            mx[A] = (unsigned long long)dmx << 32;
         }
         const bool vec4 = (a.n & 3) == 0;   // 16-byte loads of bl when rows stay aligned
         for (int32_t t0 = vec4 ? threadIdx.x * 4 : threadIdx.x; A != 2 && t0 < a.n; t0 += vec4 ? 4 * R2_THREADS : R2_THREADS) {
@@ -1023,12 +1055,31 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         const int32_t p4 = cb + lane * 4;
                         uint32_t nxt = __shfl_down_sync(0xffffffffu, Dv[h][0], 1);
                         if (lane == 31) nxt = nx[h];
+                        // numerators x = d + hd (arch 0) and y = -d + hd (arch 1) once per position
+                        uint32_t Dj[5] = {Dv[h][0], Dv[h][1], Dv[h][2], Dv[h][3], nxt};
+                        float xs[5], ys[5];
+                        bool gen = h2 == 0.0f;   // sentinels or hd = 0: the generic comparison
+#pragma unroll
+                        for (int j = 0; j < 5; j++) {
+                            const uint32_t D = Dj[j];
+                            gen |= (D == 0u || D == 0xFFFFFFFFu) && (j < 4 ? p4 + j < a.n : p4 + 4 < a.n);
+                            const float d = u2f((D & 0x80000000u) ? (D & 0x7FFFFFFFu) : ~D);
+                            xs[j] = __fadd_rn(d, h2);
+                            ys[j] = __fadd_rn(__fsub_rn(0.0f, d), h2);
+                        }
+                        const float den = __fadd_rn(h2, h2);
+                        const float lim = __fmul_rn(den, 0x1p-24f);
                         uint32_t n0 = 0, n1 = 0;
 #pragma unroll
                         for (int j = 0; j < 4; j++) {
                             if (p4 + j + 1 < a.n) {
                                 bool s0, s1;
-                                r2_same_gains(Dv[h][j], j < 3 ? Dv[h][j + 1] : nxt, h2, s0, s1);
+                                if (gen) {
+                                    r2_same_gains(Dj[j], Dj[j + 1], h2, s0, s1);
+                                } else {
+                                    s0 = r2_same_q(xs[j], xs[j + 1], den, lim);
+                                    s1 = r2_same_q(ys[j], ys[j + 1], den, lim);
+                                }
                                 n0 |= (uint32_t)s0 << j;
                                 n1 |= (uint32_t)s1 << j;
                             }

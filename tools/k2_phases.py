@@ -25,7 +25,7 @@ for it in range(3):
     torch.cuda.synchronize()
 L.mp_debug_k2_phases(buf.ctypes.data, 1)
 names = {1: "P0 hash+D+minmax", 2: "pass1 coarse hist", 3: "sub-bins", 4: "pass2 fine hist+fb", 5: "prefix+groups",
-         7: "rounds (place+rank+out)", 8: "Ps copy", 9: "eq bits", 10: "members+crit", 11: "emission", 12: "summary"}
+         7: "rounds (place+rank+out)", 8: "Ps copy", 9: "eq bits", 10: "members+crit", 11: "emission", 12: "summary", 13: "  round: scan+place", 14: "  round: rank+out"}
 tot = buf.sum()
 for i in sorted(names):
     print(f"{names[i]:28s} {100.0 * buf[i] / tot:5.1f}%  {buf[i] / R / 1.965e3:8.2f} us/replica")
