@@ -434,8 +434,17 @@ MP_INLINE bool r3_locate_hk(const R3Keys& K, int32_t t, uint32_t h, const R3Geo&
     return true;
 }
 
+// Fine bin of a key in coarse bin cb.  64-bit keys: 2^clog[cb] power-of-two sub-bins (a
+// fine bin depends only on key bits >= cs - clog, so critc is read only where needed).
+// 32-bit keys: clog[cb] = m proportional sub-bins, sub = (offset * m) >> cs (monotone,
+// < m), which sizes the bins to the coarse counts without power-of-two rounding.
+template <class KT>
 MP_INLINE uint32_t r3_fine(const R3Smem& S, const R3Geo& g, uint32_t cb, uint64_t key) {
     const uint32_t l = S.clog[cb];
+    if constexpr (sizeof(KT) == 4) {
+        const uint64_t off = key - ((g.clb + cb) << g.cs);
+        return (uint32_t)S.coff[cb] + (uint32_t)((off * l) >> g.cs);
+    }
     const uint32_t sub = l ? (uint32_t)((key >> (g.cs - l)) & ((1ull << l) - 1ull)) : 0u;
     return (uint32_t)S.coff[cb] + sub;
 }
@@ -518,7 +527,7 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
         const KT k = bk[j];
         const uint16_t v = bv[j];
         const uint64_t k64 = sizeof(KT) == 8 ? (uint64_t)k : ((uint64_t)k << 32);
-        const uint32_t f = r3_fine(S, g, (uint32_t)((k64 >> g.cs) - g.clb), k64);
+        const uint32_t f = r3_fine<KT>(S, g, (uint32_t)((k64 >> g.cs) - g.clb), k64);
         const uint32_t s0 = (f == b0 ? base : S.starts[f - 1]) - base;
         const uint32_t s1 = S.starts[f] - base;
         uint32_t rank = 0;
@@ -616,7 +625,36 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         for (int j = 0; j < CPER; j++) cc[j] = S.starts[threadIdx.x * CPER + j];
         uint32_t T = 4;
         uint32_t lg[CPER], ftot = 0, fex = 0;
-        while (true) {
+        if constexpr (sizeof(KT) == 4) {
+            // proportional: m_c = ceil(c * (NF - nonempty) / in_range) sums to <= NF
+            uint32_t ne = 0, tc = 0, NE = 0, TOT = 0;
+#pragma unroll
+            for (int j = 0; j < CPER; j++) {
+                const uint32_t b = threadIdx.x * CPER + j;
+                if (b < g.ncb) {
+                    ne += cc[j] > 0 ? 1u : 0u;
+                    tc += cc[j];
+                }
+            }
+            r3_scan(ne, S.sc, NE);
+            r3_scan(tc, S.sc, TOT);
+            const uint64_t Fn = (uint64_t)R3_NF - NE, Fd = TOT > 0 ? TOT : 1u;
+            uint32_t sm = 0;
+#pragma unroll
+            for (int j = 0; j < CPER; j++) {
+                const uint32_t b = threadIdx.x * CPER + j;
+                uint32_t m = 0;
+                if (b < g.ncb && cc[j] > 0) {
+                    m = (uint32_t)min(((uint64_t)cc[j] * Fn + Fd - 1) / Fd, (uint64_t)255);
+                    if (g.cs < 8) m = min(m, 1u << g.cs);
+                    m = max(m, 1u);
+                }
+                lg[j] = m;
+                sm += m;
+            }
+            fex = r3_scan(sm, S.sc, ftot);
+        }
+        while (sizeof(KT) == 8) {
             uint32_t s = 0;
 #pragma unroll
             for (int j = 0; j < CPER; j++) {
@@ -637,7 +675,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
                 const uint32_t b = threadIdx.x * CPER + j;
                 S.coff[b] = (uint16_t)e;
                 S.clog[b] = (uint8_t)lg[j];
-                if (b < g.ncb) e += 1u << lg[j];
+                if (b < g.ncb) e += sizeof(KT) == 4 ? lg[j] : 1u << lg[j];
             }
         }
         __syncthreads();
@@ -651,7 +689,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         __syncthreads();
         uint32_t need = 0;
         for (int w = 0; w < R2_WARPS; w++) need = max(need, S.sc[40 + w]);
-        need = g.cs - need;   // fine bins use key bits >= need
+        need = sizeof(KT) == 4 ? 0u : g.cs - need;   // fine bins use key bits >= need
         const uint32_t nfb = ftot;
         K2_PHASE(3);
         // ---- pass 2: fine histogram ----
@@ -673,7 +711,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
                 uint32_t cb;
                 uint64_t key;
                 if (r3_locate_hk(K, c0 + u, hv[u], g, need, cb, key)) {
-                    fv[u] = r3_fine(S, g, cb, key);
+                    fv[u] = r3_fine<KT>(S, g, cb, key);
                     atomicAdd(&S.starts[fv[u]], 1u);
                 }
             }
@@ -754,12 +792,22 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
                         else hi_c = mid - 1;
                     }
                     const uint32_t l = S.clog[lo_c];
-                    const uint32_t fs = g.cs - l;
-                    uint64_t blo = ((g.clb + lo_c) << g.cs) + ((uint64_t)(b0 - S.coff[lo_c]) << fs);
-                    uint64_t bhi = blo + ((1ull << fs) - 1ull);
+                    uint64_t blo, bhi;
+                    bool one = false;
+                    if constexpr (sizeof(KT) == 4) {
+                        // sub-bin s holds offsets [ceil(s W / m), ceil((s+1) W / m) - 1], W = 2^cs
+                        const uint64_t cbase = (g.clb + lo_c) << g.cs, W = 1ull << g.cs, sb = b0 - S.coff[lo_c];
+                        blo = cbase + (sb * W + l - 1) / l;
+                        bhi = cbase + ((sb + 1) * W + l - 1) / l - 1;
+                    } else {
+                        const uint32_t fs = g.cs - l;
+                        blo = ((g.clb + lo_c) << g.cs) + ((uint64_t)(b0 - S.coff[lo_c]) << fs);
+                        bhi = blo + ((1ull << fs) - 1ull);
+                        one = fs == 0;
+                    }
                     if (blo < g.lo) blo = g.lo;
                     if (bhi > g.hi || bhi < blo) bhi = g.hi;
-                    if (fs == 0) bhi = blo;
+                    if (one) bhi = blo;
                     push(blo, bhi, (uint32_t)(ob + (int32_t)e0), cnt);
                 }
                 __syncthreads();
