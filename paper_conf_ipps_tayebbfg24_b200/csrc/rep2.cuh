@@ -1435,7 +1435,8 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     using namespace mpk;
     const int32_t n = dag->n;
     const int64_t groups = (R + 31) / 32;
-    const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
+    static const int grid_env = [] { const char* e = getenv("MP_K2_GRID"); return e ? atoi(e) : 0; }();   // experiments
+    const int grid2 = std::max(1, std::min<int>(R, grid_env > 0 ? grid_env : dag->num_sms));
     const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
                    align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 8) +
