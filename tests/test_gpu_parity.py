@@ -298,6 +298,15 @@ def test_replicas_ties_stream_path():
     _replica_check(w, 40, 0, [0, 39], sigma=0.0)
 
 
+@pytest.mark.parametrize("sigma", [2.0 ** -10, 2.0 ** -16, 2.0 ** -21])
+def test_replicas_tiny_sigma_clustered_keys(sigma):
+    """Small perturbations cluster the duration differences within a few ulps: many equal
+    d values and equal-gain runs (some longer than 64 -> general path), 32-bit key bins of
+    more than 256 entries (finer sub-ranges), single-valued bins (streamed)."""
+    w = workloads.config("c2")
+    _replica_check(w, 40, 3, [0, 1, 20, 39], sigma=sigma)
+
+
 def test_replicas_two_arch_mixed_one_arch_tasks():
     """Two archs with CPU-only tasks (sparse-QR ASM, FMM P2M/M2M/L2L/L2P): d = +-inf classes."""
     a = workloads.sparse_tree(12, 64, 32)
