@@ -411,8 +411,9 @@ def run_ours(args):
         tasks_per_step = n
         result_h = torch.empty(A * mp.SUMMARY_BYTES + 4, dtype=torch.uint8).pin_memory()
 
-        def step():
-            mp.dag_rebuild(dag, n, src_d, dst_d)
+        def step(rebuild=True):
+            if rebuild:
+                mp.dag_rebuild(dag, n, src_d, dst_d)
             bl, cp, _ = mp.bottom_level(dag, dur_d, w.workers, out=outs.setdefault("bl", dict(
                 bl=torch.empty(n, dtype=torch.float32, device=dev), cp=torch.empty(1, dtype=torch.float32, device=dev),
                 nod=None)))
@@ -471,6 +472,25 @@ def run_ours(args):
     ms_per_step = float(tot.item()) / args.steps
     value = tasks_per_step / (ms_per_step * 1e-3)
     prof = {k: mp.prof_query(k) for k in mp.prof_names()}
+
+    # ---- single DAGs: the score + queue path alone on the prebuilt DAG (t covers
+    #      bottom_level -> affinity -> score -> build_queues; the ingest is reported separately) ----
+    score_only = None
+    if cfg in ("c1", "c2", "c3", "c4", "lu64"):
+        sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        torch.cuda.synchronize()
+        for i in range(args.steps):
+            flush.zero_()
+            sev[i][0].record(stream)
+            step(rebuild=False)
+            sev[i][1].record(stream)
+        torch.cuda.synchronize()
+        sc_ms = sum(a.elapsed_time(b) for a, b in sev) / args.steps
+        Q = int(np.isfinite(w.dur).sum())      # queue entries (every arch enabled by the workers)
+        b_sc = 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 4 * n * A + 4 * Q
+        score_only = {"ms_per_dag": sc_ms, "tasks_per_s": n / (sc_ms * 1e-3), "build_ms": ms_per_step - sc_ms,
+                      "alg_bytes": b_sc, "hbm_frac_of_peak": None,
+                      "note": "bottom_level + affinity + score + build_queues on the prebuilt DAG, L2 flushed"}
     step_dev_ms = {k: v[0] / args.steps for k, v in prof.items() if v[1] > 0}
     dom = max(step_dev_ms, key=step_dev_ms.get)
     dom_ms, dom_launches = prof[dom]
@@ -537,6 +557,8 @@ def run_ours(args):
         b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 4 * n * A + 4 * n * A
     roof["step_alg_bytes_per_gpu"] = b_alg
     roof["step_hbm_frac"] = b_alg / (ms_per_step * 1e-3) / 1e9 / peak
+    if score_only is not None:
+        score_only["hbm_frac_of_peak"] = score_only["alg_bytes"] / (score_only["ms_per_dag"] * 1e-3) / 1e9 / peak
 
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
@@ -578,7 +600,8 @@ def run_ours(args):
                        **({"locality": {"top_n": LOC["top_n"], "eps": LOC["eps"],
                                         "xfer_ms_per_byte": LOC["xfer_ms_per_byte"]}} if cfg == "c5loc" else {})},
             "ms_per_dag": ms_per_step / (R / world) if rep else ms_per_step,
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
+            "roofline": roof, **({"score_only": score_only} if score_only else {}),
+            "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
             "gpu_launches_per_step": launches / args.steps, "clocks": ck,
             "device": torch.cuda.get_device_name(dev)}
     print(json.dumps(line), flush=True)
