@@ -138,6 +138,14 @@ MP_INLINE uint64_t splitmix64(uint64_t seed, uint64_t c) {
     return x ^ (x >> 31);
 }
 
+// the same with u = k * 2^-24 given (k < 2^24): the perturbation at a chosen draw
+MP_INLINE float perturb_u(float d, float sigma, uint32_t k) {
+    float u = __fmul_rn((float)k, 0x1p-24f);
+    float s = __fsub_rn(__fmul_rn(2.0f, u), 1.0f);
+    float f = __fadd_rn(1.0f, __fmul_rn(sigma, s));
+    return __fmul_rn(d, f);
+}
+
 // delta_r(t,a) = delta * (1 + sigma*(2u-1)); explicit RN ops, no contraction
 MP_INLINE float perturb(float d, uint64_t seed, float sigma, uint64_t counter) {
     float u = __fmul_rn((float)(uint32_t)(splitmix64(seed, counter) >> 40), 0x1p-24f);

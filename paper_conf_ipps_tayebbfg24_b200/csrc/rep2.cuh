@@ -67,6 +67,7 @@ struct Rep2Args {
     uint32_t* s_key;             // [grid][2][npad] per-CTA hot scratch: D in id order, D in sorted order
     uint16_t* s_pi;              // [grid][2][npad] per-CTA hot scratch: fine-bin ids, sorted positions
     uint32_t* s_cold;            // [grid][A+1][npad] general path only: critc, gainc per arch
+    unsigned char* s_geo;        // [grid][R3_GEO_BYTES] two-arch path: cached sub-bin geometry
     int32_t* qtask;              // [R][n*A] or null
     mp_queue_summary* sum;       // [R][A]
     uint32_t* ticket;
@@ -545,8 +546,34 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
 
 MP_INLINE uint32_t r3_clog2(uint32_t x) { return x <= 1 ? 0u : 32u - __clz(x - 1); }   // ceil(log2 x)
 
+constexpr int R3_GEO_BYTES = 16384;   // coff (2 B) + clog (1 B) per coarse bin + fine-bin count
+
+// coarse geometry of a key range: <= R3_NC bins of width 2^cs
+MP_INLINE R3Geo r3_geo(uint64_t lo, uint64_t hi) {
+    R3Geo g;
+    g.lo = lo;
+    g.hi = hi;
+    const uint64_t span = hi - lo;
+    const uint32_t bits = 64u - (uint32_t)__clzll((long long)span);
+    constexpr uint32_t LOGNC = 31u - __builtin_clz((unsigned)R3_NC);   // NC is a power of two
+    g.cs = bits > LOGNC ? bits - LOGNC : 0;
+    g.clb = lo >> g.cs;
+    g.ncb = (uint32_t)((hi >> g.cs) - g.clb + 1);
+    while (g.ncb > (uint32_t)R3_NC) {
+        g.cs++;
+        g.clb = lo >> g.cs;
+        g.ncb = (uint32_t)((hi >> g.cs) - g.clb + 1);
+    }
+    return g;
+}
+
+// pre_nfb != 0: the top range [kmin, kmax] is pre-binned by the caller -- coff/clog hold its
+// sub-bin geometry (pre_nfb fine bins), starts[] its fine counts and K.fb every entry's fine
+// bin -- so passes 1-2 are skipped for it.  snap != null: the top range's sub-bin geometry is
+// saved there (coff, clog, fine-bin count) for a later pre-binned call on the same range.
 template <class KT, class Out>
-__device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmin, uint64_t kmax, R3Smem& S) {
+__device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmin, uint64_t kmax, R3Smem& S,
+                        uint32_t pre_nfb = 0, unsigned char* snap = nullptr) {
     constexpr int CAPK = r3_cap<KT>();
     if (n <= 0) return;
     uint32_t* stk = S.misc;                        // [R3_MAXS][6]
@@ -568,6 +595,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         push(kmin, kmax, 0, (uint32_t)n);
     }
     __syncthreads();
+    bool first = true;
     while (true) {
         const uint32_t ns = *nstk;
         if (ns == 0) break;
@@ -584,17 +612,12 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
             __syncthreads();
             continue;
         }
-        const uint64_t span = g.hi - g.lo;
-        const uint32_t bits = 64u - (uint32_t)__clzll((long long)span);
-        constexpr uint32_t LOGNC = 31u - __builtin_clz((unsigned)R3_NC);   // NC is a power of two
-        g.cs = bits > LOGNC ? bits - LOGNC : 0;
-        g.clb = g.lo >> g.cs;
-        g.ncb = (uint32_t)((g.hi >> g.cs) - g.clb + 1);
-        while (g.ncb > (uint32_t)R3_NC) {
-            g.cs++;
-            g.clb = g.lo >> g.cs;
-            g.ncb = (uint32_t)((g.hi >> g.cs) - g.clb + 1);
-        }
+        g = r3_geo(g.lo, g.hi);
+        const bool toprange = first;   // the caller's range (not a deferred sub-range)
+        const bool prebinned = toprange && pre_nfb != 0;
+        first = false;
+        uint32_t ftot = pre_nfb;
+        if (!prebinned) {
         // ---- pass 1: coarse histogram (in starts[0..NC)) ----
         for (uint32_t b = threadIdx.x; b < (uint32_t)R3_NF + 64; b += R2_THREADS) S.starts[b] = 0;
         __syncthreads();
@@ -624,15 +647,19 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
 #pragma unroll
         for (int j = 0; j < CPER; j++) cc[j] = S.starts[threadIdx.x * CPER + j];
         uint32_t T = 4;
-        uint32_t lg[CPER], ftot = 0, fex = 0;
+        uint32_t lg[CPER], fex = 0;
+        ftot = 0;
         if constexpr (sizeof(KT) == 4) {
-            // proportional: m_c = ceil(c * (NF - nonempty) / in_range) sums to <= NF
+            // proportional: m_c = ceil(c * (NF - nonempty) / in_range) sums to <= NF.  A geometry
+            // cached for other replicas (snap) gives every coarse bin >= 1 sub-bin: their keys
+            // may fall where this replica has none
+            const bool all1 = toprange && snap;
             uint32_t ne = 0, tc = 0, NE = 0, TOT = 0;
 #pragma unroll
             for (int j = 0; j < CPER; j++) {
                 const uint32_t b = threadIdx.x * CPER + j;
                 if (b < g.ncb) {
-                    ne += cc[j] > 0 ? 1u : 0u;
+                    ne += (cc[j] > 0 || all1) ? 1u : 0u;
                     tc += cc[j];
                 }
             }
@@ -644,7 +671,7 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
             for (int j = 0; j < CPER; j++) {
                 const uint32_t b = threadIdx.x * CPER + j;
                 uint32_t m = 0;
-                if (b < g.ncb && cc[j] > 0) {
+                if (b < g.ncb && (cc[j] > 0 || all1)) {
                     m = (uint32_t)min(((uint64_t)cc[j] * Fn + Fd - 1) / Fd, (uint64_t)255);
                     if (g.cs < 8) m = min(m, 1u << g.cs);
                     m = max(m, 1u);
@@ -679,6 +706,14 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
             }
         }
         __syncthreads();
+        if (toprange && snap) {   // sub-bin geometry of the top range, for later pre-binned calls
+            uint16_t* sc16 = reinterpret_cast<uint16_t*>(snap);
+            for (uint32_t b = threadIdx.x; b < (uint32_t)R3_NC; b += R2_THREADS) {
+                sc16[b] = S.coff[b];
+                snap[2 * R3_NC + b] = S.clog[b];
+            }
+            if (threadIdx.x == 0) *reinterpret_cast<uint32_t*>(snap + 3 * R3_NC) = ftot;
+        }
         // lowest key bit any fine bin depends on
         uint32_t maxl = 0;
 #pragma unroll
@@ -690,7 +725,6 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         uint32_t need = 0;
         for (int w = 0; w < R2_WARPS; w++) need = max(need, S.sc[40 + w]);
         need = sizeof(KT) == 4 ? 0u : g.cs - need;   // fine bins use key bits >= need
-        const uint32_t nfb = ftot;
         K2_PHASE(3);
         // ---- pass 2: fine histogram ----
         for (int32_t c0 = threadIdx.x * 8; c0 < n; c0 += 8 * R2_THREADS) {
@@ -728,6 +762,8 @@ __device__ void r3_sort(const R3Keys& K, const Out& out, int32_t n, uint64_t kmi
         }
         __syncthreads();
         K2_PHASE(4);
+        }
+        const uint32_t nfb = ftot;
         // ---- prefixes over fine bins (12 per thread) + group boundaries ----
         constexpr int PER = R3_NF / R2_THREADS;  // 12
         const uint32_t H = CAPK - R3_MID;        // a multi-bin group never exceeds H + MID = CAP
@@ -901,6 +937,57 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     uint16_t* ppos = fbuf + npad;
     uint32_t* dsorted = dkey + npad;   // (A == 2) D in sorted order (gains are recomputed from it)
     bool bad = false;
+    // Two archs: a key range that holds every replica's D, from the perturbation's extremes
+    // (u = 0 and u = 1 - 2^-24; every RN op on the way is monotone, so each perturbed
+    // duration, and then d = delta_1 - delta_0, lies between the values at the extremes).
+    // With one fixed range every replica has the same coarse bins, and the sub-bin geometry
+    // built for this CTA's first replica is reused: later replicas bin their keys while
+    // hashing (P0) and skip the sorter's two histogram passes.
+    __shared__ uint32_t s_flo, s_fhi, s_geo_ok, s_geo_nfb, s_out;
+    unsigned char* geo = a.s_geo ? a.s_geo + (int64_t)blockIdx.x * R3_GEO_BYTES : nullptr;
+    if constexpr (A == 2) {
+        if (threadIdx.x == 0) { s_flo = ~0u; s_fhi = 0u; s_geo_ok = 0u; s_geo_nfb = 0u; }
+        __syncthreads();
+        uint32_t lo = ~0u, hi = 0u;
+        for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
+            float xl[2], xh[2];
+            uint32_t enl = 0, enh = 0;
+            bool dummy = false;
+#pragma unroll
+            for (int b = 0; b < 2; b++) {
+                const float bv = __ldg(a.base + 2 * (int64_t)t + b);
+                const float e0 = canon_dur(perturb_u(bv, a.sigma, 0u), dummy);
+                const float e1 = canon_dur(perturb_u(bv, a.sigma, 0xFFFFFFu), dummy);
+                xl[b] = e0 < e1 ? e0 : e1;
+                xh[b] = e0 < e1 ? e1 : e0;
+                if (((a.emask >> b) & 1u) && !is_inf(xl[b])) enl |= 1u << b;
+                if (((a.emask >> b) & 1u) && !is_inf(xh[b])) enh |= 1u << b;
+            }
+            if (enl != enh || xl[0] != xl[0] || xl[1] != xl[1] || xh[0] != xh[0] || xh[1] != xh[1]) {
+                lo = 0u;            // cannot bound this task: the whole key space
+                hi = 0xFFFFFFFFu;
+            } else if (enl == 3u) {
+                const uint32_t dl = f2u(__fsub_rn(xl[1], xh[0])), dh = f2u(__fsub_rn(xh[1], xl[0]));
+                lo = min(lo, (dl >> 31) ? ~dl : (dl | 0x80000000u));
+                hi = max(hi, (dh >> 31) ? ~dh : (dh | 0x80000000u));
+            } else if (enl != 0u) {
+                const uint32_t D = enl == 1u ? 0xFFFFFFFFu : 0u;
+                lo = min(lo, D);
+                hi = max(hi, D);
+            }
+        }
+        lo = __reduce_min_sync(0xffffffffu, lo);
+        hi = __reduce_max_sync(0xffffffffu, hi);
+        if ((threadIdx.x & 31) == 0) {
+            atomicMin(&s_flo, lo);
+            atomicMax(&s_fhi, hi);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0 && s_flo > s_fhi) { s_flo = 0u; s_fhi = 0xFFFFFFFFu; }
+        __syncthreads();
+    }
+    const uint64_t kfl = (uint64_t)s_flo << 32, kfh = (uint64_t)s_fhi << 32;
+    const R3Geo gf = r3_geo(kfl, kfh > kfl ? kfh : kfl + (1ull << 32));
     while (true) {
         if (threadIdx.x == 0) s_tick = atomicAdd(a.ticket, 1u);
         if (threadIdx.x <= A) {
@@ -922,11 +1009,23 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         unsigned long long mn[A + 1], mx[A + 1];
 #pragma unroll
         for (int b = 0; b <= A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
+        const bool pre = A == 2 && geo && s_geo_ok;
+        if (pre) {   // restore the cached sub-bin geometry, zero the fine counters
+            const uint16_t* g16 = reinterpret_cast<const uint16_t*>(geo);
+            for (int32_t b = threadIdx.x; b < R3_NC; b += R2_THREADS) {
+                S.coff[b] = __ldcg(g16 + b);
+                S.clog[b] = __ldcg(geo + 2 * R3_NC + b);
+            }
+            for (int32_t b = threadIdx.x; b < R3_NF + 64; b += R2_THREADS) S.starts[b] = 0u;
+            if (threadIdx.x == 0) s_out = 0u;
+            __syncthreads();
+        }
         if constexpr (A == 2) {
             // two archs: only the orderable d is needed to sort (crit is read for equal-gain runs).
             // 4 tasks per thread and trip (t, t+1 | t+2048, t+2049): both 16-byte base loads
             // are issued before the hashing
             uint32_t dmn = ~0u, dmx = 0u;
+            bool outside = false;
             auto one = [&](int32_t t, float b0v, float b1v) {
                 const float bb[2] = {b0v, b1v};
                 const uint64_t c0 = ((uint64_t)r * (uint64_t)a.n + (uint64_t)t) * 2u + 1u;
@@ -948,6 +1047,17 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 dkey[t] = D;
                 dmn = min(dmn, D);
                 dmx = max(dmx, D);
+                if (pre) {   // fine bin of the cached geometry (pass 2 of the sorter, fused)
+                    const uint64_t key = (uint64_t)D << 32;
+                    uint32_t f = 0xFFFFu;
+                    if (key < gf.lo || key > gf.hi) {
+                        outside = true;
+                    } else {
+                        f = r3_fine<uint32_t>(S, gf, (uint32_t)((key >> gf.cs) - gf.clb), key);
+                        atomicAdd(&S.starts[f], 1u);
+                    }
+                    fbuf[t] = (uint16_t)f;
+                }
             };
             const bool al = (reinterpret_cast<uintptr_t>(a.base) & 15u) == 0;
             const int32_t n2 = al ? (a.n & ~1) : 0;
@@ -967,6 +1077,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 one(t, __ldg(a.base + 2 * (int64_t)t), __ldg(a.base + 2 * (int64_t)t + 1));
             mn[A] = (unsigned long long)dmn << 32;
             mx[A] = (unsigned long long)dmx << 32;
+            if (__any_sync(0xffffffffu, outside) && (threadIdx.x & 31) == 0) s_out = 1u;
         }
         const bool vec4 = (a.n & 3) == 0;   // 16-byte loads of bl when rows stay aligned
         for (int32_t t0 = vec4 ? threadIdx.x * 4 : threadIdx.x; A != 2 && t0 < a.n; t0 += vec4 ? 4 * R2_THREADS : R2_THREADS) {
@@ -1049,7 +1160,25 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         if constexpr (A == 2) {
             // one sort by (D, critc, t) -> P; then both queues in one pass (runs of equal gain fixed up)
             K2_PHASE(1);
-            r3_sort<uint32_t>(R3Keys{dkey, nullptr, fbuf}, R3PosOut{ppos, dsorted}, a.n, s_min[A] & ~0xFFFFFFFFull, s_max[A] & ~0xFFFFFFFFull, S);
+            {
+                const uint64_t amin = s_min[A] & ~0xFFFFFFFFull, amax = s_max[A] & ~0xFFFFFFFFull;
+                const R3Keys K{dkey, nullptr, fbuf};
+                const R3PosOut O{ppos, dsorted};
+                if (pre && !s_out) {
+                    r3_sort<uint32_t>(K, O, a.n, gf.lo, gf.hi, S, s_geo_nfb);
+                } else if (geo && !pre && amin >= gf.lo && amax <= gf.hi && gf.lo < gf.hi) {
+                    // first replica on the fixed range: build and cache its geometry
+                    if (threadIdx.x == 0) *reinterpret_cast<uint32_t*>(geo + 3 * R3_NC) = 0u;
+                    __syncthreads();
+                    r3_sort<uint32_t>(K, O, a.n, gf.lo, gf.hi, S, 0u, geo);
+                    if (threadIdx.x == 0) {
+                        s_geo_nfb = *reinterpret_cast<volatile uint32_t*>(geo + 3 * R3_NC);
+                        s_geo_ok = s_geo_nfb != 0u;
+                    }
+                } else {
+                    r3_sort<uint32_t>(K, O, a.n, amin, amax, S);
+                }
+            }
             K2_PHASE(7);
             if (threadIdx.x == 0) { s_flag = 0; s_h0 = 0xffffffffu; s_h1 = 0xffffffffu; }
             __syncthreads();
@@ -1440,7 +1569,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
                    align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 8) +
-                   align256((size_t)grid2 * ((n + 15) & ~15) * 4);
+                   align256((size_t)grid2 * ((n + 15) & ~15) * 4) + align256((size_t)grid2 * R3_GEO_BYTES);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
     Rep2Args a{};
@@ -1469,6 +1598,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.s_cold = ar.take<uint32_t>((size_t)grid2 * npad * (A + 1));
     a.s_key = ar.take<uint32_t>((size_t)grid2 * npad * 2);   // hot scratch: s_key and s_pi adjacent
     a.s_pi = ar.take<uint16_t>((size_t)grid2 * npad * 2);
+    a.s_geo = A == 2 ? ar.take<unsigned char>((size_t)grid2 * R3_GEO_BYTES) : nullptr;
     a.qtask = qtask;
     a.sum = sum;
     a.ticket = dag->tickets + 56;
