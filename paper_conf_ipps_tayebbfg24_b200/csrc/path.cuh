@@ -83,8 +83,15 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
 // in shared memory.
 constexpr int FLOW_THREADS = 256;
 constexpr uint32_t NOT_READY = 0xFFFFFFFFu;
+#ifndef MP_FLOW_PF
+#define MP_FLOW_PF 2
+#endif
+#ifndef MP_FLOW_MINB
+#define MP_FLOW_MINB 8
+#endif
+constexpr int FLOW_PF = MP_FLOW_PF;   // edges per lane whose loads k_bl_flow issues together
 
-__global__ void __launch_bounds__(FLOW_THREADS) k_bl_flow(int32_t nchunks, const int32_t* __restrict__ nodep,
+__global__ void __launch_bounds__(FLOW_THREADS, MP_FLOW_MINB) k_bl_flow(int32_t nchunks, const int32_t* __restrict__ nodep,
                                                           const int32_t* __restrict__ rowp,
                                                           const int32_t* __restrict__ colp, DurView d,
                                                           uint32_t* blp, float* bl, float* cp, uint32_t* ticket,
@@ -108,20 +115,51 @@ __global__ void __launch_bounds__(FLOW_THREADS) k_bl_flow(int32_t nchunks, const
         const float wt = v >= 0 ? task_weight(d, v, bad) : 0.0f;
         __syncwarp();
         const int32_t E0 = srow[w][0], E1 = srow[w][32];
-        for (int32_t e = E0 + lane; e < E1; e += 32) {
-            const int32_t sp = __ldg(colp + e);
-            uint32_t x;
-            do {
-                x = ld_relaxed(blp + sp);
-            } while (x == NOT_READY);
-            // owner: largest i with srow[i] <= e
+        // owner of edge e: largest i with srow[i] <= e
+        auto owner = [&](int32_t e) -> int {
             int lo = 0, hi = 31;
             while (lo < hi) {
-                int mid = (lo + hi + 1) >> 1;
+                const int mid = (lo + hi + 1) >> 1;
                 if (srow[w][mid] <= e) lo = mid;
                 else hi = mid - 1;
             }
-            atomicMax(&smax[w][lo], x);
+            return lo;
+        };
+        // the chunk's edges in batches of FLOW_PF per lane: all successor positions of a batch,
+        // then all their bl words, are loaded together and only the words not yet published
+        // are polled again -- a chunk with many edges (a TRSM feeding a whole GEMM row) costs
+        // a few round trips per batch instead of two dependent round trips per edge
+        int32_t sp[FLOW_PF];
+#pragma unroll
+        for (int k = 0; k < FLOW_PF; k++) {
+            const int32_t e = E0 + lane + 32 * k;
+            sp[k] = e < E1 ? __ldg(colp + e) : -1;
+        }
+        for (int32_t eb = E0; eb < E1; eb += 32 * FLOW_PF) {
+            uint32_t xs[FLOW_PF];
+            int32_t spn[FLOW_PF];
+#pragma unroll
+            for (int k = 0; k < FLOW_PF; k++) xs[k] = sp[k] >= 0 ? ld_relaxed(blp + sp[k]) : 0u;
+#pragma unroll
+            for (int k = 0; k < FLOW_PF; k++) {   // next batch's successor positions, in flight meanwhile
+                const int32_t e = eb + 32 * FLOW_PF + lane + 32 * k;
+                spn[k] = e < E1 ? __ldg(colp + e) : -1;
+            }
+            while (true) {
+                bool waiting = false;
+#pragma unroll
+                for (int k = 0; k < FLOW_PF; k++)
+                    if (xs[k] == NOT_READY) {
+                        xs[k] = ld_relaxed(blp + sp[k]);
+                        waiting |= xs[k] == NOT_READY;
+                    }
+                if (!waiting) break;
+            }
+#pragma unroll
+            for (int k = 0; k < FLOW_PF; k++) {
+                if (sp[k] >= 0) atomicMax(&smax[w][owner(eb + lane + 32 * k)], xs[k]);
+                sp[k] = spn[k];
+            }
         }
         __syncwarp();
         if (v >= 0) {
