@@ -1208,8 +1208,16 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             {
                 K2_PHASE(8);
                 // 4 consecutive positions per lane (one 16-byte load), 128 per warp and chunk,
-                // two chunks in flight; nibbles of 8 lanes OR-ed into one bit word
+                // two chunks in flight; nibbles of 8 lanes OR-ed into one bit word.  Near-ties
+                // (different numerators less than lim apart, ~2% of the pairs) need the two
+                // divisions; they are listed (position | arch << 31, in the free bin counters)
+                // and divided in a compact pass, so no warp runs the division code inline
+                uint32_t* nearl = S.starts + 1;
+                const uint32_t ncap = (uint32_t)R3_NF + 63u;
+                if (threadIdx.x == 0) S.starts[0] = 0u;
+                __syncthreads();
                 const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+                const bool one_arch = cC != a.n || cG != a.n;   // some D are the one-arch sentinels
                 constexpr int32_t CH = 128, STEP = CH * R2_WARPS;
                 for (int32_t cb0 = w * CH; cb0 < a.n; cb0 += 2 * STEP) {
                     uint32_t Dv[2][4], nx[2];
@@ -1239,7 +1247,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
 #pragma unroll
                         for (int j = 0; j < 5; j++) {
                             const uint32_t D = Dj[j];
-                            gen |= (D == 0u || D == 0xFFFFFFFFu) && (j < 4 ? p4 + j < a.n : p4 + 4 < a.n);
+                            if (one_arch) gen |= (D == 0u || D == 0xFFFFFFFFu) && (j < 4 ? p4 + j < a.n : p4 + 4 < a.n);
                             const float d = u2f((D & 0x80000000u) ? (D & 0x7FFFFFFFu) : ~D);
                             xs[j] = __fadd_rn(d, h2);
                             ys[j] = __fadd_rn(__fsub_rn(0.0f, d), h2);
@@ -1254,8 +1262,24 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                                 if (gen) {
                                     r2_same_gains(Dj[j], Dj[j + 1], h2, s0, s1);
                                 } else {
-                                    s0 = r2_same_q(xs[j], xs[j + 1], den, lim);
-                                    s1 = r2_same_q(ys[j], ys[j + 1], den, lim);
+                                    // sorted ascending: x non-decreasing, y non-increasing
+                                    const float dx = __fsub_rn(xs[j + 1], xs[j]), dy = __fsub_rn(ys[j], ys[j + 1]);
+                                    s0 = dx == 0.0f;
+                                    s1 = dy == 0.0f;
+                                    const bool c0 = !s0 && dx <= lim;
+                                    const bool c1 = !s1 && dy <= lim;
+                                    if (c0 || c1) {
+                                        const uint32_t cnt = (c0 ? 1u : 0u) + (c1 ? 1u : 0u);
+                                        const uint32_t at = atomicAdd(&S.starts[0], cnt);
+                                        const uint32_t pj = (uint32_t)(p4 + j);
+                                        if (at + cnt <= ncap) {
+                                            if (c0) nearl[at] = pj;
+                                            if (c1) nearl[at + (c0 ? 1u : 0u)] = pj | 0x80000000u;
+                                        } else {   // list full (not expected): divide here
+                                            if (c0) s0 = r2_same_q(xs[j], xs[j + 1], den, lim);
+                                            if (c1) s1 = r2_same_q(ys[j], ys[j + 1], den, lim);
+                                        }
+                                    }
                                 }
                                 n0 |= (uint32_t)s0 << j;
                                 n1 |= (uint32_t)s1 << j;
@@ -1273,6 +1297,19 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                             e1[(cb >> 5) + (lane >> 3)] = n1;
                         }
                     }
+                }
+                __syncthreads();
+                const uint32_t nn = min(S.starts[0], ncap);
+                const float den = __fadd_rn(h2, h2);
+                for (uint32_t i = threadIdx.x; i < nn; i += R2_THREADS) {
+                    const uint32_t ent = nearl[i];
+                    const int32_t p = (int32_t)(ent & 0x7FFFFFFFu);
+                    const uint32_t Da = __ldcg(dsorted + p), Db = __ldcg(dsorted + p + 1);   // no sentinels here
+                    const float da = u2f((Da & 0x80000000u) ? (Da & 0x7FFFFFFFu) : ~Da);
+                    const float db = u2f((Db & 0x80000000u) ? (Db & 0x7FFFFFFFu) : ~Db);
+                    const float d0 = (ent >> 31) ? __fsub_rn(0.0f, da) : da, d1 = (ent >> 31) ? __fsub_rn(0.0f, db) : db;
+                    const float xa = __fadd_rn(d0, h2), xb = __fadd_rn(d1, h2);
+                    if (__fdiv_rn(xa, den) == __fdiv_rn(xb, den)) atomicOr((ent >> 31) ? &e1[p >> 5] : &e0[p >> 5], 1u << (p & 31));
                 }
             }
             __syncthreads();

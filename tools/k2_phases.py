@@ -7,7 +7,8 @@ import ctypes as C, os, subprocess, sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 from paper_conf_ipps_tayebbfg24_b200 import build as B
-subprocess.check_call([B.NVCC, *B.FLAGS, "-DMP_PHASES", "-o", B.LIB, os.path.join(B.CSRC, "libmp.cu")])
+subprocess.check_call([B.NVCC, *B.FLAGS, "-DMP_PHASES", *os.environ.get("K2_DEFS", "").split(), "-o", B.LIB,
+                       os.path.join(B.CSRC, "libmp.cu")])
 import numpy as np, torch
 import paper_conf_ipps_tayebbfg24_b200 as mp, workloads
 from paper_conf_ipps_tayebbfg24_b200 import _lib
