@@ -443,6 +443,11 @@ template <class KT>
 MP_INLINE uint32_t r3_fine(const R3Smem& S, const R3Geo& g, uint32_t cb, uint64_t key) {
     const uint32_t l = S.clog[cb];
     if constexpr (sizeof(KT) == 4) {
+        if (g.cs >= 32) {   // the key is k << 32: all in 32 bits (offset < 2^(cs-32) <= 2^21, m < 2^8)
+            const uint32_t c32 = g.cs - 32u;
+            const uint32_t off = (uint32_t)(key >> 32) - (((uint32_t)g.clb + cb) << c32);
+            return (uint32_t)S.coff[cb] + ((off * l) >> c32);
+        }
         const uint64_t off = key - ((g.clb + cb) << g.cs);
         return (uint32_t)S.coff[cb] + (uint32_t)((off * l) >> g.cs);
     }
