@@ -455,6 +455,19 @@ MP_INLINE uint32_t r3_fine(const R3Smem& S, const R3Geo& g, uint32_t cb, uint64_
     return (uint32_t)S.coff[cb] + sub;
 }
 
+// fine bin of a 32-bit key k (64-bit key k << 32) in range geometry g, coarse bin included
+MP_INLINE uint32_t r3_bin32(const R3Smem& S, const R3Geo& g, uint32_t k) {
+    if (g.cs >= 32) {
+        const uint32_t c32 = g.cs - 32u;
+        const uint32_t cb = (k >> c32) - (uint32_t)g.clb;
+        const uint32_t off = k - ((k >> c32) << c32);
+        return (uint32_t)S.coff[cb] + ((off * (uint32_t)S.clog[cb]) >> c32);
+    }
+    const uint64_t key = (uint64_t)k << 32;
+    return r3_fine<uint32_t>(S, g, (uint32_t)((key >> g.cs) - g.clb), key);
+}
+
+
 // stable stream of all entries with key == k (id order) to out[ob ...]
 template <class Out>
 __device__ void r3_stream_equal(const R3Keys& K, const Out& out, int32_t n, uint64_t k, int32_t ob, uint32_t* sc) {
@@ -533,7 +546,9 @@ __device__ void r3_round(const R3Keys& K, const Out& out, int32_t n, const R3Geo
         const KT k = bk[j];
         const uint16_t v = bv[j];
         const uint64_t k64 = sizeof(KT) == 8 ? (uint64_t)k : ((uint64_t)k << 32);
-        const uint32_t f = r3_fine<KT>(S, g, (uint32_t)((k64 >> g.cs) - g.clb), k64);
+        uint32_t f;
+        if constexpr (sizeof(KT) == 4) f = r3_bin32(S, g, (uint32_t)k);
+        else f = r3_fine<KT>(S, g, (uint32_t)((k64 >> g.cs) - g.clb), k64);
         const uint32_t s0 = (f == b0 ? base : S.starts[f - 1]) - base;
         const uint32_t s1 = S.starts[f] - base;
         uint32_t rank = 0;
@@ -1058,7 +1073,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                     if (key < gf.lo || key > gf.hi) {
                         outside = true;
                     } else {
-                        f = r3_fine<uint32_t>(S, gf, (uint32_t)((key >> gf.cs) - gf.clb), key);
+                        f = r3_bin32(S, gf, D);
                         atomicAdd(&S.starts[f], 1u);
                     }
                     fbuf[t] = (uint16_t)f;
