@@ -72,6 +72,7 @@ def parse():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--no-probe", action="store_true", help="single DAGs: skip the chain-DAG depth probe")
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
     p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c5sim", "c5loc", "c2push", "lu64", "c2n4"))
     p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS,
@@ -215,6 +216,48 @@ def oracle_sample(cfg, w, budget_s, R):
     return reps * w.n / dt, f"1 DAG build + {reps} full score+queue passes of {cfg}", dt
 
 
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def oracle_c5_parallel(w, budget_s, R, threads=None):
+    """c5 on all host cores: the oracle as it stands, one replica per call, independent replicas
+    spread over `threads` Python threads (ctypes drops the GIL inside the C oracle, which keeps
+    no global state).  Returns (tasks/s, sample text, seconds, threads)."""
+    import threading
+    import oracle
+    threads = threads or host_cores()
+    t0 = time.perf_counter()
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    nxt = [0]
+    lock = threading.Lock()
+    done = [0]
+
+    def work():
+        while True:
+            with lock:
+                k = nxt[0]
+                if k >= R or time.perf_counter() - t0 >= budget_s:
+                    return
+                nxt[0] += 1
+            oracle.replica(od, w.dur, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, k, want_queue=True)
+            with lock:
+                done[0] += 1
+
+    ts = [threading.Thread(target=work) for _ in range(threads)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    dt = time.perf_counter() - t0
+    return (done[0] * w.n / dt,
+            f"1 DAG build + {done[0]} of {R} replicas of c2 on {threads} threads (perturbation seed {workloads.C5_SEED})",
+            dt, threads)
+
+
 def run_reference(args):
     rank, local, world = env_rank()
     if rank != 0:
@@ -225,9 +268,13 @@ def run_reference(args):
     w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc", "c2n4") else cfg)
     per_step_budget = 3.0 if cfg != "c4" else 10.0
     times, tasks = [], []
+    cores = 1
     for i in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        v, sample, dt = oracle_sample(cfg, w, per_step_budget, args.replicas)
+        if cfg == "c5":
+            v, sample, dt, cores = oracle_c5_parallel(w, per_step_budget, args.replicas)
+        else:
+            v, sample, dt = oracle_sample(cfg, w, per_step_budget, args.replicas)
         if i >= args.warmup:
             times.append(dt)
             tasks.append(v * dt)
@@ -237,7 +284,7 @@ def run_reference(args):
             "scaling": "none", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": CONFIG_TEXT[cfg], "name": cfg,
                        "step": "bounded sample: " + sample},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -411,20 +458,23 @@ def run_ours(args):
         tasks_per_step = n
         result_h = torch.empty(A * mp.SUMMARY_BYTES + 4, dtype=torch.uint8).pin_memory()
 
+        cur = {"dag": dag, "src": src_d, "dst": dst_d}   # the depth probe swaps in its own DAG
+
         def step(rebuild=True):
+            dag_ = cur["dag"]
             if rebuild:
-                mp.dag_rebuild(dag, n, src_d, dst_d)
-            bl, cp, _ = mp.bottom_level(dag, dur_d, w.workers, out=outs.setdefault("bl", dict(
+                mp.dag_rebuild(dag_, n, cur["src"], cur["dst"])
+            bl, cp, _ = mp.bottom_level(dag_, dur_d, w.workers, out=outs.setdefault("bl", dict(
                 bl=torch.empty(n, dtype=torch.float32, device=dev), cp=torch.empty(1, dtype=torch.float32, device=dev),
                 nod=None)))
-            gain, hd, flags = mp.affinity(dag, dur_d, w.workers, out=outs.setdefault("aff", dict(
+            gain, hd, flags = mp.affinity(dag_, dur_d, w.workers, out=outs.setdefault("aff", dict(
                 gain=torch.empty((n, A), dtype=torch.float32, device=dev),
                 hd=torch.empty(A, dtype=torch.float32, device=dev),
                 flags=torch.empty((n, A), dtype=torch.uint8, device=dev))))
-            cn, key = mp.score(dag, 0, bl, gain, flags, out=outs.setdefault("sc", dict(
+            cn, key = mp.score(dag_, 0, bl, gain, flags, out=outs.setdefault("sc", dict(
                 crit_norm=torch.empty(n, dtype=torch.float32, device=dev),
                 key=torch.empty((n, A), dtype=torch.int64, device=dev))))
-            qptr, qtask, summ = mp.build_queues(dag, key, flags, dur_d, out=outs.setdefault("q", dict(
+            qptr, qtask, summ = mp.build_queues(dag_, key, flags, dur_d, out=outs.setdefault("q", dict(
                 qptr=torch.empty(A + 1, dtype=torch.int64, device=dev),
                 qtask=torch.empty(n * A, dtype=torch.int32, device=dev),
                 summary=torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev))))
@@ -491,6 +541,41 @@ def run_ours(args):
         score_only = {"ms_per_dag": sc_ms, "tasks_per_s": n / (sc_ms * 1e-3), "build_ms": ms_per_step - sc_ms,
                       "alg_bytes": b_sc, "hbm_frac_of_peak": None,
                       "note": "bottom_level + affinity + score + build_queues on the prebuilt DAG, L2 flushed"}
+        # Depth probe (SURVEY §8(d) two-term roofline): the same calls on a DAG with the same n
+        # and the same depth L but no fan-in/fan-out -- a chain of L tasks plus n - L isolated
+        # tasks -- so the same kernels run; its time is the per-level latency floor plus the
+        # per-task (not per-edge) work.  probe / actual says how much of the time depth explains.
+        Lv = dag.n_levels
+        if not args.no_probe and Lv > 1:
+            src_p = torch.arange(Lv - 1, dtype=torch.int32, device=dev)
+            dst_p = src_p + 1
+            dagp = mp.build_dag(n, src_p, dst_p)
+            assert dagp.n_levels == Lv
+            cur.update(dag=dagp, src=src_p, dst=dst_p)
+            pt = {}
+            for rb in (True, False):
+                for _ in range(2):
+                    step(rebuild=rb)
+                pev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                       for _ in range(args.steps)]
+                torch.cuda.synchronize()
+                for i in range(args.steps):
+                    flush.zero_()
+                    pev[i][0].record(stream)
+                    step(rebuild=rb)
+                    pev[i][1].record(stream)
+                torch.cuda.synchronize()
+                pt[rb] = sum(a.elapsed_time(b) for a, b in pev) / args.steps
+            mp.check(dagp)
+            cur.update(dag=dag, src=src_d, dst=dst_d)
+            dagp.free()
+            score_only["depth_probe"] = {
+                "dag": f"chain of L = {Lv} tasks + {n - Lv} isolated tasks (same n, same depth, E = {Lv - 1})",
+                "ms_score_only": pt[False], "ms_with_ingest": pt[True],
+                "t_level_us_score": pt[False] / Lv * 1e3, "t_level_us_with_ingest": pt[True] / Lv * 1e3,
+                "frac_of_score_only": pt[False] / sc_ms, "frac_of_step": pt[True] / ms_per_step,
+                "note": "two-term roofline: max(bytes floor, depth probe); the probe is a measured lower "
+                        "bound for this n and L through the same calls"}
     step_dev_ms = {k: v[0] / args.steps for k, v in prof.items() if v[1] > 0}
     dom = max(step_dev_ms, key=step_dev_ms.get)
     dom_ms, dom_launches = prof[dom]
@@ -559,13 +644,24 @@ def run_ours(args):
     roof["step_hbm_frac"] = b_alg / (ms_per_step * 1e-3) / 1e9 / peak
     if score_only is not None:
         score_only["hbm_frac_of_peak"] = score_only["alg_bytes"] / (score_only["ms_per_dag"] * 1e-3) / 1e9 / peak
+        if "depth_probe" in score_only:
+            dp = score_only["depth_probe"]
+            dp["bytes_floor_ms"] = score_only["alg_bytes"] / 1e9 / peak * 1e3
+            dp["two_term_floor_ms"] = max(dp["bytes_floor_ms"], dp["ms_score_only"])
+            dp["frac_of_two_term"] = dp["two_term_floor_ms"] / score_only["ms_per_dag"]
 
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         import oracle
         oracle.build()
-        v, sample, dt = oracle_sample(cfg, w, args.cpu_budget_s, args.replicas)
-        cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, "seconds": round(dt, 2)}
+        if cfg == "c5":   # all host cores over independent replicas, plus the 1-core figure
+            v1, sample1, dt1 = oracle_sample(cfg, w, args.cpu_budget_s / 2, args.replicas)
+            v, sample, dt, nth = oracle_c5_parallel(w, args.cpu_budget_s / 2, args.replicas)
+            cpu = {"value": v, "unit": UNIT, "cores": nth, "kind": "oracle", "sample": sample,
+                   "seconds": round(dt, 2), "value_1core": v1, "sample_1core": sample1}
+        else:
+            v, sample, dt = oracle_sample(cfg, w, args.cpu_budget_s, args.replicas)
+            cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, "seconds": round(dt, 2)}
 
     rep = cfg in ("c5", "c5sim")
     line = {"metric": METRIC_SIM if cfg in ("c5sim", "c5loc") else METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
