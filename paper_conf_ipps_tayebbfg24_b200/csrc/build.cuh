@@ -155,36 +155,100 @@ __device__ __forceinline__ int csr_row_bitonic(const int32_t* in, int32_t L, int
 
 // one warp per row (rows longer than CSR_WARP_MAX are listed for the radix path).
 // srt[rs[r] .. rs[r] + ucnt[r]) = sorted distinct successors of r.
+// 32 rows per warp: rows of <= 8 entries are sorted by their own lane in registers
+// (odd-even transposition network, then dedup), longer rows one at a time by the whole
+// warp (rows longer than CSR_WARP_MAX are listed for the radix path).
+// srt[rs[r] .. rs[r] + ucnt[r]) = sorted distinct successors of r.
+constexpr int CSR_LANE_MAX = 8;
+__device__ __forceinline__ int csr_row_warp(const int32_t* tmp, int32_t s, int32_t L, int32_t* run, int32_t* srt,
+                                            int lane) {
+    if (L <= 32) return csr_row_sort<1>(tmp + s, L, run, srt + s, lane);
+    if (L <= 64) return csr_row_bitonic<64>(tmp + s, L, run, srt + s, lane);
+    if (L <= 128) return csr_row_bitonic<128>(tmp + s, L, run, srt + s, lane);
+    return csr_row_bitonic<CSR_WARP_MAX>(tmp + s, L, run, srt + s, lane);
+}
+
+// rpw rows per warp (1..32; the host picks fewer for small n so every warp has work);
+// mid_list != null: rows of CSR_LANE_MAX < L <= CSR_WARP_MAX are listed for
+// k_csr_rowsort_mid (one warp each) instead of being sorted one after another here.
 __global__ void __launch_bounds__(256) k_csr_rowsort(int32_t n, const int32_t* rs, const int32_t* tmp, int32_t* srt,
                                                      int32_t* ucnt, int32_t* big_list,
-                                                     int32_t* big_ctr /* [0]=rows, [1]=entries */,
-                                                     int32_t* big_off) {
+                                                     int32_t* big_ctr /* [0]=rows, [1]=entries, [2]=mid rows */,
+                                                     int32_t* big_off, int rpw, int32_t* mid_list) {
     __shared__ int32_t runs[8][CSR_WARP_MAX];
     const int lane = threadIdx.x & 31;
     int32_t* run = runs[threadIdx.x >> 5];
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {
-        const int32_t s = rs[r], L = rs[r + 1] - s;
-        int c;
-        if (L <= 1) {
-            if (L == 1 && lane == 0) srt[s] = tmp[s];
-            c = L;
-        } else if (L <= 32) {
-            c = csr_row_sort<1>(tmp + s, L, run, srt + s, lane);
-        } else if (L <= 64) {
-            c = csr_row_bitonic<64>(tmp + s, L, run, srt + s, lane);
-        } else if (L <= 128) {
-            c = csr_row_bitonic<128>(tmp + s, L, run, srt + s, lane);
-        } else if (L <= CSR_WARP_MAX) {
-            c = csr_row_bitonic<CSR_WARP_MAX>(tmp + s, L, run, srt + s, lane);
-        } else {
-            if (lane == 0) {
-                int idx = atomicAdd(&big_ctr[0], 1);
-                big_list[idx] = (int32_t)r;
-                big_off[idx] = atomicAdd(&big_ctr[1], L);
-            }
-            continue;
+    for (int64_t r0 = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5) * rpw; r0 < n; r0 += nw * rpw) {
+        const int64_t rl = r0 + lane;
+        int32_t sl = 0, Ll = 0;
+        if (lane < rpw && rl < n) {
+            sl = rs[rl];
+            Ll = rs[rl + 1] - sl;
         }
+        if (lane < rpw && rl < n && Ll <= CSR_LANE_MAX) {
+            int32_t x[CSR_LANE_MAX];
+#pragma unroll
+            for (int q = 0; q < CSR_LANE_MAX; q++) x[q] = q < Ll ? tmp[sl + q] : 0x7fffffff;
+#pragma unroll
+            for (int rd = 0; rd < CSR_LANE_MAX; rd++) {
+#pragma unroll
+                for (int q = rd & 1; q + 1 < CSR_LANE_MAX; q += 2) {
+                    const int32_t lo = min(x[q], x[q + 1]), hi = max(x[q], x[q + 1]);
+                    x[q] = lo;
+                    x[q + 1] = hi;
+                }
+            }
+            int c = 0;
+#pragma unroll
+            for (int q = 0; q < CSR_LANE_MAX; q++) {
+                if (q < Ll && (q == 0 || x[q] != x[q - 1])) {
+                    srt[sl + c] = x[q];
+                    c++;
+                }
+            }
+            ucnt[rl] = c;
+        }
+        const bool listed = mid_list && lane < rpw && rl < n && Ll > CSR_LANE_MAX && Ll <= CSR_WARP_MAX;
+        if (listed) {
+            cg::coalesced_group g = cg::coalesced_threads();
+            int32_t base = 0;
+            if (g.thread_rank() == 0) base = atomicAdd(&big_ctr[2], (int32_t)g.size());
+            mid_list[g.shfl(base, 0) + (int32_t)g.thread_rank()] = (int32_t)rl;
+        }
+        unsigned bigm = __ballot_sync(0xffffffffu, !listed && lane < rpw && rl < n && Ll > CSR_LANE_MAX);
+        while (bigm) {
+            const int l = __ffs(bigm) - 1;
+            bigm &= bigm - 1;
+            const int64_t r = r0 + l;
+            const int32_t s = __shfl_sync(0xffffffffu, sl, l), L = __shfl_sync(0xffffffffu, Ll, l);
+            if (L > CSR_WARP_MAX) {
+                if (lane == 0) {
+                    int idx = atomicAdd(&big_ctr[0], 1);
+                    big_list[idx] = (int32_t)r;
+                    big_off[idx] = atomicAdd(&big_ctr[1], L);
+                }
+                continue;
+            }
+            const int c = csr_row_warp(tmp, s, L, run, srt, lane);
+            if (lane == 0) ucnt[r] = c;
+        }
+    }
+}
+
+// the listed medium rows, one warp each
+__global__ void __launch_bounds__(256) k_csr_rowsort_mid(const int32_t* mid_list, const int32_t* mid_cnt,
+                                                         const int32_t* rs, const int32_t* tmp, int32_t* srt,
+                                                         int32_t* ucnt) {
+    __shared__ int32_t runs[8][CSR_WARP_MAX];
+    const int lane = threadIdx.x & 31;
+    int32_t* run = runs[threadIdx.x >> 5];
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int32_t cnt = *mid_cnt;
+    for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < cnt; i += nw) {
+        const int32_t r = mid_list[i];
+        const int32_t s = rs[r], L = rs[r + 1] - s;
+        const int c = csr_row_warp(tmp, s, L, run, srt, lane);
         if (lane == 0) ucnt[r] = c;
     }
 }
@@ -243,15 +307,42 @@ __global__ void k_csr_big_compact(const int32_t* big_list, const SortPlan* plan,
 
 // deduplicated rows -> final CSR (row_ptr = exclusive scan of ucnt) + in-degrees
 __global__ void k_csr_emit(int32_t n, const int32_t* rs, const int32_t* srt, const int32_t* ucnt,
-                           const int32_t* row_ptr, int32_t* col, int32_t* indeg) {
+                           const int32_t* row_ptr, int32_t* col, int32_t* indeg, int rpw) {
+    // 32 rows per warp (lanes = rows), their entries spread over the lanes as in k_qcols
     const int lane = threadIdx.x & 31;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {
-        const int32_t s = rs[r], c = ucnt[r], o = row_ptr[r];
-        for (int j = lane; j < c; j += 32) {
-            int32_t v = srt[s + j];
-            col[o + j] = v;
-            atomicAdd(&indeg[v], 1);
+    for (int64_t r0 = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5) * rpw; r0 < n; r0 += nw * rpw) {
+        const int64_t r = r0 + lane;
+        int32_t s = 0, c = 0, o = 0;
+        if (lane < rpw && r < n) {
+            s = rs[r];
+            c = ucnt[r];
+            o = row_ptr[r];
+        }
+        int32_t inc = c;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const int32_t y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        const int32_t exc = inc - c;
+        const int32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+        for (int32_t kb = 0; kb < tot; kb += 32) {
+            const int32_t k = kb + lane;
+            int lo = 0;
+#pragma unroll
+            for (int step = 16; step >= 1; step >>= 1) {
+                const int32_t ev = __shfl_sync(0xffffffffu, exc, lo + step);
+                if (ev <= k) lo += step;
+            }
+            const int32_t os = __shfl_sync(0xffffffffu, s, lo);
+            const int32_t oe = __shfl_sync(0xffffffffu, exc, lo);
+            const int32_t oo = __shfl_sync(0xffffffffu, o, lo);
+            if (k < tot) {
+                const int32_t v = srt[os + (k - oe)];
+                col[oo + (k - oe)] = v;
+                atomicAdd(&indeg[v], 1);
+            }
         }
     }
 }
@@ -263,7 +354,7 @@ struct KahnArgs {
     const int32_t* indeg;
     int32_t* rem;
     int32_t* level;
-    int32_t* front[2];
+    int32_t* front[2];    // frontier lists of int2 {row start, row end} (successor range of each node)
     int32_t* counts;      // [n+2], zeroed: counts[k] = size of frontier k
     int32_t* out;         // [0] = number of levels L, [1] = processed
     uint32_t* err;
@@ -271,15 +362,22 @@ struct KahnArgs {
 
 // Light grid barrier for a co-resident (cooperative) grid: one monotonically
 // increasing arrival counter, thread 0 of each block spins with acquire loads.
-MP_INLINE void grid_barrier(unsigned* bar, unsigned& epoch) {
+MP_INLINE void grid_barrier(unsigned* bar, unsigned& epoch, bool rel = false) {
     // bar[0]: arrivals (monotonic); bar[32]: release flag (its own 128-byte line).  The last
     // block to arrive publishes the epoch; the others poll the flag, not the atomic counter.
+    // rel: the arrival is one acq_rel atomic at gpu scope (cumulative over the block's writes
+    // ordered before it by the __syncthreads) instead of a full fence + relaxed atomic.
     __syncthreads();
     epoch++;
     if (threadIdx.x == 0) {
-        __threadfence();
         const unsigned target = epoch * gridDim.x;
-        const unsigned old = atomicAdd(bar, 1u);
+        unsigned old;
+        if (rel) {
+            asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(old) : "l"(bar) : "memory");
+        } else {
+            __threadfence();
+            old = atomicAdd(bar, 1u);
+        }
         if (old + 1u == target) {
             asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(bar + 32), "r"(epoch) : "memory");
         } else {
@@ -292,12 +390,49 @@ MP_INLINE void grid_barrier(unsigned* bar, unsigned& epoch) {
     __syncthreads();
 }
 
-MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int32_t v) {
+// grid_barrier that also broadcasts the size of the next frontier: the last block to arrive
+// reads *cnt_next (every append of the level happened before its block's arrival) and
+// publishes (count << 32 | epoch) in one 64-bit release store; the pollers get the count
+// with the flag instead of one more dependent L2 read per level.
+MP_INLINE int32_t grid_barrier_cnt(unsigned* bar, unsigned& epoch, const int32_t* cnt_next, int32_t* s_bc) {
+    __syncthreads();
+    epoch++;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const unsigned target = epoch * gridDim.x;
+        const unsigned old = atomicAdd(bar, 1u);
+        unsigned long long v;
+        if (old + 1u == target) {
+            __threadfence();
+            const int32_t c = *((const volatile int32_t*)cnt_next);
+            v = ((unsigned long long)(uint32_t)c << 32) | epoch;
+            asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(bar + 32), "l"(v) : "memory");
+        } else {
+            do {
+                asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(bar + 32) : "memory");
+            } while ((int)((unsigned)v - epoch) < 0);
+        }
+        *s_bc = (int32_t)(v >> 32);
+    }
+    __syncthreads();
+    return *s_bc;
+}
+
+MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int2 v) {
     cg::coalesced_group g = cg::coalesced_threads();
     int32_t base = 0;
     if (g.thread_rank() == 0) base = atomicAdd(counter, (int32_t)g.size());
     base = g.shfl(base, 0);
-    list[base + g.thread_rank()] = v;
+    reinterpret_cast<int2*>(list)[base + g.thread_rank()] = v;
+}
+
+// v just became ready: its level, and its successor range into the next frontier (the row
+// bounds are loaded while the append's atomic is in flight, so the consumer of the frontier
+// reads the range directly instead of one more dependent load of row_ptr)
+MP_INLINE void kahn_ready(const KahnArgs& a, int32_t* counter, int32_t* list, int32_t v, int32_t lvl) {
+    a.level[v] = lvl;
+    const int32_t r0 = a.row_ptr[v], r1 = a.row_ptr[v + 1];
+    kahn_append(counter, list, make_int2(r0, r1));
 }
 
 // Kahn, level-synchronous (a task is ready when all its predecessors are done,
@@ -308,7 +443,7 @@ MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int32_t v) {
 // (one block per SM) with a light grid barrier per level; with one block the
 // barrier is a __syncthreads and the remaining-predecessor counters and the
 // frontier counter live in shared memory.
-__global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int smem_rem) {
+__global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int smem_rem, int var) {
     extern __shared__ int32_t srem[];
     __shared__ int32_t s_row[1024], s_pre[1025];
     __shared__ uint32_t s_sc[40];
@@ -324,18 +459,36 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
         int32_t d = a.indeg[v];
         rem[v] = d;
         a.level[v] = 0;
-        if (d == 0) kahn_append(single ? &s_cnt[0] : &a.counts[0], a.front[0], (int32_t)v);
+        if (d == 0) kahn_append(single ? &s_cnt[0] : &a.counts[0], a.front[0], make_int2(a.row_ptr[v], a.row_ptr[v + 1]));
     }
-    if (single) __syncthreads(); else grid_barrier(bar, epoch);
+    __shared__ int32_t s_bc;
+    int32_t cnt_bc = 0;
+    if (single) __syncthreads();
+    else if (var & 4) cnt_bc = grid_barrier_cnt(bar, epoch, &a.counts[0], &s_bc);
+    else grid_barrier(bar, epoch);
     int32_t k = 0;
     int64_t processed = 0;
     while (true) {
-        const int32_t cnt = single ? *((volatile int32_t*)&s_cnt[k & 1]) : *((volatile int32_t*)&a.counts[k]);
+        const int32_t cnt = single ? *((volatile int32_t*)&s_cnt[k & 1])
+                                   : ((var & 4) ? cnt_bc : *((volatile int32_t*)&a.counts[k]));
         if (cnt == 0) break;
         processed += cnt;
-        const int32_t* cur = a.front[k & 1];
+        const int2* cur = reinterpret_cast<const int2*>(a.front[k & 1]);
         int32_t* nxt = a.front[(k + 1) & 1];
         int32_t* nctr = single ? &s_cnt[(k + 1) & 1] : &a.counts[k + 1];
+        if ((var & 1) && cnt <= (int32_t)((var & 8) ? gridDim.x : gridDim.x * (blockDim.x >> 5))) {
+            // narrow level: one warp per frontier node (spread over the blocks), lanes over its
+            // successors -- no block scan, no block barrier inside the level
+            const int64_t gw = (int64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
+            if (gw < cnt) {
+                const int2 rr = cur[gw];
+                for (int32_t e = rr.x + (int32_t)(threadIdx.x & 31); e < rr.y; e += 32) {
+                    const int32_t v = a.col[e];
+                    if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1);
+                }
+            }
+            if (single) __syncthreads();   // every thread has read cnt before its slot is reset
+        } else {
         // chunk = frontier nodes per block: spread a level over all blocks (so each thread
         // relaxes ~1 edge) but never more than one node per thread
         int64_t chunk = (cnt + gridDim.x - 1) / gridDim.x;
@@ -344,10 +497,9 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
             const int64_t i = threadIdx.x < chunk ? c0 + threadIdx.x : cnt;
             int32_t deg = 0;
             if (i < cnt) {
-                const int32_t u = cur[i];
-                const int32_t r0 = a.row_ptr[u];
-                deg = a.row_ptr[u + 1] - r0;
-                s_row[threadIdx.x] = r0;
+                const int2 rr = cur[i];
+                deg = rr.y - rr.x;
+                s_row[threadIdx.x] = rr.x;
             }
             // block exclusive scan of the degrees
             const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -382,19 +534,19 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
                     else hi = mid - 1;
                 }
                 const int32_t v = a.col[s_row[lo] + (e - s_pre[lo])];
-                if (atomicSub(&rem[v], 1) == 1) {
-                    a.level[v] = k + 1;
-                    kahn_append(nctr, nxt, v);
-                }
+                if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1);
             }
             __syncthreads();
+        }
         }
         k++;
         if (single) {
             if (threadIdx.x == 0) s_cnt[(k + 1) & 1] = 0;   // the list after next starts empty
             __syncthreads();
+        } else if (var & 4) {
+            cnt_bc = grid_barrier_cnt(bar, epoch, &a.counts[k], &s_bc);
         } else {
-            grid_barrier(bar, epoch);
+            grid_barrier(bar, epoch, (var & 2) != 0);
         }
     }
     if (gtid == 0) {
@@ -445,16 +597,45 @@ __global__ void k_qmaps(int32_t n, const int32_t* level, const int32_t* level_pt
 }
 
 // colX[rowX[x] + j] = map[col[row_ptr[v] + j]] for every position x of node v (warp per node)
+// colX[rowX[x] + i] = map[col[row_ptr[nodeX[x]] + i]]: a warp takes 32 consecutive positions
+// (lanes = nodes), scans their degrees and then spreads the batch's edges over its lanes
+// (each lane finds its edge's owner by a 5-step shuffle search), so low-degree nodes do
+// not leave 29 of 32 lanes idle and a high-degree node does not serialise a warp.
 __global__ void k_qcols(int32_t npos, const int32_t* nodeX, const int32_t* rowX, const int32_t* row_ptr,
-                        const int32_t* col, const int32_t* map, int32_t* colX) {
+                        const int32_t* col, const int32_t* map, int32_t* colX, int rpw) {
     const int lane = threadIdx.x & 31;
-    int64_t wid = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t x = wid; x < npos; x += nw) {
-        int32_t v = nodeX[x];
-        if (v < 0) continue;
-        int32_t b = row_ptr[v], e = row_ptr[v + 1], o = rowX[x];
-        for (int32_t j = b + lane; j < e; j += 32) colX[o + (j - b)] = map[col[j]];
+    const int64_t wid = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t x0 = wid * rpw; x0 < npos; x0 += nw * rpw) {
+        const int64_t x = x0 + lane;
+        const int32_t v = (lane < rpw && x < npos) ? nodeX[x] : -1;
+        int32_t b = 0, d = 0, o = 0;
+        if (v >= 0) {
+            b = row_ptr[v];
+            d = row_ptr[v + 1] - b;
+            o = rowX[x];
+        }
+        int32_t inc = d;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const int32_t y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        const int32_t exc = inc - d;
+        const int32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+        for (int32_t kb = 0; kb < tot; kb += 32) {
+            const int32_t k = kb + lane;
+            int lo = 0;   // last lane whose first edge is <= k (its range holds k)
+#pragma unroll
+            for (int step = 16; step >= 1; step >>= 1) {
+                const int32_t ev = __shfl_sync(0xffffffffu, exc, lo + step);
+                if (ev <= k) lo += step;
+            }
+            const int32_t ob = __shfl_sync(0xffffffffu, b, lo);
+            const int32_t oe = __shfl_sync(0xffffffffu, exc, lo);
+            const int32_t oo = __shfl_sync(0xffffffffu, o, lo);
+            if (k < tot) colX[oo + (k - oe)] = map[col[ob + (k - oe)]];
+        }
     }
 }
 
@@ -466,6 +647,13 @@ inline int bits_for(int64_t x) {  // smallest b >= 1 with x <= 2^b
     int b = 1;
     while ((1ll << b) < x) b++;
     return b;
+}
+
+// rows per warp for the batched row kernels: one row per warp while there are more warps
+// than rows / 32 (small DAGs keep every warp busy), up to 32 (lanes = rows) for large ones
+inline int rows_per_warp(int64_t rows, int64_t warps) {
+    int64_t r = rows * 2 / (warps > 0 ? warps : 1);
+    return (int)(r < 1 ? 1 : (r > 32 ? 32 : r));
 }
 
 inline int grid_for(int64_t n, int threads = 256, int64_t cap = 148 * 32) {
@@ -526,7 +714,7 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     const int npass = (2 * b + 7) / 8;
     const int64_t tps = (mm + SORT_TILE - 1) / SORT_TILE;
     size_t bytes = sort_bytes(mm, 1, npass, false) + 2 * align256(mm * 4) + 2 * align256((nn + 1) * 4) + align256(2 * (nn + 1) * 4) +
-                   align256(64) + 256 * 4;
+                   align256((nn + 1) * 4) + align256(64) + 256 * 4;
     {
         mp_status s = ensure_ws(dag, bytes, st);
         if (s) return cleanup(s);
@@ -540,6 +728,7 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     int32_t* cnt = ar.take<int32_t>(nn + 1);   // out-degree counts, then unique counts
     int32_t* rs = ar.take<int32_t>(nn + 1);    // bucket starts
     int32_t* bigb = ar.take<int32_t>(2 * (nn + 1));  // long-row list | offsets
+    int32_t* midl = ar.take<int32_t>(nn + 1);        // medium-row list
     uint64_t** kb = ar.take<uint64_t*>(2);
     int32_t* d_scal = ar.take<int32_t>(8);  // [0]=E, [2..3] = long rows / entries
     ALLOC(dag->col, mm);
@@ -552,8 +741,13 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
             if (s) return cleanup(s);
         }
         MP_LAUNCH(k_csr_fill, grid_for(m), 256, 0, st, d_src, d_dst, m, n, rs, cnt, tmp);
-        MP_LAUNCH(k_csr_rowsort, grid_for((int64_t)n * 32, 256, (int64_t)dag->num_sms * 8), 256, 0, st, n, rs, tmp, srt, cnt, bigb, d_scal + 2,
-                                                                bigb + nn + 1);
+        {
+            const int gr = grid_for((int64_t)n * 32, 256, (int64_t)dag->num_sms * 8);
+            const int rpw = rows_per_warp(n, (int64_t)gr * 8);
+            MP_LAUNCH(k_csr_rowsort, gr, 256, 0, st, n, rs, tmp, srt, cnt, bigb, d_scal + 2, bigb + nn + 1, rpw,
+                      rpw > 1 ? midl : nullptr);
+            if (rpw > 1) MP_LAUNCH(k_csr_rowsort_mid, gr, 256, 0, st, midl, d_scal + 4, rs, tmp, srt, cnt);
+        }
         int32_t h_big[2] = {0, 0};
         CK(cudaMemcpyAsync(h_big, d_scal + 2, 8, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
@@ -574,15 +768,15 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
             if (s) return cleanup(s);
         }
         MP_LAUNCH(k_csr_emit, grid_for((int64_t)n * 32), 256, 0, st, n, rs, srt, cnt, dag->row_ptr, dag->col,
-                                                             dag->indeg);
+                                                             dag->indeg, rows_per_warp(n, (int64_t)grid_for((int64_t)n * 32) * 8));
     } else {
         CK(cudaMemsetAsync(d_scal, 0, 4, st));
     }
 
     // ---- a2: Kahn levels ----------------------------------------------------------------
     ALLOC(dag->b_rem, nn);
-    ALLOC(dag->b_f0, nn);
-    ALLOC(dag->b_f1, nn);
+    ALLOC(dag->b_f0, 2 * nn);   // int2 entries
+    ALLOC(dag->b_f1, 2 * nn);
     ALLOC(dag->b_counts, nn + 2);
     ALLOC(dag->b_kout, 4);
     ALLOC(dag->b_bar, 64);
@@ -612,7 +806,14 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
             CK(cudaFuncSetAttribute(k_kahn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSmemRem * 4)));
             attr = true;
         }
-        void* args[] = {&ka, &bar, &smem_rem};
+        // variant bits (experiments; MP_KAHN_V): 1 = warp-per-node narrow levels, 2 = acq_rel barrier arrival
+        //   4 = the barrier broadcasts the next frontier size, 8 = narrow only up to one node per block
+        // defaults (measured, tools/kahn_ab.sh, with the int2 frontier): one block -> narrow levels
+        // (c2 k_kahn 0.48 -> 0.42 ms); a grid -> frontier size broadcast by the barrier + narrow levels
+        // up to one node per block (c3 2.03 -> 1.72 ms, c4 3.03 -> 2.65 ms)
+        static const int kahn_var = getenv("MP_KAHN_V") ? atoi(getenv("MP_KAHN_V")) : -1;
+        int var = kahn_var >= 0 ? kahn_var : (g == 1 ? 1 : 13);
+        void* args[] = {&ka, &bar, &smem_rem, &var};
         mph::ProfScope kahn_scope("k_kahn", st);
         CK(cudaLaunchCooperativeKernel((void*)k_kahn, dim3((unsigned)g), dim3(1024), args, smem, st));
     }
@@ -698,9 +899,9 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
         }
         if (dag->E > 0) {
             MP_LAUNCH(k_qcols, grid_for((int64_t)n * 32), 256, 0, st, n, dag->nodeq, dag->rowq, dag->row_ptr, dag->col,
-                                                              dag->qof, dag->colq);
+                      dag->qof, dag->colq, rows_per_warp(n, (int64_t)grid_for((int64_t)n * 32) * 8));
             MP_LAUNCH(k_qcols, grid_for(P * 32), 256, 0, st, (int32_t)P, dag->nodep, dag->rowp, dag->row_ptr, dag->col,
-                                                     pof, dag->colp);
+                      pof, dag->colp, rows_per_warp(P, (int64_t)grid_for(P * 32) * 8));
         }
     } else {
         ALLOC(dag->lvlq, 1);
