@@ -123,6 +123,56 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
 #pragma unroll
     for (int q = 0; q < A; q++) { hd[q] = 0; cnt[q] = 0; blo[q] = 0; bhi[q] = 0; }
     float cpm = 0.0f;
+    // Two-arch fast path, decided once per launch from the perturbation's extremes (every
+    // RN op of perturb() is monotone in u, so each perturbed duration lies between its
+    // values at u = 0 and u = 1 - 2^-24; K2 uses the same bound): if every task is enabled
+    // on both archs and every extreme is a nonzero domain value, no perturbed duration can
+    // be 0, +inf or out of the domain, so the enabled masks, the domain checks and the
+    // per-arch counters (= tasks processed) drop out, hd is one |x1 - x0| per task, and if
+    // the exponents span few enough binades, best_remaining_work is summed exactly in one
+    // uint64 of units 2^(emin - 150) (mantissa << (e - emin)) instead of a 128-bit fixed
+    // point per task; converted to the 2^-64 units at the end.
+    __shared__ uint32_t s_fok, s_emin, s_emax;
+    bool fast = false;
+    uint32_t emin = 0;
+    uint64_t acc[2] = {0ull, 0ull};
+    uint32_t hdf = 0, nproc = 0;
+    uint64_t cbase = 0;
+    if constexpr (A == 2) {
+        if (threadIdx.x == 0) {
+            s_fok = (a.emask == 3u && (reinterpret_cast<uintptr_t>(a.base) & 7u) == 0u) ? 1u : 0u;
+            s_emin = 255u;
+            s_emax = 0u;
+        }
+        __syncthreads();
+        bool ok = true;
+        uint32_t lmin = 255u, lmax = 0u;
+        for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
+#pragma unroll
+            for (int b = 0; b < 2; b++) {
+                const float bv = __ldg(a.base + 2 * (int64_t)t + b);
+                const float e0 = perturb_u(bv, a.sigma, 0u), e1 = perturb_u(bv, a.sigma, 0xFFFFFFu);
+                const uint32_t ul = f2u(e0 < e1 ? e0 : e1), uh = f2u(e0 < e1 ? e1 : e0);
+                // both extremes in [2^-41, 2^20) (excludes 0, -0, negatives, inf, NaN)
+                if (!(ul >= 0x2B000000u && ul < 0x49800000u && uh >= 0x2B000000u && uh < 0x49800000u)) ok = false;
+                lmin = min(lmin, ul >> 23);
+                lmax = max(lmax, uh >> 23);
+            }
+        }
+        ok = __all_sync(0xffffffffu, ok);
+        lmin = __reduce_min_sync(0xffffffffu, lmin);
+        lmax = __reduce_max_sync(0xffffffffu, lmax);
+        if (lane == 0) {
+            if (!ok) atomicAnd(&s_fok, 0u);
+            atomicMin(&s_emin, lmin);
+            atomicMax(&s_emax, lmax);
+        }
+        __syncthreads();
+        const uint32_t nb = 32u - __clz((uint32_t)a.n);   // n < 2^nb
+        fast = s_fok && s_emin <= s_emax && 24u + (s_emax - s_emin) + nb <= 64u;
+        emin = s_emin;
+        cbase = (uint64_t)r * (uint64_t)a.n * 2u + 1u;
+    }
     for (int32_t lv = 0; lv < a.L; lv++) {
         const int32_t q1 = __ldg(a.lvlq + lv + 1);
         int32_t q = __ldg(a.lvlq + lv) + w;
@@ -144,10 +194,22 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
                 e1n = __ldg(a.rowq + qn + 1);
                 svn = lane < e1n - e0n ? __ldg(a.colq + e0n + lane) : 0;
             }
+            float wt;
+            if (A == 2 && fast) {
+                const float2 bb = __ldg(reinterpret_cast<const float2*>(a.base) + v);
+                const uint64_t c0 = cbase + 2u * (uint64_t)(uint32_t)v;
+                const float x0 = perturb(bb.x, a.seed, a.sigma, c0), x1 = perturb(bb.y, a.seed, a.sigma, c0 + 1u);
+                wt = x1 < x0 ? x1 : x0;
+                nproc++;
+                const uint32_t ab = f2u(fabsf(__fsub_rn(x1, x0)));
+                hdf = ab > hdf ? ab : hdf;
+                const uint32_t u0 = f2u(x0), u1 = f2u(x1);
+                if (x0 == wt) acc[0] += (uint64_t)((u0 & 0x7fffffu) | 0x800000u) << ((u0 >> 23) - emin);
+                if (x1 == wt) acc[1] += (uint64_t)((u1 & 0x7fffffu) | 0x800000u) << ((u1 >> 23) - emin);
+            } else {
             float x[A];
             uint32_t en;
             int k;
-            float wt;
             r2_durs<A>(a, r, v, x, en, k, wt, bad);
             if (live) {
 #pragma unroll
@@ -170,6 +232,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
                 }
             }
             if (!k) wt = 0.0f;
+            }
             // successors: 32 positions per coalesced load, broadcast by shuffles, gathers 8 at a time
             float m = 0.0f;
             for (int32_t eb = e0; eb < e1; eb += 32) {
@@ -221,6 +284,22 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
         __syncthreads();
         return m;
     };
+    if (A == 2 && fast) {
+        const uint32_t sh = emin - 86u;   // units 2^(emin-150) -> 2^-64 (emin >= 86 in the domain)
+#pragma unroll
+        for (int q = 0; q < A; q++) {
+            if (q >= 2) break;
+            cnt[q] = (int32_t)nproc;
+            hd[q] = hdf;
+            if (sh < 64u) {
+                blo[q] = acc[q] << sh;
+                bhi[q] = sh == 0u ? 0ull : (acc[q] >> (64u - sh));
+            } else {
+                blo[q] = 0ull;
+                bhi[q] = acc[q] << (sh - 64u);
+            }
+        }
+    }
     const uint32_t cpb = colmax(f2u(cpm));
     uint32_t hdb[A];
     int32_t cntb[A];

@@ -292,6 +292,27 @@ def test_replicas_one_arch_and_disabled_arch():
     _replica_check(dis, 33, 64, [0, 31, 32])
 
 
+def test_replicas_k1_fast_path_boundaries():
+    """Two archs, all enabled: k_rep2_bl's fast path (single-uint64 best_remaining_work in
+    units of the smallest binade) on its edges -- equal durations on both archs (every task
+    tied best on both at sigma = 0, and near-ties otherwise), durations at the domain's ends
+    (span too wide: the 128-bit path), and one task whose lower extreme leaves the domain."""
+    w = workloads.config("c1")
+    eq = np.ascontiguousarray(np.repeat(w.dur[:, 1:2], 2, axis=1))
+    We = workloads.Workload("c1eq", w.n, w.src, w.dst, eq, w.arch_names, w.workers)
+    _replica_check(We, 64, 0, range(64), sigma=0.0)
+    _replica_check(We, 64, 0, range(64))
+    wide = w.dur.copy()
+    wide[0, 0] = np.float32(2.0 ** -40)
+    wide[1, 1] = np.float32(2.0 ** 19)
+    Ww = workloads.Workload("c1wide", w.n, w.src, w.dst, np.ascontiguousarray(wide), w.arch_names, w.workers)
+    _replica_check(Ww, 64, 3, range(64))
+    edge = w.dur.copy()
+    edge[2, 0] = np.float32(2.0 ** -41)            # u = 0 draws go below 2^-41 only if sigma > 0: keep sigma 0
+    Wd = workloads.Workload("c1edge", w.n, w.src, w.dst, np.ascontiguousarray(edge), w.arch_names, w.workers)
+    _replica_check(Wd, 32, 9, range(32), sigma=0.0)
+
+
 def test_replicas_ties_stream_path():
     """sigma = 0 on c2: 41,664 GEMMs share one gain -> key ranges with one value > 16384 entries."""
     w = workloads.config("c2")
