@@ -138,6 +138,19 @@ MP_INLINE uint64_t splitmix64(uint64_t seed, uint64_t c) {
     return x ^ (x >> 31);
 }
 
+// perturb() split at the splitmix64 state: x = seed + counter * golden (callers that walk
+// counters add multiples of golden instead of multiplying); the same bits as perturb()
+MP_INLINE float perturb_x(float d, uint64_t x, float sigma) {
+    x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+    x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+    x ^= x >> 31;
+    float u = __fmul_rn((float)(uint32_t)(x >> 40), 0x1p-24f);
+    float s = __fsub_rn(__fmul_rn(2.0f, u), 1.0f);
+    float f = __fadd_rn(1.0f, __fmul_rn(sigma, s));
+    return __fmul_rn(d, f);
+}
+constexpr uint64_t SPLITMIX_GOLDEN = 0x9E3779B97F4A7C15ull;
+
 // the same with u = k * 2^-24 given (k < 2^24): the perturbation at a chosen draw
 MP_INLINE float perturb_u(float d, float sigma, uint32_t k) {
     float u = __fmul_rn((float)k, 0x1p-24f);

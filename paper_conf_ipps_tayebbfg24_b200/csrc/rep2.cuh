@@ -116,6 +116,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
     const bool live = rl < a.R;
     const int64_t r = a.r0 + rl;                 // global replica id
     float* bl32 = a.bl32 + g * (int64_t)a.n * 32;
+    const float* bll = bl32 + lane;              // this lane's (replica's) column
     bool bad = false;
     uint32_t hd[A];
     int32_t cnt[A];
@@ -171,7 +172,8 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
         const uint32_t nb = 32u - __clz((uint32_t)a.n);   // n < 2^nb
         fast = s_fok && s_emin <= s_emax && 24u + (s_emax - s_emin) + nb <= 64u;
         emin = s_emin;
-        cbase = (uint64_t)r * (uint64_t)a.n * 2u + 1u;
+        // splitmix64 state of (r, t = 0, arch 0): seed + ((r n + t) 2 + 1) golden
+        cbase = a.seed + ((uint64_t)r * (uint64_t)a.n * 2u + 1u) * SPLITMIX_GOLDEN;
     }
     for (int32_t lv = 0; lv < a.L; lv++) {
         const int32_t q1 = __ldg(a.lvlq + lv + 1);
@@ -197,15 +199,16 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
             float wt;
             if (A == 2 && fast) {
                 const float2 bb = __ldg(reinterpret_cast<const float2*>(a.base) + v);
-                const uint64_t c0 = cbase + 2u * (uint64_t)(uint32_t)v;
-                const float x0 = perturb(bb.x, a.seed, a.sigma, c0), x1 = perturb(bb.y, a.seed, a.sigma, c0 + 1u);
+                const uint64_t x0s = cbase + (uint64_t)(uint32_t)v * (2u * SPLITMIX_GOLDEN);
+                const float x0 = perturb_x(bb.x, x0s, a.sigma), x1 = perturb_x(bb.y, x0s + SPLITMIX_GOLDEN, a.sigma);
                 wt = x1 < x0 ? x1 : x0;
                 nproc++;
                 const uint32_t ab = f2u(fabsf(__fsub_rn(x1, x0)));
                 hdf = ab > hdf ? ab : hdf;
-                const uint32_t u0 = f2u(x0), u1 = f2u(x1);
-                if (x0 == wt) acc[0] += (uint64_t)((u0 & 0x7fffffu) | 0x800000u) << ((u0 >> 23) - emin);
-                if (x1 == wt) acc[1] += (uint64_t)((u1 & 0x7fffffu) | 0x800000u) << ((u1 >> 23) - emin);
+                const uint32_t uw = f2u(wt);
+                const uint64_t term = (uint64_t)((uw & 0x7fffffu) | 0x800000u) << ((uw >> 23) - emin);
+                acc[0] += x0 == wt ? term : 0ull;
+                acc[1] += x1 == wt ? term : 0ull;
             } else {
             float x[A];
             uint32_t en;
@@ -244,12 +247,12 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
 #pragma unroll
                     for (int u = 0; u < 8; u++) {
                         const int32_t sp = __shfl_sync(0xffffffffu, s32, j + u);
-                        t8[u] = bl32[(int64_t)sp * 32 + lane];
+                        t8[u] = bll[sp * 32];
                     }
 #pragma unroll
                     for (int u = 0; u < 8; u++) m = fmaxf(m, t8[u]);
                 }
-                for (; j < cb; j++) m = fmaxf(m, bl32[(int64_t)__shfl_sync(0xffffffffu, s32, j) * 32 + lane]);
+                for (; j < cb; j++) m = fmaxf(m, bll[__shfl_sync(0xffffffffu, s32, j) * 32]);
             }
             const float bb = __fadd_rn(wt, m);
             bl32[(int64_t)q * 32 + lane] = bb;
