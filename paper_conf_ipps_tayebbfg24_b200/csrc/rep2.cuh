@@ -63,6 +63,7 @@ struct Rep2Args {
     int32_t* counts;             // [R][A]
     unsigned long long* brw;     // [R][A][2]
     uint32_t* err;
+    int flow;                    // K1: 1 = dataflow over the whole q range (one CTA per group)
     // K2
     uint32_t* s_key;             // [grid][2][npad] per-CTA hot scratch: D in id order, D in sorted order
     uint16_t* s_pi;              // [grid][2][npad] per-CTA hot scratch: fine-bin ids, sorted positions
@@ -175,9 +176,23 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
         // splitmix64 state of (r, t = 0, arch 0): seed + ((r n + t) 2 + 1) golden
         cbase = a.seed + ((uint64_t)r * (uint64_t)a.n * 2u + 1u) * SPLITMIX_GOLDEN;
     }
-    for (int32_t lv = 0; lv < a.L; lv++) {
-        const int32_t q1 = __ldg(a.lvlq + lv + 1);
-        int32_t q = __ldg(a.lvlq + lv) + w;
+    // Dataflow mode (one CTA per group): no barrier per level.  The warps walk the whole
+    // q range (reverse level order) with stride 32; a node's bl line is published by a
+    // per-position ready byte in shared memory (data stores, __syncwarp, block fence, flag),
+    // and a gather first waits for its successor's byte (a successor has a smaller q, so
+    // the smallest unfinished node can always proceed: no deadlock).  Narrow levels then
+    // overlap with the next ones instead of idling 32 - width warps at a barrier.
+    const bool flow = a.flow != 0 && cs == 1;
+    volatile uint8_t* rdy = reinterpret_cast<volatile uint8_t*>(r2_smem);
+    if (flow) {
+        for (int32_t i = threadIdx.x; i < (a.n + 3) / 4; i += R2_THREADS)
+            reinterpret_cast<volatile uint32_t*>(r2_smem)[i] = 0u;
+        __syncthreads();
+    }
+    const int32_t nlv = flow ? 1 : a.L;
+    for (int32_t lv = 0; lv < nlv; lv++) {
+        const int32_t q1 = flow ? a.n : __ldg(a.lvlq + lv + 1);
+        int32_t q = (flow ? 0 : __ldg(a.lvlq + lv)) + w;
         // software pipeline: the CSR slice of the warp's next node is loaded while the
         // current node hashes its durations and gathers its successors' bottom-levels
         int32_t v = 0, e0 = 0, e1 = 0, sv = 0;
@@ -244,6 +259,14 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
                 int32_t j = 0;
                 for (; j + 8 <= cb; j += 8) {
                     float t8[8];
+                    if (flow) {
+#pragma unroll
+                        for (int u = 0; u < 8; u++) {
+                            const int32_t sp = __shfl_sync(0xffffffffu, s32, j + u);
+                            while (rdy[sp] == 0) {}
+                        }
+                        __threadfence_block();
+                    }
 #pragma unroll
                     for (int u = 0; u < 8; u++) {
                         const int32_t sp = __shfl_sync(0xffffffffu, s32, j + u);
@@ -252,11 +275,25 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
 #pragma unroll
                     for (int u = 0; u < 8; u++) m = fmaxf(m, t8[u]);
                 }
-                for (; j < cb; j++) m = fmaxf(m, bll[__shfl_sync(0xffffffffu, s32, j) * 32]);
+                for (; j < cb; j++) {
+                    const int32_t sp = __shfl_sync(0xffffffffu, s32, j);
+                    if (flow) {
+                        while (rdy[sp] == 0) {}
+                        __threadfence_block();
+                    }
+                    m = fmaxf(m, bll[sp * 32]);
+                }
             }
             const float bb = __fadd_rn(wt, m);
             bl32[(int64_t)q * 32 + lane] = bb;
             cpm = fmaxf(cpm, bb);
+            if (flow) {   // publish: every lane's store, then the ready byte
+                __syncwarp();
+                if (lane == 0) {
+                    __threadfence_block();
+                    rdy[q] = 1;
+                }
+            }
             q = qn;
             v = vn;
             e0 = e0n;
@@ -1776,6 +1813,8 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         at[0].val.clusterDim.z = 1;
         cfg.attrs = at;
         cfg.numAttrs = 1;
+        static const int k1_flow = getenv("MP_K1_FLOW") ? atoi(getenv("MP_K1_FLOW")) : 1;
+        a.flow = cs == 1 ? k1_flow : 0;
         cudaError_t e;
         {
             mph::ProfScope ps("k_rep2_bl<A>", st);

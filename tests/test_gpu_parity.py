@@ -313,6 +313,20 @@ def test_replicas_k1_fast_path_boundaries():
     _replica_check(Wd, 32, 9, range(32), sigma=0.0)
 
 
+def test_replicas_k1_dataflow_many_groups():
+    """>= 75 groups of 32 replicas: one CTA per group, k_rep2_bl's dataflow mode (ready bytes
+    instead of level barriers), on 1, 2 and 3 archs (masks, one-arch tasks)."""
+    rng = np.random.default_rng(5)
+    c1 = workloads.config("c1")
+    R = 2600
+    sample = sorted(set([0, 31, 32, R - 1] + rng.integers(0, R, 60).tolist()))
+    _replica_check(c1, R, 17, sample)
+    one = workloads.Workload("c1a1", c1.n, c1.src, c1.dst, np.ascontiguousarray(c1.dur[:, :1]), ("CPU",),
+                             np.ones(1, np.int32))
+    _replica_check(one, R, 0, sample)
+    _replica_check(workloads.qr(6), R, 3, sample)
+
+
 def test_replicas_ties_stream_path():
     """sigma = 0 on c2: 41,664 GEMMs share one gain -> key ranges with one value > 16384 entries."""
     w = workloads.config("c2")
