@@ -358,6 +358,7 @@ struct KahnArgs {
     int32_t* counts;      // [n+2], zeroed: counts[k] = size of frontier k
     int32_t* out;         // [0] = number of levels L, [1] = processed
     uint32_t* err;
+    int32_t sfcap;        // one block: frontier entries [0, sfcap) live in shared memory (after rem)
 };
 
 // Light grid barrier for a co-resident (cooperative) grid: one monotonically
@@ -418,22 +419,32 @@ MP_INLINE int32_t grid_barrier_cnt(unsigned* bar, unsigned& epoch, const int32_t
     return *s_bc;
 }
 
-MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int2 v) {
+// frontier slot i: the first `cap` slots of a one-block frontier are in shared memory `sl`
+MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int2 v, int2* sl, int32_t cap) {
     cg::coalesced_group g = cg::coalesced_threads();
     int32_t base = 0;
     if (g.thread_rank() == 0) base = atomicAdd(counter, (int32_t)g.size());
     base = g.shfl(base, 0);
-    reinterpret_cast<int2*>(list)[base + g.thread_rank()] = v;
+    const int32_t i = base + (int32_t)g.thread_rank();
+    if (i < cap) sl[i] = v;
+    else reinterpret_cast<int2*>(list)[i] = v;
 }
 
-// v just became ready: its level, and its successor range into the next frontier (the row
-// bounds are loaded while the append's atomic is in flight, so the consumer of the frontier
-// reads the range directly instead of one more dependent load of row_ptr)
-MP_INLINE void kahn_ready(const KahnArgs& a, int32_t* counter, int32_t* list, int32_t v, int32_t lvl) {
-    a.level[v] = lvl;
-    const int32_t r0 = a.row_ptr[v], r1 = a.row_ptr[v + 1];
-    kahn_append(counter, list, make_int2(r0, r1));
+MP_INLINE int2 kahn_slot(const int2* cur, const int2* sl, int32_t cap, int64_t i) {
+    return i < cap ? sl[i] : cur[i];
 }
+
+// v just became ready: its level, and its successor range into the next frontier, so the
+// consumer of the frontier reads the range directly instead of one more dependent load of
+// row_ptr.  The range is loaded by the caller BEFORE the remaining-predecessor decrement
+// (speculatively, for every edge), so the row_ptr round trip overlaps the atomic's.
+MP_INLINE void kahn_ready(const KahnArgs& a, int32_t* counter, int32_t* list, int32_t v, int32_t lvl, int2 rr,
+                          int2* sl, int32_t cap) {
+    a.level[v] = lvl;
+    kahn_append(counter, list, rr, sl, cap);
+}
+
+MP_INLINE int2 kahn_range(const KahnArgs& a, int32_t v) { return make_int2(a.row_ptr[v], a.row_ptr[v + 1]); }
 
 // Kahn, level-synchronous (a task is ready when all its predecessors are done,
 // P:l.91): level k+1 = successors whose last remaining predecessor is in level
@@ -452,6 +463,8 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
     const bool single = gridDim.x == 1;
     int32_t* rem = smem_rem ? srem : a.rem;
+    const int32_t sfcap = single && smem_rem ? a.sfcap : 0;
+    int2* sfb = reinterpret_cast<int2*>(srem + ((a.n + 1) & ~1));   // [2][sfcap] after rem
     unsigned epoch = 0;
     if (single && threadIdx.x < 2) s_cnt[threadIdx.x] = 0;
     if (single) __syncthreads();
@@ -459,7 +472,7 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
         int32_t d = a.indeg[v];
         rem[v] = d;
         a.level[v] = 0;
-        if (d == 0) kahn_append(single ? &s_cnt[0] : &a.counts[0], a.front[0], make_int2(a.row_ptr[v], a.row_ptr[v + 1]));
+        if (d == 0) kahn_append(single ? &s_cnt[0] : &a.counts[0], a.front[0], kahn_range(a, (int32_t)v), sfb, sfcap);
     }
     __shared__ int32_t s_bc;
     int32_t cnt_bc = 0;
@@ -475,16 +488,19 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
         processed += cnt;
         const int2* cur = reinterpret_cast<const int2*>(a.front[k & 1]);
         int32_t* nxt = a.front[(k + 1) & 1];
+        const int2* scur = sfb + (k & 1) * sfcap;
+        int2* snxt = sfb + ((k + 1) & 1) * sfcap;
         int32_t* nctr = single ? &s_cnt[(k + 1) & 1] : &a.counts[k + 1];
         if ((var & 1) && cnt <= (int32_t)((var & 8) ? gridDim.x : gridDim.x * (blockDim.x >> 5))) {
             // narrow level: one warp per frontier node (spread over the blocks), lanes over its
             // successors -- no block scan, no block barrier inside the level
             const int64_t gw = (int64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
             if (gw < cnt) {
-                const int2 rr = cur[gw];
+                const int2 rr = kahn_slot(cur, scur, sfcap, gw);
                 for (int32_t e = rr.x + (int32_t)(threadIdx.x & 31); e < rr.y; e += 32) {
                     const int32_t v = a.col[e];
-                    if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1);
+                    const int2 vr = kahn_range(a, v);
+                    if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1, vr, snxt, sfcap);
                 }
             }
             if (single) __syncthreads();   // every thread has read cnt before its slot is reset
@@ -497,7 +513,7 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
             const int64_t i = threadIdx.x < chunk ? c0 + threadIdx.x : cnt;
             int32_t deg = 0;
             if (i < cnt) {
-                const int2 rr = cur[i];
+                const int2 rr = kahn_slot(cur, scur, sfcap, i);
                 deg = rr.y - rr.x;
                 s_row[threadIdx.x] = rr.x;
             }
@@ -534,7 +550,8 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
                     else hi = mid - 1;
                 }
                 const int32_t v = a.col[s_row[lo] + (e - s_pre[lo])];
-                if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1);
+                const int2 vr = kahn_range(a, v);
+                if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1, vr, snxt, sfcap);
             }
             __syncthreads();
         }
@@ -788,10 +805,11 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     CK(cudaMemsetAsync(counts, 0, (nn + 2) * 4, st));
     CK(cudaMemsetAsync(kout, 0, 16, st));
     if (n > 0) {
-        KahnArgs ka{n, dag->row_ptr, dag->col, dag->indeg, rem, dag->level, {f0, f1}, counts, kout, dag->err};
+        KahnArgs ka{n, dag->row_ptr, dag->col, dag->indeg, rem, dag->level, {f0, f1}, counts, kout, dag->err, 0};
         unsigned* bar = (unsigned*)dag->b_bar;
         CK(cudaMemsetAsync(bar, 0, 64 * 4, st));
-        // small DAGs: one CTA, remaining-predecessor counters in shared memory
+        // small DAGs: one CTA, remaining-predecessor counters in shared memory, and the first
+        // sfcap entries of both frontier lists after them (the rest spill to the global lists)
         const int64_t kSmemRem = 48 * 1024;
         int smem_rem = (int64_t)n <= kSmemRem ? 1 : 0;
         int g = 1;
@@ -800,11 +818,22 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
             CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_kahn, 1024, 0));
             g = std::max(1, std::min(bps, 1) * dag->num_sms);
         }
-        size_t smem = smem_rem ? (size_t)n * 4 : 0;
-        static bool attr = false;
-        if (!attr) {
-            CK(cudaFuncSetAttribute(k_kahn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(kSmemRem * 4)));
-            attr = true;
+        static int max_dyn = 0;
+        if (max_dyn == 0) {
+            cudaFuncAttributes fa{};
+            CK(cudaFuncGetAttributes(&fa, k_kahn));
+            int optin = 0;
+            CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dag->device));
+            max_dyn = optin - (int)fa.sharedSizeBytes;
+            CK(cudaFuncSetAttribute(k_kahn, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
+        }
+        static const int sf_env = getenv("MP_KAHN_SF") ? atoi(getenv("MP_KAHN_SF")) : 1;   // experiments
+        size_t smem = 0;
+        if (smem_rem) {
+            const size_t remb = (size_t)((n + 1) & ~1) * 4;
+            const int64_t cap = sf_env ? std::min<int64_t>(8192, ((int64_t)max_dyn - (int64_t)remb) / 16) : 0;
+            ka.sfcap = (int32_t)std::max<int64_t>(0, cap);
+            smem = remb + (size_t)ka.sfcap * 16;
         }
         // variant bits (experiments; MP_KAHN_V): 1 = warp-per-node narrow levels, 2 = acq_rel barrier arrival
         //   4 = the barrier broadcasts the next frontier size, 8 = narrow only up to one node per block

@@ -124,6 +124,19 @@ def test_deep_chain_and_wide_star():
     compare(n, s2, d2, random_dags.dyadic_durations(n, 2, 4), np.ones(2, np.int32))
 
 
+def test_one_block_kahn_frontier_spill():
+    """a2 ingest, one-block Kahn (n <= 48K): the first sfcap (<= 8192) entries of a frontier
+    live in shared memory, the rest spill to the global list -- levels narrower than, equal
+    to and wider than the shared part, and a star whose one level holds 39,999 tasks."""
+    n = 40000
+    s, d = random_dags.star(n)
+    compare(n, s, d, random_dags.dyadic_durations(n, 2, 21), np.ones(2, np.int32))
+    compare(n, d.copy(), s.copy(), random_dags.dyadic_durations(n, 2, 22), np.ones(2, np.int32))
+    n, s, d = random_dags.layered_dag([1, 2047, 2048, 2049, 8191, 8192, 8193, 12000, 5], fan=6, seed=23)
+    assert n <= 48 * 1024
+    compare(n, s, d, random_dags.dyadic_durations(n, 2, 23, tiny_set=True), np.ones(2, np.int32))
+
+
 def test_csr_row_length_boundaries():
     """a1 ingest: rows of every length class of the counting-sort builder (warp rank sort
     up to 256 entries, radix path above), heavy duplication, shuffled edge order."""
