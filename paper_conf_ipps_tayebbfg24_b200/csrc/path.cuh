@@ -44,6 +44,11 @@ MP_INLINE float task_weight(const DurView& d, int32_t v, bool& bad) {
 // ---- a4, small DAGs: one CTA, bottom-levels resident in shared memory ------------
 // Levels are walked from the deepest (q-space is reverse level order) with one
 // __syncthreads per level; bl(v) = w(v) + max bl(succ) with a single RN add.
+// Nothing but the successors' bl depends on the previous level, so it is taken off
+// the per-level chain: a prologue writes every w(v) into its slot sbl[q] (all loads
+// in flight at once), and each thread's first row range of the next level is loaded
+// one level ahead.  A level then costs the colq round trip + the shared-memory max +
+// the barrier (max is exact and order-free, so the bits are unchanged).
 __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
                                                    const int32_t* __restrict__ nodeq,
                                                    const int32_t* __restrict__ rowq,
@@ -52,20 +57,47 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
     extern __shared__ float sbl[];
     bool bad = false;
     float cpm = 0.0f;
+    const int32_t t = (int32_t)threadIdx.x;
+    const int32_t nq = __ldg(lvlq + L);
+    for (int32_t q = t; q < nq; q += blockDim.x) sbl[q] = task_weight(d, __ldg(nodeq + q), bad);
+    int32_t qa = __ldg(lvlq), qb = L > 0 ? __ldg(lvlq + 1) : qa;
+    int32_t pe0 = 0, pe1 = 0;
+    if (qa + t < qb) {
+        pe0 = __ldg(rowq + qa + t);
+        pe1 = __ldg(rowq + qa + t + 1);
+    }
+    __syncthreads();
     for (int32_t r = 0; r < L; r++) {
-        const int32_t q1 = __ldg(lvlq + r + 1);
-        for (int32_t q = __ldg(lvlq + r) + threadIdx.x; q < q1; q += blockDim.x) {
+        const int32_t qc = r + 2 <= L ? __ldg(lvlq + r + 2) : qb;
+        int32_t ne0 = 0, ne1 = 0;
+        if (qb + t < qc) {
+            ne0 = __ldg(rowq + qb + t);
+            ne1 = __ldg(rowq + qb + t + 1);
+        }
+        for (int32_t q = qa + t; q < qb; q += blockDim.x) {
+            int32_t e = pe0, e1 = pe1;
+            if (q != qa + t) {
+                e = __ldg(rowq + q);
+                e1 = __ldg(rowq + q + 1);
+            }
             const int32_t v = __ldg(nodeq + q);
-            const float w = task_weight(d, v, bad);
             float m = 0.0f;  // bl >= 0, and w + 0 = w: same as "bl = w without successors"
-            const int32_t e1 = __ldg(rowq + q + 1);
-            for (int32_t e = __ldg(rowq + q); e < e1; e++) m = fmaxf(m, sbl[__ldg(colq + e)]);
-            const float b = __fadd_rn(w, m);
+            for (; e + 4 <= e1; e += 4) {
+                const int32_t c0 = __ldg(colq + e), c1 = __ldg(colq + e + 1);
+                const int32_t c2 = __ldg(colq + e + 2), c3 = __ldg(colq + e + 3);
+                m = fmaxf(m, fmaxf(fmaxf(sbl[c0], sbl[c1]), fmaxf(sbl[c2], sbl[c3])));
+            }
+            for (; e < e1; e++) m = fmaxf(m, sbl[__ldg(colq + e)]);
+            const float b = __fadd_rn(sbl[q], m);
             sbl[q] = b;
             bl[v] = b;
             cpm = fmaxf(cpm, b);
         }
         __syncthreads();
+        qa = qb;
+        qb = qc;
+        pe0 = ne0;
+        pe1 = ne1;
     }
     cpm = warp_max(cpm);
     if ((threadIdx.x & 31) == 0) atomicMax((uint32_t*)cp, f2u(cpm));
