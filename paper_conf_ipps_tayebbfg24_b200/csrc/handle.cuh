@@ -55,6 +55,7 @@ struct mp_dag {
     int32_t* b_kout = nullptr;
     int32_t* b_pof = nullptr;
     int32_t* b_bar = nullptr;   // grid barrier: arrivals [0], release flag [32]
+    int4* b_colr = nullptr;     // one-block Kahn: per edge {target, its row start, row end, 0}
     std::map<const void*, size_t> caps;  // capacity (bytes) of every grow-only field
 };
 

@@ -59,6 +59,13 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
     float cpm = 0.0f;
     const int32_t t = (int32_t)threadIdx.x;
     const int32_t nq = __ldg(lvlq + L);
+    {
+        // the level walk reads every successor id and row bound once, a level at a time:
+        // pull them into L2 now (one prefetch per 128-byte line) so no level waits on HBM
+        const int32_t E = __ldg(rowq + nq);
+        for (int32_t e = t * 32; e < E; e += blockDim.x * 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(colq + e));
+        for (int32_t q = t * 32; q <= nq; q += blockDim.x * 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(rowq + q));
+    }
     for (int32_t q = t; q < nq; q += blockDim.x) sbl[q] = task_weight(d, __ldg(nodeq + q), bad);
     int32_t qa = __ldg(lvlq), qb = L > 0 ? __ldg(lvlq + 1) : qa;
     int32_t pe0 = 0, pe1 = 0;
