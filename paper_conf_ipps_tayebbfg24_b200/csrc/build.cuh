@@ -431,43 +431,50 @@ MP_INLINE int32_t grid_barrier_cnt(unsigned* bar, unsigned& epoch, const int32_t
 }
 
 // frontier slot i: the first `cap` slots of a one-block frontier are in shared memory `sl`
+template <bool SF>
 MP_INLINE void kahn_append(int32_t* counter, int32_t* list, int2 v, int2* sl, int32_t cap) {
     cg::coalesced_group g = cg::coalesced_threads();
     int32_t base = 0;
     if (g.thread_rank() == 0) base = atomicAdd(counter, (int32_t)g.size());
     base = g.shfl(base, 0);
     const int32_t i = base + (int32_t)g.thread_rank();
-    if (i < cap) sl[i] = v;
+    if (SF && i < cap) sl[i] = v;
     else reinterpret_cast<int2*>(list)[i] = v;
 }
 
+template <bool SF>
 MP_INLINE int2 kahn_slot(const int2* cur, const int2* sl, int32_t cap, int64_t i) {
-    return i < cap ? sl[i] : cur[i];
+    if (SF && i < cap) return sl[i];
+    return cur[i];
 }
 
 // v just became ready: its level, and its successor range into the next frontier, so the
 // consumer of the frontier reads the range directly instead of one more dependent load of
 // row_ptr.  The range is loaded by the caller BEFORE the remaining-predecessor decrement
 // (speculatively, for every edge), so the row_ptr round trip overlaps the atomic's.
+template <bool SF>
 MP_INLINE void kahn_ready(const KahnArgs& a, int32_t* counter, int32_t* list, int32_t v, int32_t lvl, int2 rr,
                           int2* sl, int32_t cap) {
     a.level[v] = lvl;
-    kahn_append(counter, list, rr, sl, cap);
+    kahn_append<SF>(counter, list, rr, sl, cap);
 }
 
 MP_INLINE int2 kahn_range(const KahnArgs& a, int32_t v) { return make_int2(a.row_ptr[v], a.row_ptr[v + 1]); }
 
 // edge e's target and the target's successor range
-MP_INLINE int32_t kahn_edge(const KahnArgs& a, int64_t e, int2& vr) {
+// (late: the range is loaded only once the decrement made the target ready, see kahn_late)
+MP_INLINE int32_t kahn_edge(const KahnArgs& a, int64_t e, int2& vr, bool late) {
     if (a.colr) {
         const int4 c = a.colr[e];
         vr = make_int2(c.y, c.z);
         return c.x;
     }
     const int32_t v = a.col[e];
-    vr = kahn_range(a, v);
+    if (!late) vr = kahn_range(a, v);
     return v;
 }
+
+MP_INLINE int2 kahn_late(const KahnArgs& a, int32_t v, int2 vr, bool late) { return late ? kahn_range(a, v) : vr; }
 
 // Kahn, level-synchronous (a task is ready when all its predecessors are done,
 // P:l.91): level k+1 = successors whose last remaining predecessor is in level
@@ -477,6 +484,7 @@ MP_INLINE int32_t kahn_edge(const KahnArgs& a, int64_t e, int2& vr) {
 // (one block per SM) with a light grid barrier per level; with one block the
 // barrier is a __syncthreads and the remaining-predecessor counters and the
 // frontier counter live in shared memory.
+template <bool SF>   // SF: one block with the shared-memory frontier (the grid path has no smem slots)
 __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int smem_rem, int var) {
     extern __shared__ int32_t srem[];
     __shared__ int32_t s_row[1024], s_pre[1025];
@@ -486,7 +494,8 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
     const bool single = gridDim.x == 1;
     int32_t* rem = smem_rem ? srem : a.rem;
-    const int32_t sfcap = single && smem_rem ? a.sfcap : 0;
+    const int32_t sfcap = SF ? a.sfcap : 0;
+    const bool late = (var & 16) != 0;
     int2* sfb = reinterpret_cast<int2*>(srem + ((a.n + 1) & ~1));   // [2][sfcap] after rem
     unsigned epoch = 0;
     if (single && threadIdx.x < 2) s_cnt[threadIdx.x] = 0;
@@ -495,7 +504,7 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
         int32_t d = a.indeg[v];
         rem[v] = d;
         a.level[v] = 0;
-        if (d == 0) kahn_append(single ? &s_cnt[0] : &a.counts[0], a.front[0], kahn_range(a, (int32_t)v), sfb, sfcap);
+        if (d == 0) kahn_append<SF>(single ? &s_cnt[0] : &a.counts[0], a.front[0], kahn_range(a, (int32_t)v), sfb, sfcap);
     }
     __shared__ int32_t s_bc;
     int32_t cnt_bc = 0;
@@ -519,11 +528,11 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
             // successors -- no block scan, no block barrier inside the level
             const int64_t gw = (int64_t)(threadIdx.x >> 5) * gridDim.x + blockIdx.x;
             if (gw < cnt) {
-                const int2 rr = kahn_slot(cur, scur, sfcap, gw);
+                const int2 rr = kahn_slot<SF>(cur, scur, sfcap, gw);
                 for (int32_t e = rr.x + (int32_t)(threadIdx.x & 31); e < rr.y; e += 32) {
-                    int2 vr;
-                    const int32_t v = kahn_edge(a, e, vr);
-                    if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1, vr, snxt, sfcap);
+                    int2 vr = make_int2(0, 0);
+                    const int32_t v = kahn_edge(a, e, vr, late);
+                    if (atomicSub(&rem[v], 1) == 1) kahn_ready<SF>(a, nctr, nxt, v, k + 1, kahn_late(a, v, vr, late), snxt, sfcap);
                 }
             }
             if (single) __syncthreads();   // every thread has read cnt before its slot is reset
@@ -536,7 +545,7 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
             const int64_t i = threadIdx.x < chunk ? c0 + threadIdx.x : cnt;
             int32_t deg = 0;
             if (i < cnt) {
-                const int2 rr = kahn_slot(cur, scur, sfcap, i);
+                const int2 rr = kahn_slot<SF>(cur, scur, sfcap, i);
                 deg = rr.y - rr.x;
                 s_row[threadIdx.x] = rr.x;
             }
@@ -572,9 +581,9 @@ __global__ void __launch_bounds__(1024) k_kahn(KahnArgs a, unsigned* bar, int sm
                     if (s_pre[mid] <= e) lo = mid;
                     else hi = mid - 1;
                 }
-                int2 vr;
-                const int32_t v = kahn_edge(a, s_row[lo] + (e - s_pre[lo]), vr);
-                if (atomicSub(&rem[v], 1) == 1) kahn_ready(a, nctr, nxt, v, k + 1, vr, snxt, sfcap);
+                int2 vr = make_int2(0, 0);
+                const int32_t v = kahn_edge(a, s_row[lo] + (e - s_pre[lo]), vr, late);
+                if (atomicSub(&rem[v], 1) == 1) kahn_ready<SF>(a, nctr, nxt, v, k + 1, kahn_late(a, v, vr, late), snxt, sfcap);
             }
             __syncthreads();
         }
@@ -838,17 +847,18 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
         int g = 1;
         if (!smem_rem) {
             int bps = 0;
-            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_kahn, 1024, 0));
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_kahn<false>, 1024, 0));
             g = std::max(1, std::min(bps, 1) * dag->num_sms);
         }
         static int max_dyn = 0;
         if (max_dyn == 0) {
             cudaFuncAttributes fa{};
-            CK(cudaFuncGetAttributes(&fa, k_kahn));
+            CK(cudaFuncGetAttributes(&fa, k_kahn<true>));
             int optin = 0;
             CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dag->device));
             max_dyn = optin - (int)fa.sharedSizeBytes;
-            CK(cudaFuncSetAttribute(k_kahn, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
+            CK(cudaFuncSetAttribute(k_kahn<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
+            CK(cudaFuncSetAttribute(k_kahn<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
         }
         static const int sf_env = getenv("MP_KAHN_SF") ? atoi(getenv("MP_KAHN_SF")) : 1;   // experiments
         size_t smem = 0;
@@ -865,15 +875,19 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
             }
         }
         // variant bits (experiments; MP_KAHN_V): 1 = warp-per-node narrow levels, 2 = acq_rel barrier arrival
-        //   4 = the barrier broadcasts the next frontier size, 8 = narrow only up to one node per block
+        //   4 = the barrier broadcasts the next frontier size, 8 = narrow only up to one node per block,
+        //   16 = a target's row range loaded after its decrement instead of speculatively with it
         // defaults (measured, tools/kahn_ab.sh, with the int2 frontier): one block -> narrow levels
         // (c2 k_kahn 0.48 -> 0.42 ms); a grid -> frontier size broadcast by the barrier + narrow levels
         // up to one node per block (c3 2.03 -> 1.72 ms, c4 3.03 -> 2.65 ms)
         static const int kahn_var = getenv("MP_KAHN_V") ? atoi(getenv("MP_KAHN_V")) : -1;
-        int var = kahn_var >= 0 ? kahn_var : (g == 1 ? 1 : 13);
+        // bit 16 (ranges loaded after the decrement) measured faster than the speculative load on
+        // every config (tools/kahn_late.sh: c3 1.86 -> 1.79 ms, c4 2.83 -> 2.74, lu64 0.95 -> 0.90)
+        int var = kahn_var >= 0 ? kahn_var : (g == 1 ? 17 : 29);
         void* args[] = {&ka, &bar, &smem_rem, &var};
         mph::ProfScope kahn_scope("k_kahn", st);
-        CK(cudaLaunchCooperativeKernel((void*)k_kahn, dim3((unsigned)g), dim3(1024), args, smem, st));
+        const void* kf = ka.sfcap > 0 ? (const void*)k_kahn<true> : (const void*)k_kahn<false>;
+        CK(cudaLaunchCooperativeKernel(kf, dim3((unsigned)g), dim3(1024), args, smem, st));
     }
     int32_t h_scal[2] = {0, 0};
     int32_t h_k[2] = {0, 0};
