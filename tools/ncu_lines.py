@@ -31,7 +31,7 @@ for r in rows[2:]:
     if len(r) == len(h) and r[0].startswith("0x") and r[0] not in seen:
         seen.add(r[0]); data.append(r)
 base = int(data[0][0], 16)
-col = "Warp Stall Sampling (All Samples)"
+col = os.environ.get("NCU_COL", "Warp Stall Sampling (All Samples)")
 agg = collections.Counter()
 reasons = collections.defaultdict(collections.Counter)
 rcols = [k for k in h if k.startswith("stall_") and "Not Issued" not in k]
