@@ -269,7 +269,8 @@ def score_and_queue(dag: Dag, dur, workers, kind=CRIT_BL, done=None):
 # discrete-event MultiPrio simulation (mp_sim_oracle.c)
 # --------------------------------------------------------------------------
 SIM_STATS_DTYPE = np.dtype([("makespan", "<f8"), ("pops", "<i8"), ("evictions", "<i8"), ("dups", "<i8"),
-                            ("rounds", "<i8"), ("moved", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,))])
+                            ("rounds", "<i8"), ("moved", "<i8"), ("busy", "<f8", (8,)), ("ran", "<i4", (8,)),
+                            ("stale", "<i8")])
 SIM_ERR_STUCK = 6
 
 

@@ -14,10 +14,38 @@
  *
  * Citations: "P:l.N" = /root/reference/PAPER.md line N.
  *
- * Pins (tests/test_oracle_pins.py): Table II (P:l.180-187), Fig. 3 NOD values
- * (P:l.198), brute-force longest paths on tiny dyadic DAGs, the tiled
- * Cholesky closed forms, networkx topological generations, Fraction sums for
- * best_remaining_work, Appendix-A golden queues.  No function is unpinned.
+ * Pins, function by function (tests/test_oracle_pins.py unless noted; each
+ * pins the function against something other than itself):
+ *   or_build_dag        networkx topological_generations (levels), Cholesky /
+ *                       QR closed forms n, E, depth, dedup and
+ *                       id/self-loop errors (test_levels_equal_networkx_*,
+ *                       test_cholesky_closed_forms, test_qr_closed_forms,
+ *                       test_error_paths)
+ *   or_check_durations  domain edges 2^-41 / 2^20, NaN, -0, no enabled arch
+ *                       (test_error_paths, test_best_remaining_work_exact)
+ *   or_bottom_level     brute-force path enumeration on dyadic DAGs, networkx
+ *                       longest path, chain/star, Cholesky CP closed form
+ *   or_bottom_level_w   Fractions (mean-weight longest path) (test_n4_oracle)
+ *   or_nod              Fig. 3's printed 2.5 / 1 (P:l.198), Fractions within
+ *                       the c11 bound, in-tree 1/indeg
+ *   or_nod_remaining    Fig. 3's dynamic scenario, Fractions (test_n4_oracle)
+ *   or_affinity         Table II's six printed gains and hd = 19 (P:l.180-187),
+ *                       the rule as worded in P:l.170-172, brute-force hd,
+ *                       two-arch symmetry, hd = 0, workers = 0
+ *   or_affinity_prefix  Table II in the paper's push order, a hand-worked
+ *                       other order (test_n4_oracle)
+ *   or_score  (BL)      Appendix-A crit_n (bl / CP), key order vs Python tuple
+ *                       order on float32 values (test_score_key_packing_order)
+ *   or_score  (NOD)     per-arch normalisation (P:l.166, reading c9) against
+ *                       hand-worked Fig. 3 values with a masked arch and exact
+ *                       Fractions on 3-arch masked DAGs
+ *                       (test_nod_crit_norm_*)
+ *   or_build_queues     Python sorted() on (-gain, -crit_n, id), membership and
+ *                       duplication (P:l.104), READY membership, Appendix-A
+ *                       queues, brw exact vs Fractions
+ *   or_perturb          splitmix64 published reference vector, sigma range and
+ *                       sigma = 0 identity
+ *   or_replica          equals the stepwise path; sigma = 0 equals c2
  */
 #include <math.h>
 #include <stdint.h>

@@ -29,6 +29,12 @@
  * W^-1 sum w + (1 - 1/W) CP (one arch), and trace invariants (precedence,
  * no overlap, exactly-once, greedy / highest-priority-first without
  * eviction), plus Fig. 4's direction (eviction lowers GPU idle time).
+ * `stale` (lazy removals, P:l.130) is pinned by the hand-worked counts in
+ * tests/golden/sim_worked.json; `dups` (duplicates a pop leaves) equals
+ * (enabled archs - 1) per task without eviction, and stale == dups at
+ * completion.  N3 (top_n, any n >= 1; the paper puts no cap on n, P:l.207):
+ * hand-worked locality schedules and an independent replay
+ * (test_locality_replay, top_n up to 64).
  */
 #include <math.h>
 #include <stdint.h>
@@ -48,6 +54,8 @@ typedef struct {             /* per simulated instance                         *
     int64_t moved;           /* bytes of accessed data not resident at start   */
     double busy[8];          /* sum of delta(t,a) over tasks run on arch a     */
     int32_t ran[8];          /* tasks run on arch a                            */
+    int64_t stale;           /* processed duplicates met at a heap root and     */
+                             /* dropped there ("lazily removed", P:l.130)      */
 } so_stats;
 
 /* delta as an exact integer count of 2^-64 ms (domain: 0 or [2^-41, 2^20)) */
@@ -122,6 +130,7 @@ typedef struct {
     const uint64_t* size;    /* [H] bytes                                      */
     int32_t H, M;            /* handles, memory nodes                          */
     uint8_t* resident;       /* [M][H]                                         */
+    int32_t* cand;           /* [max(top_n, 1)] candidates of one POP          */
 } sched;
 
 static int en(const sched* s, int32_t t, int32_t a) {
@@ -192,15 +201,15 @@ static uint64_t ls_sdh2(const sched* s, int32_t m, int32_t t) {
  * the higher priority (l3).  On the binary heap: pop the candidates, put
  * back the ones not chosen.  Processed duplicates met on the way are dropped
  * (s5).  Returns the chosen task, already removed from the heap, or -1. */
-static int32_t take_most_local(sched* s, int32_t a, int32_t m) {
+static int32_t take_most_local(sched* s, int32_t a, int32_t m, so_stats* st) {
     heap* h = &s->h[a];
-    int32_t cand[32];
+    int32_t* cand = s->cand;
     int k = 0, kmax = s->top_n > 1 ? s->top_n : 1;
     float g0 = 0.0f;
     while (k < kmax && h->size > 0) {
         int32_t t = h->v[0];
         heap_pop_root(h);
-        if (s->started[t]) continue;
+        if (s->started[t]) { st->stale += 1; continue; }    /* lazy removal (P:l.130) */
         float g = s->gain ? s->gain[(int64_t)t * s->A + a] : 0.0f;
         if (k == 0) g0 = g;
         else {
@@ -230,7 +239,7 @@ static int32_t pop(sched* s, int32_t a, int32_t m, so_stats* st, int* hit_max) {
     int tries = 0;
     *hit_max = 0;
     while (tries < s->max_tries) {
-        int32_t t = take_most_local(s, a, m);      /* already off heap a */
+        int32_t t = take_most_local(s, a, m, st);  /* already off heap a */
         if (t < 0) return -1;
         if (pop_condition(s, t, a)) {              /* heaps_pop_and_update      */
             for (int32_t b = 0; b < s->A; b++)     /* "any duplicate tasks in   */
@@ -276,7 +285,7 @@ typedef struct {               /* simulation options                            
 int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col, const int32_t* indeg,
                 const float* dur, const int32_t* workers, const uint64_t* key, const float* gain,
                 const so_config* cfg, so_stats* st, double* start, int32_t* worker) {
-    if (n < 0 || A < 1 || A > 8 || !cfg || cfg->max_tries < 1 || cfg->top_n > 32) return SO_ERR_ARG;
+    if (n < 0 || A < 1 || A > 8 || !cfg || cfg->max_tries < 1) return SO_ERR_ARG;
     if (cfg->top_n > 1 && !gain) return SO_ERR_ARG;
     int32_t W = 0;
     for (int32_t a = 0; a < A; a++) W += workers[a] > 0 ? workers[a] : 0;
@@ -291,6 +300,7 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
     s.H = cfg->acc_ptr ? cfg->n_handles : 0;
     size_t nn = (size_t)n + 1;
     s.counted = (uint8_t*)calloc(nn * (size_t)A, 1);
+    s.cand = (int32_t*)malloc((size_t)(s.top_n > 1 ? s.top_n : 1) * sizeof(int32_t));
     s.started = (uint8_t*)calloc(nn, 1);
     s.rem = (int32_t*)malloc(nn * sizeof(int32_t));
     int32_t* warch = (int32_t*)malloc((size_t)W * sizeof(int32_t));
@@ -305,7 +315,7 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
         s.h[a].key = key; s.h[a].A = A; s.h[a].a = a;
         if (!s.h[a].v) goto out;
     }
-    if (!s.counted || !s.started || !s.rem || !warch || !wtask || !wend || !again || !wnode) goto out;
+    if (!s.counted || !s.cand || !s.started || !s.rem || !warch || !wtask || !wend || !again || !wnode) goto out;
     for (int32_t a = 0, w = 0; a < A; a++)
         for (int32_t k = 0; k < workers[a]; k++, w++) { warch[w] = a; wtask[w] = -1; wend[w] = 0.0; }
     /* memory nodes (l5): given, or arch-0 workers share node 0 and every
@@ -392,6 +402,6 @@ int or_simulate(int32_t n, int32_t A, const int32_t* row_ptr, const int32_t* col
 out:
     for (int32_t a = 0; a < A; a++) free(s.h[a].v);
     free(s.counted); free(s.started); free(s.rem); free(warch); free(wtask); free(wend); free(again);
-    free(wnode); free(s.resident);
+    free(wnode); free(s.resident); free(s.cand);
     return rc;
 }

@@ -175,6 +175,94 @@ def test_nod_in_tree_is_reciprocal_indegree():
     assert nod[n - 1, 0] == 0
 
 
+def _rn32(q: Fraction) -> np.float32:
+    """Correctly rounded binary32 of an exact rational (ties to even)."""
+    f = np.float32(float(q))
+    cands = [np.nextafter(f, np.float32(-np.inf)), f, np.nextafter(f, np.float32(np.inf))]
+    best = min(cands, key=lambda c: (abs(Fraction(float(c)) - q), int(np.float32(c).view(np.uint32)) & 1))
+    return np.float32(best)
+
+
+def test_nod_crit_norm_fig3_two_archs_hand_worked():
+    """a7 with MP_CRIT_NOD: "All values are normalized between 0 and 1" (P:l.166)
+    applied to eq. 2 (P:l.193), reading c9 = divide NOD_a by its max over the
+    tasks enabled on a -- per arch, not one global max.  Fig. 3's DAG with T3
+    unable to run on arch 1; values worked by hand from eq. 2 with the c10
+    filter:
+      arch 0 (all enabled): NOD = T1 2, T2 2.5, T3 1, T5 1/2 (T7's preds T3, T5),
+        others 0; max 2.5  -> crit_n 0.8, 1, 0.4, 0, 0.2, 0, 0
+      arch 1 (T3 off): T1 -> {T2} (indeg_1 1) = 1; T2 -> T4, T5, T6 (T6's
+        arch-1 preds {T2}) = 3; T5 -> T7 (arch-1 preds {T5}) = 1; max 3
+        -> crit_n 1/3, 1, 0, 0, 1/3, 0, 0
+    A global max (3) would give T2 on arch 0 2.5/3, not 1."""
+    g = load("fig3_nod.json")
+    idx = {t: i for i, t in enumerate(g["tasks"])}
+    src = [idx[u] for u, v in g["edges"]]
+    dst = [idx[v] for u, v in g["edges"]]
+    dag = oracle.build_dag(len(idx), src, dst)
+    dur = np.ones((7, 2), np.float32)
+    dur[idx["T3"], 1] = np.inf
+    w = np.ones(2, np.int32)
+    nod = oracle.nod(dag, dur, w)
+    want_nod = [[2, 2.5, 1, 0, 0.5, 0, 0], [1, 3, 0, 0, 1, 0, 0]]
+    assert nod.T.tolist() == want_nod
+    _, _, flags = oracle.affinity(dur, w)
+    gain = np.full((7, 2), 0.5, np.float32)
+    cn, key = oracle.score(oracle.CRIT_NOD, nod, gain, flags)
+    want = [[Fraction(4, 5), 1, Fraction(2, 5), 0, Fraction(1, 5), 0, 0],
+            [Fraction(1, 3), 1, 0, 0, Fraction(1, 3), 0, 0]]
+    for a in range(2):
+        assert [float(x) for x in cn[:, a]] == [float(_rn32(Fraction(q))) for q in want[a]]
+    assert key[idx["T3"], 1] == np.iinfo(np.uint64).max      # not enabled: no queue entry
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_nod_crit_norm_three_archs_masked_against_fractions(seed):
+    """crit_n(t,a) = NOD_a(t) / max over enabled t' of NOD_a(t') (P:l.166,
+    P:l.193, reading c9), checked against exact Fractions computed here from
+    the edge list (not the oracle's NOD): 3 archs, arch 2 enabled on a small
+    subset so the per-arch maxima differ and any other normaliser (global max,
+    max over all tasks, sum) fails."""
+    n = 300
+    rng = np.random.default_rng(40 + seed)
+    src, dst = random_dags.random_dag(n, 3.0, 40 + seed, dup=0.1)
+    dur = random_dags.dyadic_durations(n, 3, 40 + seed, p_inf=0.0)
+    dur[rng.random(n) < 0.3, 1] = np.inf
+    dur[rng.random(n) < 0.8, 2] = np.inf
+    w = np.ones(3, np.int32)
+    dag = oracle.build_dag(n, src, dst)
+    succ = {u: set() for u in range(n)}
+    pred = {u: set() for u in range(n)}
+    for u, v in zip(src.tolist(), dst.tolist()):
+        succ[u].add(v)
+        pred[v].add(u)
+    nod = oracle.nod(dag, dur, w)
+    _, _, flags = oracle.affinity(dur, w)
+    gain = np.full((n, 3), 0.5, np.float32)
+    cn, _ = oracle.score(oracle.CRIT_NOD, nod, gain, flags)
+    maxima = []
+    for a in range(3):
+        en = np.isfinite(dur[:, a])
+        exact = {t: sum((Fraction(1, sum(1 for p in pred[s] if en[p])) for s in succ[t] if en[s]), Fraction(0))
+                 for t in range(n) if en[t]}
+        mx = max(exact.values())
+        maxima.append(mx)
+        assert mx > 0
+        for t in range(n):
+            if not en[t]:
+                assert cn[t, a] == 0
+                continue
+            q = exact[t] / mx
+            # NOD_a is within outdeg 2^-32 + 2^-24 rel of exact (c11), then one RN division
+            tol = float(q) * 2.0 ** -21 + len(succ[t]) * 2.0 ** -32 / float(mx)
+            assert abs(float(cn[t, a]) - float(q)) <= tol, (t, a)
+        # the maximisers get exactly 1
+        arg = [t for t in exact if exact[t] == mx]
+        assert all(cn[t, a] == 1.0 for t in arg)
+        assert 0.0 <= cn[:, a].min() and cn[:, a].max() == 1.0
+    assert len(set(maxima)) == 3             # per-arch maxima differ: the normaliser is visible
+
+
 # ----------------------------------------------------------------------------
 # a1/a2 DAG + levels: networkx, closed forms, invariants
 # ----------------------------------------------------------------------------
