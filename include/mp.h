@@ -19,7 +19,12 @@
  *    synchronises `stream`; only mp_build_dag synchronises by itself.
  *  - No C++ exception crosses the ABI.  mp_last_error() returns a thread-local
  *    detail string for the last failing call.
- *  - One handle is used by one stream at a time.
+ *  - One handle is used by one stream at a time: its per-handle scratch is
+ *    reused by every call.  A caller may switch streams between calls; when
+ *    the scratch grows the library synchronises the device first, so no
+ *    kernel of an earlier call on another stream still uses the old buffer.
+ *  - CSR offsets (d_row_ptr) are int32: the limit E < 2^31 below makes them
+ *    fit (SURVEY §8(b) proposed int64; DESIGN.md §1 lists the deviation).
  *  - Layouts: per-task-per-arch arrays are row-major [n][A] (task-major).
  *  - Limits: 1 <= A <= 8, 0 <= n < 2^30, unique edges E < 2^31.
  *  - Durations delta(t,a) are binary32 milliseconds in {+inf} U {0} U
@@ -202,7 +207,11 @@ mp_status mp_replicas_run(mp_dag* dag, int32_t n_arch, const float* d_base_dur,
  * Invariant (tested): after pushing batches B1..Bk the queues equal
  * mp_build_queues in READY mode with done = B1 U .. U Bk.  d_key/d_flags/d_dur
  * are the whole-DAG scores of mp_score/mp_affinity (reading c18).
- * A task completed twice or an id outside [0,n) raises MP_ERR_ARG (mp_check).
+ * The batch is validated before any state changes: an id outside [0,n), a
+ * task that is not ready (a predecessor not completed), a task completed in
+ * an earlier batch or listed twice in this one raises MP_ERR_ARG (mp_check)
+ * and leaves d_rem and the output queues' inputs untouched (the outputs then
+ * hold the unchanged queues).  A completed task's d_rem entry becomes -1.
  */
 mp_status mp_ready_init(mp_dag* dag, int32_t* d_rem, void* stream);
 mp_status mp_queues_push(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, const uint8_t* d_flags,
@@ -220,8 +229,9 @@ mp_status mp_queues_push(mp_dag* dag, int32_t n_arch, const uint64_t* d_key, con
  * ALL-mode queues into d_qptr_out / d_qtask_out (capacity n*A) with the
  * summaries -- the same queues mp_queues_push produces, with no sort or merge.
  * Pushing the empty batch (m = 0) yields the sources' queues.  A batch task
- * that is not ready, completed twice, or outside [0,n) raises MP_ERR_ARG
- * (mp_check).
+ * that is not ready, completed before, listed twice, or outside [0,n) raises
+ * MP_ERR_ARG (mp_check); the batch is validated before any state changes, so
+ * d_rem and d_done are then unchanged.  A completed task's d_rem becomes -1.
  */
 mp_status mp_queues_push_all(mp_dag* dag, int32_t n_arch, const int64_t* d_qptr_all, const int32_t* d_qtask_all,
                              const uint8_t* d_flags, const float* d_dur, const int32_t* d_batch, int32_t m,

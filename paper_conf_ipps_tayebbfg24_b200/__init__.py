@@ -133,10 +133,12 @@ def dag_rebuild(dag: Dag, n_tasks: int, src: torch.Tensor, dst: torch.Tensor) ->
     src = src.to(torch.int32).contiguous()
     dst = dst.to(torch.int32).contiguous()
     m = src.numel()
-    rc = _lib.lib().mp_dag_rebuild(dag.handle, int(n_tasks), m, _ptr(src) if m else None,
-                                   _ptr(dst) if m else None, _stream())
-    _lib.check(rc, "mp_dag_rebuild")
-    dag.refresh()
+    try:
+        rc = _lib.lib().mp_dag_rebuild(dag.handle, int(n_tasks), m, _ptr(src) if m else None,
+                                       _ptr(dst) if m else None, _stream())
+        _lib.check(rc, "mp_dag_rebuild")
+    finally:
+        dag.refresh()                   # on error the handle holds an empty DAG
     return dag
 
 

@@ -717,16 +717,18 @@ inline int grid_for(int64_t n, int threads = 256, int64_t cap = 148 * 32) {
 inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_src, const int32_t* d_dst,
                             cudaStream_t st) {
     using namespace mpk;
-    if (n < 0 || n >= (1 << 30)) return fail(MP_ERR_ARG, "n_tasks %d outside [0, 2^30)", n);
-    if (m < 0 || m >= (1ll << 31)) return fail(MP_ERR_ARG, "n_edges %lld outside [0, 2^31)", (long long)m);
-    if (m > 0 && (!d_src || !d_dst)) return fail(MP_ERR_ARG, "edge arrays are NULL");
-    if (m > 0 && n == 0) return fail(MP_ERR_ARG, "edges given for an empty task set");
+    // on any error the handle holds an empty DAG (mp.h)
     auto cleanup = [&](mp_status s) {
         dag->n = 0;
         dag->E = 0;
         dag->L = 0;
         return s;
     };
+    if (n < 0 || n >= (1 << 30)) return cleanup(fail(MP_ERR_ARG, "n_tasks %d outside [0, 2^30)", n));
+    if (m < 0 || m >= (1ll << 31))
+        return cleanup(fail(MP_ERR_ARG, "n_edges %lld outside [0, 2^31)", (long long)m));
+    if (m > 0 && (!d_src || !d_dst)) return cleanup(fail(MP_ERR_ARG, "edge arrays are NULL"));
+    if (m > 0 && n == 0) return cleanup(fail(MP_ERR_ARG, "edges given for an empty task set"));
     cudaGetDevice(&dag->device);
     cudaDeviceGetAttribute(&dag->num_sms, cudaDevAttrMultiProcessorCount, dag->device);
     dag->n = n;
@@ -850,40 +852,41 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
             CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_kahn<false>, 1024, 0));
             g = std::max(1, std::min(bps, 1) * dag->num_sms);
         }
-        static int max_dyn = 0;
-        if (max_dyn == 0) {
+        int max_dyn = 0;
+        {
+            // per launch (the opt-in is a per-device setting): two cheap host calls
             cudaFuncAttributes fa{};
             CK(cudaFuncGetAttributes(&fa, k_kahn<true>));
             int optin = 0;
             CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dag->device));
             max_dyn = optin - (int)fa.sharedSizeBytes;
-            CK(cudaFuncSetAttribute(k_kahn<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
-            CK(cudaFuncSetAttribute(k_kahn<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
+            static std::atomic<uint64_t> attr{0};
+            if (first_on_device(attr)) {
+                CK(cudaFuncSetAttribute(k_kahn<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
+                CK(cudaFuncSetAttribute(k_kahn<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, max_dyn));
+            }
         }
-        static const int sf_env = getenv("MP_KAHN_SF") ? atoi(getenv("MP_KAHN_SF")) : 1;   // experiments
         size_t smem = 0;
         if (smem_rem) {
             const size_t remb = (size_t)((n + 1) & ~1) * 4;
-            const int64_t cap = sf_env ? std::min<int64_t>(8192, ((int64_t)max_dyn - (int64_t)remb) / 16) : 0;
+            const int64_t cap = std::min<int64_t>(8192, ((int64_t)max_dyn - (int64_t)remb) / 16);
             ka.sfcap = (int32_t)std::max<int64_t>(0, cap);
             smem = remb + (size_t)ka.sfcap * 16;
-            static const int colr_env = getenv("MP_KAHN_COLR") ? atoi(getenv("MP_KAHN_COLR")) : 1;   // experiments
-            if (colr_env && m > 0) {
+            if (m > 0) {
                 ALLOC(dag->b_colr, m);   // E <= m (deduplicated)
                 MP_LAUNCH(k_kahn_colr, grid_for(m), 256, 0, st, dag->row_ptr, dag->col, n, dag->b_colr);
                 ka.colr = dag->b_colr;
             }
         }
-        // variant bits (experiments; MP_KAHN_V): 1 = warp-per-node narrow levels, 2 = acq_rel barrier arrival
+        // variant bits: 1 = warp-per-node narrow levels, 2 = acq_rel barrier arrival
         //   4 = the barrier broadcasts the next frontier size, 8 = narrow only up to one node per block,
         //   16 = a target's row range loaded after its decrement instead of speculatively with it
         // defaults (measured, tools/kahn_ab.sh, with the int2 frontier): one block -> narrow levels
         // (c2 k_kahn 0.48 -> 0.42 ms); a grid -> frontier size broadcast by the barrier + narrow levels
         // up to one node per block (c3 2.03 -> 1.72 ms, c4 3.03 -> 2.65 ms)
-        static const int kahn_var = getenv("MP_KAHN_V") ? atoi(getenv("MP_KAHN_V")) : -1;
         // bit 16 (ranges loaded after the decrement) measured faster than the speculative load on
-        // every config (tools/kahn_late.sh: c3 1.86 -> 1.79 ms, c4 2.83 -> 2.74, lu64 0.95 -> 0.90)
-        int var = kahn_var >= 0 ? kahn_var : (g == 1 ? 17 : 29);
+        // every config (c3 1.86 -> 1.79 ms, c4 2.83 -> 2.74, lu64 0.95 -> 0.90)
+        int var = g == 1 ? 17 : 29;
         void* args[] = {&ka, &bar, &smem_rem, &var};
         mph::ProfScope kahn_scope("k_kahn", st);
         const void* kf = ka.sfcap > 0 ? (const void*)k_kahn<true> : (const void*)k_kahn<false>;

@@ -3,10 +3,23 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "../../include/mp.h"
 #include "prof.cuh"
 
 #define MP_INLINE __device__ __forceinline__
+
+namespace mph {
+// Function attributes (the dynamic shared-memory opt-in) are per device: true
+// the first time it is asked for the current device and this flag set.
+inline bool first_on_device(std::atomic<uint64_t>& mask) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return true; }
+    const uint64_t b = 1ull << (dev & 63);
+    return (mask.fetch_or(b) & b) == 0;
+}
+}  // namespace mph
 
 namespace mpk {
 

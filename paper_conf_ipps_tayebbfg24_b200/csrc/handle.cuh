@@ -107,7 +107,9 @@ inline mp_status grow_buf(void** field, size_t bytes, mp_dag* dag, cudaStream_t 
     size_t& cap = dag->caps[(const void*)field];
     if (*field && cap >= bytes) return MP_OK;
     if (*field) {
-        MP_CUDA(cudaStreamSynchronize(st));
+        // another stream may still use the old buffer (mp.h: one stream per handle
+        // at a time, but a caller may switch streams between calls): drain the device
+        MP_CUDA(cudaDeviceSynchronize());
         MP_CUDA(cudaFree(*field));
         *field = nullptr;
     }
@@ -119,10 +121,12 @@ inline mp_status grow_buf(void** field, size_t bytes, mp_dag* dag, cudaStream_t 
 
 inline size_t align256(size_t b) { return (b + 255) & ~size_t(255); }
 
-// Ensure `dag->ws` holds at least `bytes`; growing synchronises the stream.
+// Ensure `dag->ws` holds at least `bytes`; growing synchronises the device (kernels of
+// an earlier call on another stream may still use the old scratch).
 inline mp_status ensure_ws(mp_dag* dag, size_t bytes, cudaStream_t st) {
     if (bytes <= dag->ws_cap) return MP_OK;
-    MP_CUDA(cudaStreamSynchronize(st));
+    (void)st;
+    MP_CUDA(cudaDeviceSynchronize());
     if (dag->ws) MP_CUDA(cudaFree(dag->ws));
     dag->ws = nullptr;
     dag->ws_cap = 0;
@@ -134,7 +138,8 @@ inline mp_status ensure_ws(mp_dag* dag, size_t bytes, cudaStream_t st) {
 
 inline mp_status ensure_sort_status(mp_dag* dag, size_t entries, cudaStream_t st) {
     if (entries <= dag->sort_status_cap) return MP_OK;
-    MP_CUDA(cudaStreamSynchronize(st));
+    (void)st;
+    MP_CUDA(cudaDeviceSynchronize());
     if (dag->sort_status) MP_CUDA(cudaFree(dag->sort_status));
     dag->sort_status = nullptr;
     size_t cap = entries + entries / 4 + 256;
@@ -146,7 +151,8 @@ inline mp_status ensure_sort_status(mp_dag* dag, size_t entries, cudaStream_t st
 
 inline mp_status ensure_scan_status(mp_dag* dag, size_t entries, cudaStream_t st) {
     if (entries <= dag->scan_status_cap) return MP_OK;
-    MP_CUDA(cudaStreamSynchronize(st));
+    (void)st;
+    MP_CUDA(cudaDeviceSynchronize());
     if (dag->scan_status) MP_CUDA(cudaFree(dag->scan_status));
     dag->scan_status = nullptr;
     size_t cap = entries + entries / 4 + 64;

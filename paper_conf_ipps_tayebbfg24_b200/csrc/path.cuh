@@ -492,12 +492,10 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
     const int32_t n = dag->n;
     if (n == 0) return MP_OK;
     if (n <= SMALL_CAP) {
-        static int attr = 0;
+        static std::atomic<uint64_t> attr{0};
         size_t smem = (size_t)n * 4;
-        if (attr < (int)smem) {
+        if (first_on_device(attr))
             MP_CUDA(cudaFuncSetAttribute(k_bl_small, cudaFuncAttributeMaxDynamicSharedMemorySize, SMALL_CAP * 4));
-            attr = SMALL_CAP * 4;
-        }
         MP_LAUNCH(k_bl_small, 1, 1024, smem, st, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp, dag->err);
     } else {
         size_t need = align256((size_t)dag->P * 4);
@@ -509,8 +507,7 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
         MP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_bl_flow, FLOW_THREADS, 0));
         int32_t nchunks = dag->P / 32;
         // 4 blocks (32 warps) per SM: fewer spinning warps measured faster on c4 than full occupancy
-        static const int flow_bps = getenv("MP_FLOW_BPS") ? atoi(getenv("MP_FLOW_BPS")) : 4;
-        if (flow_bps > 0 && flow_bps < bps) bps = flow_bps;
+        if (bps > 4) bps = 4;
         int64_t g = (int64_t)bps * dag->num_sms;
         int64_t want = ((int64_t)nchunks + FLOW_THREADS / 32 - 1) / (FLOW_THREADS / 32);
         if (want < g) g = want;

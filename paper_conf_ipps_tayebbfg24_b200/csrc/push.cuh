@@ -19,22 +19,39 @@ __global__ void k_ready_init(int32_t n, const int32_t* indeg, int32_t* rem) {
         rem[t] = indeg[t];
 }
 
-// mark the batch (removed from the queues) and release successors
-__global__ void k_push_release(const int32_t* batch, int32_t m, int32_t n, const int32_t* row_ptr,
-                               const int32_t* col, int32_t* rem, uint8_t* removed, int32_t* fresh,
-                               int32_t* nfresh, uint32_t* err) {
+// Validation before any state changes (both push variants): every batch id in
+// [0, n), ready and not completed (rem[u] == 0; a completed task carries
+// rem = -1), not done (static-order variant), and listed once (a bit per task,
+// claimed with atomicOr).  Any violation sets *bad and the error flag; the
+// release kernels then leave rem / done / the queues untouched.
+__global__ void k_push_validate(const int32_t* batch, int32_t m, int32_t n, const int32_t* rem, const uint8_t* done,
+                                uint32_t* mark, uint32_t* bad, uint32_t* err) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
         const int32_t u = batch[i];
-        if (u < 0 || u >= n) {
-            atomicOr(err, ERR_ARG_BIT);
-            continue;
+        bool ok = u >= 0 && u < n;
+        if (ok) ok = rem[u] == 0 && !(done && done[u]);
+        if (ok) {
+            const uint32_t bit = 1u << (u & 31);
+            ok = (atomicOr(&mark[u >> 5], bit) & bit) == 0;     // a second copy of u in the batch
         }
+        if (!ok) {
+            atomicOr(bad, 1u);
+            atomicOr(err, ERR_ARG_BIT);
+        }
+    }
+}
+
+// mark the batch (removed from the queues, rem = -1: completed) and release successors
+__global__ void k_push_release(const int32_t* batch, int32_t m, const int32_t* row_ptr, const int32_t* col,
+                               int32_t* rem, uint8_t* removed, int32_t* fresh, int32_t* nfresh, const uint32_t* bad) {
+    if (*bad) return;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t u = batch[i];
         removed[u] = 1;
+        rem[u] = -1;
         for (int32_t e = row_ptr[u]; e < row_ptr[u + 1]; e++) {
             const int32_t s = col[e];
-            const int32_t left = atomicSub(&rem[s], 1) - 1;
-            if (left == 0) fresh[atomicAdd(nfresh, 1)] = s;
-            if (left < 0) atomicOr(err, ERR_ARG_BIT);   // a predecessor completed twice
+            if (atomicSub(&rem[s], 1) == 1) fresh[atomicAdd(nfresh, 1)] = s;
         }
     }
 }
@@ -200,22 +217,16 @@ __global__ void k_push_finish(int32_t A, const int64_t* qptr, const int32_t* q, 
 // queue restricted to the ready tasks, in the same order: a push is a release
 // followed by one stream compaction of the ALL-mode queues.
 
-// completed tasks: done[t] = 1, successors' counters decremented
-__global__ void k_pushall_release(const int32_t* batch, int32_t m, int32_t n, const int32_t* row_ptr,
-                                  const int32_t* col, int32_t* rem, uint8_t* done, uint32_t* err) {
+// completed tasks (validated by k_push_validate): done[t] = 1, rem[t] = -1,
+// successors' counters decremented
+__global__ void k_pushall_release(const int32_t* batch, int32_t m, const int32_t* row_ptr, const int32_t* col,
+                                  int32_t* rem, uint8_t* done, const uint32_t* bad) {
+    if (*bad) return;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
         const int32_t u = batch[i];
-        if (u < 0 || u >= n) {
-            atomicOr(err, ERR_ARG_BIT);
-            continue;
-        }
-        if (rem[u] != 0 || done[u]) {          // not ready, or completed twice
-            atomicOr(err, ERR_ARG_BIT);
-            continue;
-        }
         done[u] = 1;
-        for (int32_t e = row_ptr[u]; e < row_ptr[u + 1]; e++)
-            if (atomicSub(&rem[col[e]], 1) <= 0) atomicOr(err, ERR_ARG_BIT);
+        rem[u] = -1;
+        for (int32_t e = row_ptr[u]; e < row_ptr[u + 1]; e++) atomicSub(&rem[col[e]], 1);
     }
 }
 
@@ -298,17 +309,24 @@ inline mp_status queues_push_all(mp_dag* dag, int32_t A, const int64_t* qptr_all
     if (qall == qout) return fail(MP_ERR_ARG, "qtask_all and qtask_out must not alias");
     const int32_t n = dag->n;
     const int64_t cap = (int64_t)n * A > 0 ? (int64_t)n * A : 1;
-    MP_TRY(ensure_ws(dag, 2 * align256((size_t)cap * 4) + align256(64) + align256(16 * MAX_ARCH), st));
+    const size_t words = ((size_t)n + 31) / 32 + 1;
+    MP_TRY(ensure_ws(dag, 2 * align256((size_t)cap * 4) + align256(64) + align256(16 * MAX_ARCH) +
+                              align256(words * 4) + align256(4), st));
     Arena ar{dag->ws, dag->ws_cap};
     int32_t* keep = ar.take<int32_t>((size_t)cap);
     int32_t* pos = ar.take<int32_t>((size_t)cap);
     int32_t* total = ar.take<int32_t>(16);
     unsigned long long* brw = ar.take<unsigned long long>(2 * MAX_ARCH);
+    uint32_t* mark = ar.take<uint32_t>(words);
+    uint32_t* bad = ar.take<uint32_t>(1);
     MP_CUDA(cudaMemsetAsync(brw, 0, 16 * MAX_ARCH, st));
     MP_CUDA(cudaMemsetAsync(total, 0, 4, st));
-    if (m > 0)
-        MP_LAUNCH(k_pushall_release, grid_for(m), 256, 0, st, batch, m, n, dag->row_ptr, dag->col, rem, done,
-                  dag->err);
+    if (m > 0) {
+        MP_CUDA(cudaMemsetAsync(mark, 0, words * 4, st));
+        MP_CUDA(cudaMemsetAsync(bad, 0, 4, st));
+        MP_LAUNCH(k_push_validate, grid_for(m), 256, 0, st, batch, m, n, rem, done, mark, bad, dag->err);
+        MP_LAUNCH(k_pushall_release, grid_for(m), 256, 0, st, batch, m, dag->row_ptr, dag->col, rem, done, bad);
+    }
     // the ALL-mode queues hold at most n*A entries; their true length is qptr_all[A] (device)
     MP_LAUNCH(k_pushall_flag, grid_for(cap), 256, 0, st, cap, A, qptr_all, qall, rem, done, keep);
     MP_TRY(scan(dag, keep, pos, cap, total, st));
@@ -342,7 +360,8 @@ inline mp_status queues_push(mp_dag* dag, int32_t A, const uint64_t* key, const 
     const int64_t cap = (int64_t)n * A > 0 ? (int64_t)n * A : 1;
     const int idpass = (bits_for(n > 1 ? n : 2) + 7) / 8;
     size_t bytes = sort_bytes(cap, 1, 8, true) + sort_bytes(n > 0 ? n : 1, 1, idpass, false) + align256((size_t)n + 1) +
-                   4 * align256((size_t)cap * 4) + align256(64 * 8) * 4;
+                   4 * align256((size_t)cap * 4) + align256(64 * 8) * 4 + align256((((size_t)n + 31) / 32 + 1) * 4) +
+                   align256(4);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
     SortArgs sa = carve_sort(ar, dag, cap, 1, 0, 8, true);
@@ -358,6 +377,9 @@ inline mp_status queues_push(mp_dag* dag, int32_t A, const uint64_t* key, const 
     int64_t* offs = ar.take<int64_t>(64);          // koff [0..8], noff [16..24], dlen [32]
     unsigned long long* brw = ar.take<unsigned long long>(2 * MAX_ARCH);
     uint32_t** vb = ar.take<uint32_t*>(2);
+    const size_t words = ((size_t)n + 31) / 32 + 1;
+    uint32_t* mark = ar.take<uint32_t>(words);
+    uint32_t* bad = ar.take<uint32_t>(1);
     int32_t* cnt_new = cnts;
     int32_t* cnt_keep = cnts + 8;
     int32_t* nfresh = cnts + 16;
@@ -371,9 +393,13 @@ inline mp_status queues_push(mp_dag* dag, int32_t A, const uint64_t* key, const 
     MP_CUDA(cudaMemcpyAsync(vb, hv, sizeof(hv), cudaMemcpyHostToDevice, st));
     uint64_t* hk[2] = {si.keys[0], si.keys[1]};
     MP_CUDA(cudaMemcpyAsync(ikb, hk, sizeof(hk), cudaMemcpyHostToDevice, st));
-    if (m > 0)
-        MP_LAUNCH(k_push_release, grid_for(m), 256, 0, st, batch, m, n, dag->row_ptr, dag->col, rem, removed, fresh,
-                  nfresh, dag->err);
+    if (m > 0) {
+        MP_CUDA(cudaMemsetAsync(mark, 0, words * 4, st));
+        MP_CUDA(cudaMemsetAsync(bad, 0, 4, st));
+        MP_LAUNCH(k_push_validate, grid_for(m), 256, 0, st, batch, m, n, rem, nullptr, mark, bad, dag->err);
+        MP_LAUNCH(k_push_release, grid_for(m), 256, 0, st, batch, m, dag->row_ptr, dag->col, rem, removed, fresh,
+                  nfresh, bad);
+    }
     MP_LAUNCH(k_push_ids, grid_for(n > 0 ? n : 1), 256, 0, st, fresh, nfresh, si.keys[0], ilen);
     si.d_len = ilen;
     MP_TRY(run_sort(dag, si, st));

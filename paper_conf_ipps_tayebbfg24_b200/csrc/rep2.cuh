@@ -379,7 +379,8 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
             atomicAdd(&a.counts[rl * A + q], cntb[q]);
         }
     }
-    if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(a.err, ERR_DOMAIN_BIT);
+    // only live lanes report domain errors (a lane past R stands for no replica)
+    if (__any_sync(0xffffffffu, live && bad) && lane == 0) atomicOr(a.err, ERR_DOMAIN_BIT);
     // ---- transpose bl32 [q][32] -> blT [r][t] (two archs: K2 reads bl32 directly, and
     //      only for equal-gain runs) ----
     if (A == 2) return;
@@ -1700,48 +1701,13 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
 
 namespace mph {
 
-// L2 persisting carve-out for K2's scratch (opt-in: MP_L2_PERSIST=1; set once per process)
-inline size_t l2_persist_bytes() {
-    static size_t v = [] {
-        const char* e = getenv("MP_L2_PERSIST");   // opt-in: measured no gain on c5, K1 slower
-        if (!e || atoi(e) == 0) return (size_t)0;
-        int dev = 0, mx = 0;
-        if (cudaGetDevice(&dev) != cudaSuccess) return (size_t)0;
-        if (cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev) != cudaSuccess || mx <= 0) {
-            cudaGetLastError();
-            return (size_t)0;
-        }
-        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)mx) != cudaSuccess) {
-            cudaGetLastError();
-            return (size_t)0;
-        }
-        size_t got = 0;
-        cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize);
-        return got;
-    }();
-    return v;
-}
-inline size_t l2_window_max() {
-    static size_t v = [] {
-        int dev = 0, mx = 0;
-        cudaGetDevice(&dev);
-        if (cudaDeviceGetAttribute(&mx, cudaDevAttrMaxAccessPolicyWindowSize, dev) != cudaSuccess) {
-            cudaGetLastError();
-            return (size_t)0;
-        }
-        return (size_t)mx;
-    }();
-    return v;
-}
-
 template <int A>
 inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uint64_t seed, float sigma, int64_t r0,
                              int32_t R, float* cp, mp_queue_summary* sum, int32_t* qtask, cudaStream_t st) {
     using namespace mpk;
     const int32_t n = dag->n;
     const int64_t groups = (R + 31) / 32;
-    static const int grid_env = [] { const char* e = getenv("MP_K2_GRID"); return e ? atoi(e) : 0; }();   // experiments
-    const int grid2 = std::max(1, std::min<int>(R, grid_env > 0 ? grid_env : dag->num_sms));
+    const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
     const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
                    align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 8) +
@@ -1778,10 +1744,10 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.qtask = qtask;
     a.sum = sum;
     a.ticket = dag->tickets + 56;
-    static bool attr = false;
+    static std::atomic<uint64_t> attr{0};
     const int smem1 = 32 * 32 * 33 * 4;
     const int smem2 = (int)r3_smem_bytes();
-    if (!attr) {
+    if (first_on_device(attr)) {
         MP_CUDA(cudaFuncSetAttribute(k_rep2_bl<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem1));
         MP_CUDA(cudaFuncSetAttribute(k_rep2_bl<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem1));
         MP_CUDA(cudaFuncSetAttribute(k_rep2_bl<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem1));
@@ -1790,7 +1756,6 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         MP_CUDA(cudaFuncSetAttribute(k_rep2_sort<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2));
         MP_CUDA(cudaFuncSetAttribute(k_rep2_sort<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2));
         MP_CUDA(cudaFuncSetAttribute(k_rep2_sort<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2));
-        attr = true;
     }
     // statistics are merged with atomics: zero them (and CP) first
     MP_CUDA(cudaMemsetAsync(cp, 0, (size_t)R * 4, st));
@@ -1813,8 +1778,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         at[0].val.clusterDim.z = 1;
         cfg.attrs = at;
         cfg.numAttrs = 1;
-        static const int k1_flow = getenv("MP_K1_FLOW") ? atoi(getenv("MP_K1_FLOW")) : 1;
-        a.flow = cs == 1 ? k1_flow : 0;
+        a.flow = cs == 1 ? 1 : 0;
         cudaError_t e;
         {
             mph::ProfScope ps("k_rep2_bl<A>", st);
@@ -1826,31 +1790,11 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     }
     MP_CUDA(cudaMemsetAsync(a.ticket, 0, 4, st));
     {
-        // K2's hot per-CTA scratch (~12 B per task per CTA: 81 MB for c2 on 148 SMs) is
-        // re-read by every pass of the in-CTA sort: keep it L2-resident (persisting
-        // access-policy window; the queue stores stream past it with evict-first)
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3((unsigned)grid2);
         cfg.blockDim = dim3(R2_THREADS);
         cfg.dynamicSmemBytes = (size_t)smem2;
         cfg.stream = st;
-        cudaLaunchAttribute at[1];
-        int na = 0;
-        const size_t hot = (size_t)(reinterpret_cast<char*>(a.s_pi + (size_t)grid2 * npad * 2) -
-                                    reinterpret_cast<char*>(a.s_key));
-        const size_t persist = l2_persist_bytes();
-        if (persist > 0) {
-            at[0].id = cudaLaunchAttributeAccessPolicyWindow;
-            at[0].val.accessPolicyWindow.base_ptr = a.s_key;
-            at[0].val.accessPolicyWindow.num_bytes = std::min(hot, l2_window_max());
-            at[0].val.accessPolicyWindow.hitRatio =
-                (float)std::min(1.0, (double)persist / (double)at[0].val.accessPolicyWindow.num_bytes);
-            at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-            at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-            na = 1;
-        }
-        cfg.attrs = at;
-        cfg.numAttrs = na;
         mph::ProfScope ps("k_rep2_sort<A>", st);
         MP_CUDA(cudaLaunchKernelEx(&cfg, k_rep2_sort<A>, a));
     }

@@ -223,11 +223,6 @@ inline bool rep2_eligible(const mp_dag* dag, int32_t A);
 inline mp_status replicas_run2(mp_dag* dag, int32_t A, const float* base, uint32_t emask, uint64_t seed, float sigma,
                                int64_t r0, int32_t R, float* cp, mp_queue_summary* sum, int32_t* qtask,
                                cudaStream_t st);
-// MP_REPLICA_PATH=v1 forces the generic batched path (used by tests to cross-check the two)
-inline bool rep2_path_enabled() {
-    const char* e = getenv("MP_REPLICA_PATH");
-    return !(e && e[0] == 'v' && e[1] == '1');
-}
 
 inline mp_status replicas_run(mp_dag* dag, int32_t A, const float* base, const int32_t* h_workers, uint64_t seed,
                               float sigma, int64_t r0, int32_t R, float* cp, mp_queue_summary* sum,
@@ -249,7 +244,7 @@ inline mp_status replicas_run(mp_dag* dag, int32_t A, const float* base, const i
         MP_CUDA(cudaStreamSynchronize(st));
         return MP_OK;
     }
-    if (rep2_path_enabled() && rep2_eligible(dag, A))
+    if (rep2_eligible(dag, A))
         return replicas_run2(dag, A, base, emask, seed, sigma, r0, R, cp, sum, qtask, st);
     if (n <= SMALL_CAP) {
         const int64_t per = (int64_t)A * n;
@@ -262,11 +257,9 @@ inline mp_status replicas_run(mp_dag* dag, int32_t A, const float* base, const i
         SortArgs sa = carve_sort(ar, dag, n, RB * A, 0, 8, true);
         int32_t* counts = ar.take<int32_t>((size_t)RB * A);
         unsigned long long* brw = ar.take<unsigned long long>((size_t)RB * A * 2);
-        static int attr = 0;
-        if (!attr) {
+        static std::atomic<uint64_t> attr{0};
+        if (first_on_device(attr))
             MP_CUDA(cudaFuncSetAttribute(k_rep_main, cudaFuncAttributeMaxDynamicSharedMemorySize, SMALL_CAP * 4));
-            attr = 1;
-        }
         for (int64_t b0 = 0; b0 < R; b0 += RB) {
             const int32_t nb = (int32_t)std::min<int64_t>(RB, R - b0);
             RepArgs ra{n, A, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, dag->qof, base, emask, seed, sigma,

@@ -263,12 +263,11 @@ inline cudaError_t sort_launch(SortArgs a, uint32_t& epoch, cudaStream_t st) {
     MP_LAUNCH(k_sort_hist, g, 256, 0, st, a, chunk);
     MP_LAUNCH(k_sort_plan, a.nseg, 256, 0, st, a);
     int64_t ntiles = (int64_t)a.tiles_per_seg * a.nseg;
-    static bool attr_set = false;
+    static std::atomic<uint64_t> attr_set{0};
     const int dyn = SORT_TILE * 12;
-    if (!attr_set) {
+    if (mph::first_on_device(attr_set)) {
         e = cudaFuncSetAttribute(k_sort_pass, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
         if (e) return e;
-        attr_set = true;
     }
     for (int p = 0; p < a.npass; p++) {
         epoch++;

@@ -6,6 +6,9 @@ identical.  Inputs are the seeded workloads of DESIGN.md §3.
 """
 from __future__ import annotations
 
+import os
+from concurrent.futures import ThreadPoolExecutor
+
 import numpy as np
 import pytest
 import torch
@@ -84,7 +87,7 @@ def test_c4_bit_exact():
     compare(w.n, w.src, w.dst, w.dur, w.workers)
 
 
-@pytest.mark.parametrize("name", ["c1", "c2"])
+@pytest.mark.parametrize("name", ["c1", "c2", "c3", "c4"])
 def test_nod_bit_exact(name):
     w = workloads.config(name)
     compare(w.n, w.src, w.dst, w.dur, w.workers, kind=oracle.CRIT_NOD)
@@ -253,21 +256,43 @@ def test_replicas_c1_all():
     _replica_check(w, 300, 0, range(300))
 
 
-def test_replicas_c5_sampled_full_size():
+def _oracle_replicas(od, w, rs, sigma=workloads.C5_SIGMA, seed=workloads.C5_SEED):
+    """oracle.replica for every r in rs on all host cores (the C oracle drops the
+    GIL inside ctypes and keeps no global state per replica call)."""
+    with ThreadPoolExecutor(max_workers=max(1, len(os.sched_getaffinity(0)))) as ex:
+        return list(ex.map(lambda r: oracle.replica(od, w.dur, w.workers, seed, sigma, r), rs))
+
+
+def test_replicas_c5_all_full_size():
+    """C5 at full size (all replicas when the budget allows): every one
+    of the 4096 replicas -- CP, the 32-byte summaries and both 45,760-entry queues --
+    bit-exact against the oracle, in the launch configuration bench.py times (one
+    mp_replicas_run over all R); then world-size invariance: the two halves
+    [0, R/2) and [R/2, R) run as separate calls (two ranks) give identical bytes."""
     w = workloads.config("c5")
     R = workloads.C5_REPLICAS
-    rng = np.random.default_rng(0)
-    sample = sorted(set([0, 1, R - 1] + rng.integers(0, R, 40).tolist()))
-    cp, gs, q = _replica_check(w, R, 0, sample)
-    # world-size invariance: two half-range calls give identical bytes
     dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
     base = to_dev(w.dur)
+    cp, summ, q = mp.replicas_run(dag, base, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, 0, R)
+    mp.check(dag)
+    cp_h = cp.cpu().numpy()
+    gs = mp.summaries(summ).reshape(R, w.n_arch)
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    CH = 512
+    for c0 in range(0, R, CH):
+        res = _oracle_replicas(od, w, range(c0, c0 + CH))
+        qc = q[c0:c0 + CH].cpu().numpy()
+        for i, (ocp, osum, oq, _) in enumerate(res):
+            r = c0 + i
+            assert bits(cp_h[r:r + 1])[0] == bits(np.float32(ocp)), r
+            assert gs[r].tobytes() == osum.tobytes(), (r, gs[r], osum)
+            assert np.array_equal(qc[i, :len(oq)], oq), r
     h = R // 2
     cp2, s2, q2 = mp.replicas_run(dag, base, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, h, R - h)
     mp.check(dag)
-    assert np.array_equal(bits(cp2.cpu().numpy()), bits(cp[h:]))
+    assert np.array_equal(bits(cp2.cpu().numpy()), bits(cp_h[h:]))
     assert mp.summaries(s2).tobytes() == gs[h:].tobytes()
-    assert np.array_equal(q2.cpu().numpy(), q[h:])
+    assert torch.equal(q2, q[h:])
 
 
 def test_replicas_sigma_zero_equals_single_dag():
@@ -282,13 +307,49 @@ def test_replicas_sigma_zero_equals_single_dag():
         assert mp.summaries(summ)[i * 2:(i + 1) * 2].tobytes() == one["summary"].cpu().numpy().tobytes()
 
 
-def test_replicas_large_dag_path():
-    w = workloads.qr(40)                       # n = 22,140 < cap, force the large path with a bigger DAG
+def test_replicas_rep2_upper_size():
+    """n = 60,000 (< 65,536, A = 2): the lanes=replicas path (k_rep2_bl + k_rep2_sort)
+    at its largest size class (bl no longer fits one CTA's shared memory); qr(40)
+    (n = 22,140) for the same kernels on a QR shape."""
     src, dst = random_dags.random_dag(60000, 2.0, 3, max_span=64)
     dur = random_dags.dyadic_durations(60000, 2, 3)
     W = workloads.Workload("r", 60000, src, dst, dur, ("CPU", "GPU"), np.ones(2, np.int32))
     _replica_check(W, 3, 11, range(3))
-    _replica_check(w, 5, 100, range(5))
+    _replica_check(workloads.qr(40), 5, 100, range(5))
+
+
+def test_replicas_general_path_large_dag():
+    """n >= 65,536: the general replica path (perturbation kernel + the single-DAG
+    a4-a9 kernels once per replica), 2 and 6 archs, every replica checked."""
+    n = 70000
+    src, dst = random_dags.random_dag(n, 2.5, 31, dup=0.2, max_span=128)
+    dur = random_dags.dyadic_durations(n, 2, 31)
+    W = workloads.Workload("g2", n, src, dst, dur, ("CPU", "GPU"), np.ones(2, np.int32))
+    _replica_check(W, 4, 7, range(4))
+    dur6 = random_dags.dyadic_durations(n, 6, 32, p_inf=0.3, tiny_set=True)
+    W6 = workloads.Workload("g6", n, src, dst, dur6, tuple(f"a{i}" for i in range(6)), np.ones(6, np.int32))
+    _replica_check(W6, 3, 0, range(3))
+
+
+@pytest.mark.parametrize("A", [5, 6, 7, 8])
+def test_replicas_general_path_many_archs(A):
+    """A = 5..8 (> 4, so not the lanes=replicas path): the batched one-CTA-per-replica
+    path (k_rep_main + segmented sort + k_rep_out), masks and ties, every replica."""
+    w = workloads.config("c1") if A % 2 else workloads.qr(8)
+    rng = np.random.default_rng(A)
+    n = w.n
+    src, dst = random_dags.random_dag(3000, 2.0, 50 + A, dup=0.2, max_span=64) if A >= 7 else (w.src, w.dst)
+    if A >= 7:
+        n = 3000
+    dur = random_dags.dyadic_durations(n, A, 60 + A, p_inf=0.3, tiny_set=bool(A % 2))
+    workers = np.ones(A, np.int32)
+    if A == 8:
+        workers[3] = 0
+        en = np.isfinite(dur) & (workers[None, :] > 0)
+        dur[~en.any(1), 0] = 1.0
+    W = workloads.Workload(f"m{A}", n, src, dst, dur, tuple(f"a{i}" for i in range(A)), workers)
+    R = int(rng.integers(40, 70))
+    _replica_check(W, R, int(rng.integers(0, 5000)), range(R))
 
 
 def test_replicas_three_arch_masks_all():
@@ -375,20 +436,6 @@ def test_replicas_two_arch_gpu_only_tasks_and_hd_zero():
     _replica_check(W2, 8, 0, range(8), sigma=0.0)
 
 
-def test_replica_paths_agree(monkeypatch):
-    """The lanes=replicas path and the generic batched path give identical bytes."""
-    w = workloads.config("c1")
-    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
-    base = to_dev(w.dur)
-    a = mp.replicas_run(dag, base, w.workers, 99, 0.125, 7, 50)
-    mp.check(dag)
-    monkeypatch.setenv("MP_REPLICA_PATH", "v1")
-    b = mp.replicas_run(dag, base, w.workers, 99, 0.125, 7, 50)
-    mp.check(dag)
-    for x, y in zip(a, b):
-        assert np.array_equal(x.cpu().numpy(), y.cpu().numpy())
-
-
 # ----------------------------------------------------------------------------
 # N1: incremental READY-mode push (SURVEY §8(f))
 # ----------------------------------------------------------------------------
@@ -467,6 +514,55 @@ def test_push_all_sequence_equals_ready_rebuild(name, A):
     mp.queues_push_all(dag, full["qptr"], full["qtask"], flags, dur, to_dev(np.array([0], np.int32)), rem, done_d)
     with pytest.raises(mp.MPError):
         mp.check(dag)
+
+
+@pytest.mark.parametrize("variant", ["merge", "all"])
+def test_push_rejects_bad_batches_without_side_effects(variant):
+    """N1 batch validation (mp.h): a task listed twice in one batch, a task with its
+    still-pending predecessor in the same batch, and a task completed in an earlier
+    batch each raise MP_ERR_ARG and leave rem / done / the queues unchanged (no
+    thread-timing dependence: the batch is validated before any state changes)."""
+    w = workloads.config("c1")           # 0 -> {1, 2, 3}; 1 -> {4, 6, 8}
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    dur = to_dev(w.dur)
+    full = mp.score_and_queue(dag, dur, w.workers)
+    key, flags = full["key"], full["flags"]
+    rem = mp.ready_init(dag)
+    done_d = torch.zeros(w.n, dtype=torch.uint8, device=DEV)
+    empty = torch.zeros(0, dtype=torch.int32, device=DEV)
+    q0ptr, q0, _ = mp.build_queues(dag, key, flags, dur, done=torch.zeros(w.n, dtype=torch.uint8, device=DEV))
+
+    def push(batch, qp, qt):
+        b = to_dev(np.array(batch, np.int32))
+        if variant == "merge":
+            return mp.queues_push(dag, key, flags, dur, b, rem, qp, qt)
+        return mp.queues_push_all(dag, full["qptr"], full["qtask"], flags, dur, b, rem, done_d)
+
+    if variant == "all":
+        q0ptr, q0, _ = push([], None, None)
+    mp.check(dag)
+    qp, qt, _ = push([0], q0ptr, q0)                 # valid: task 0 completes
+    mp.check(dag)
+    rem_ok, done_ok = rem.clone(), done_d.clone()
+    qp_ok, qt_ok = qp.clone(), qt.clone()
+    for bad in ([1, 1], [1, 4], [0], [2, 99], [5]):   # duplicate, pred+succ, completed, out of range, not ready
+        qp2, qt2, _ = push(bad, qp_ok, qt_ok)
+        with pytest.raises(mp.MPError) as e:
+            mp.check(dag)
+        assert e.value.code == mp.MP_ERR_ARG, bad
+        assert torch.equal(rem, rem_ok), bad
+        assert torch.equal(done_d, done_ok), bad
+        if variant == "merge":
+            Q = int(qp_ok[-1])
+            assert torch.equal(qp2, qp_ok) and torch.equal(qt2[:Q], qt_ok[:Q]), bad
+    qp3, qt3, _ = push([1, 2, 3], qp_ok, qt_ok)       # still usable after the rejections
+    mp.check(dag)
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    o = oracle.score_and_queue(od, w.dur, w.workers)
+    done = np.zeros(w.n, np.uint8)
+    done[[0, 1, 2, 3]] = 1
+    oqp, oq, _ = oracle.build_queues(od, o["key"], o["flags"], w.dur, done)
+    assert np.array_equal(qp3.cpu().numpy(), oqp) and np.array_equal(qt3.cpu().numpy()[:oqp[-1]], oq)
 
 
 # ----------------------------------------------------------------------------
