@@ -1,19 +1,32 @@
 #!/usr/bin/env python
-"""bench.py -- MultiPrio scoring + queue build on B200 (DESIGN.md §6).
+"""bench.py -- MultiPrio scoring + queue build on B200 (DESIGN.md §6, §9).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config c5|c1..c4]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config c5|c1..c4|...]
 
-A step is one pass of the whole hot path over one batch:
-  c5 (default): ingest the 64x64 tiled-Cholesky DAG (mp_dag_rebuild: a1+a2),
-      score + queue this rank's block of the 4096 duration-perturbed replicas
-      (mp_replicas_run: a3-a10, queues materialised in HBM), and allgather the
-      per-replica records (CP + queue summaries) over NCCL.  Total replicas
-      are fixed as N grows (strong scaling, BASELINE config 5).
-  c1..c4: one DAG per step (rebuild + bottom_level + affinity + score + queues).
-Rank 0 prints ONE JSON line.  Under torchrun every rank runs; the timed
-region is bracketed by barrier + synchronize and the per-rank device time is
-max-reduced.  `--impl reference` times the CPU oracle (the reference arm of
-this tier) on rank 0 only.
+A step is one pass of the hot path over one batch, on a DAG
+already ingested ("t covers mp_bottom_level -> mp_affinity ->
+mp_score -> mp_build_queues (or mp_replicas_run) on a prebuilt DAG;
+mp_build_dag is timed and reported separately, and also as build+score"):
+  c5 (default): score + queue this rank's block of the 4096 duration-perturbed
+      replicas of the 64x64 Cholesky DAG (mp_replicas_run: a3-a10, every
+      replica's queues materialised in HBM), then allgather the 68-byte
+      per-replica records (CP + queue summaries) over NCCL.  --scaling strong
+      (default, BASELINE config 5): 4096 replicas in total split over the N
+      ranks; --scaling weak: 4096 per rank.
+  c1..c4, c4fmm, lu64, hier: one DAG per step (bottom_level + affinity + score
+      + build_queues).
+The ingest (mp_dag_rebuild, a1+a2) is timed on its own (`build_ms`), and the
+e2e figure runs the whole thing from host buffers (H2D of edges + durations,
+ingest, step, D2H of the results).  The headline timed region runs with
+libmp's per-launch profiling OFF; per-kernel times (roofline) come from a
+second, profiled pass of the same steps.
+
+--gpus N > 1 without a torchrun environment re-launches this script under
+`python -m torch.distributed.run --nproc-per-node N` (127.0.0.1).  Under
+torchrun every rank runs; the timed region is bracketed by barrier +
+synchronize and the per-rank device time is max-reduced; rank 0 prints ONE
+JSON line.  `--impl reference` times the CPU oracle (the reference arm of this
+tier) on rank 0 only.
 """
 from __future__ import annotations
 
@@ -52,6 +65,8 @@ CONFIG_TEXT = {
              "(Intel-V100-like node, PAPER.md l.235)",
     "c5loc": "N3: as c5sim with POP's data-locality pick (LS_SDH^2, n = 10, eps = 0.8, PAPER.md l.238) on "
              "960x960-double tiles, per-node residency, transfers at 2^-24 ms/byte (~16.8 GB/s)",
+    "c4fmm": "the FMM octree part of c4 alone (depth 8, 2^19 particles, 1,099,435 tasks, 24,008,280 edges, "
+             "13 levels; TBFMM-shaped, PAPER.md l.263-270), 2 resource types",
     "lu64": "N4 workload: tiled LU without pivoting 64x64 tiles (getrf, PAPER.md l.251; 89,440 tasks), 2 resource types",
     "c2n4": "N4 variants on the 64x64 Cholesky DAG: mean-cost (HEFT) bottom-level, hd as a running max along the "
             "push order (id order), NOD on the remaining graph (first half of the level order completed), "
@@ -60,6 +75,8 @@ CONFIG_TEXT = {
               "(each step: sources, then one mp_queues_push per completion batch = every ready task)",
 }
 L2_FLUSH_BYTES = 256 << 20
+REPLICA_CFGS = ("c5", "c5sim", "c5loc")
+SINGLE_CFGS = ("c1", "c2", "c3", "c4", "c4fmm", "lu64")
 KERNELS = ("k_rep_main", "k_rep_out", "k_sort_pass", "k_sort_hist", "k_sort_plan", "k_kahn", "k_csr_count",
            "k_csr_fill", "k_csr_rowsort", "k_csr_emit", "k_scan_excl", "k_iota_level_keys", "k_level_order", "k_qmaps",
            "k_qcols", "k_bl_small", "k_bl_flow", "k_aff_hd", "k_aff_gain", "k_crit_max", "k_score",
@@ -74,12 +91,12 @@ def parse():
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--no-probe", action="store_true", help="single DAGs: skip the chain-DAG depth probe")
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    p.add_argument("--config", default="c5", choices=("c1", "c2", "c3", "c4", "c5", "c5sim", "c5loc", "c2push", "lu64", "c2n4"))
+    p.add_argument("--config", default="c5", choices=REPLICA_CFGS + SINGLE_CFGS + ("c2push", "c2n4"))
     p.add_argument("--replicas", type=int, default=workloads.C5_REPLICAS,
-                   help="c5: replicas per GPU (weak scaling, default) or in total (--scaling strong)")
-    p.add_argument("--scaling", choices=("weak", "strong"), default="weak",
-                   help="c5 sharding: weak = every rank scores its own block of --replicas replicas "
-                        "(global ids rank*R..), strong = --replicas in total split across ranks")
+                   help="c5: replicas in total (--scaling strong, default) or per GPU (--scaling weak)")
+    p.add_argument("--scaling", choices=("weak", "strong"), default="strong",
+                   help="c5 sharding: strong = --replicas in total split across ranks (BASELINE config 5), "
+                        "weak = every rank scores its own block of --replicas replicas (global ids rank*R..)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-budget-s", type=float, default=12.0)
@@ -150,10 +167,21 @@ class Clocks:
 # --------------------------------------------------------------------------------------------------
 # the oracle as a baseline (rank 0 only)
 # --------------------------------------------------------------------------------------------------
+_ORACLE_DAGS = {}
+
+
+def oracle_dag(w):
+    """The oracle's DAG for workload w, built once (prebuilt, as in our arm's timed step)."""
+    import oracle
+    if w.name not in _ORACLE_DAGS:
+        _ORACLE_DAGS[w.name] = oracle.build_dag(w.n, w.src, w.dst)
+    return _ORACLE_DAGS[w.name]
+
+
 def oracle_sample(cfg, w, budget_s, R):
     import oracle
+    od = oracle_dag(w)
     t0 = time.perf_counter()
-    od = oracle.build_dag(w.n, w.src, w.dst)
     if cfg in ("c5sim", "c5loc"):
         loc = {}
         if cfg == "c5loc":
@@ -167,7 +195,7 @@ def oracle_sample(cfg, w, budget_s, R):
             if time.perf_counter() - t0 >= budget_s or k >= R:
                 break
         dt = time.perf_counter() - t0
-        return k * w.n / dt, (f"1 DAG build + {k} of {R} replicas of c2: queues + simulated schedule "
+        return k * w.n / dt, (f"prebuilt DAG, {k} of {R} replicas of c2: queues + simulated schedule "
                               f"(perturbation seed {workloads.C5_SEED})"), dt
     if cfg == "c5":
         k = 0
@@ -177,10 +205,11 @@ def oracle_sample(cfg, w, budget_s, R):
             if time.perf_counter() - t0 >= budget_s or k >= R:
                 break
         dt = time.perf_counter() - t0
-        return k * w.n / dt, f"1 DAG build + {k} of {R} replicas of c2 (perturbation seed {workloads.C5_SEED})", dt
+        return k * w.n / dt, f"prebuilt DAG, {k} of {R} replicas of c2 (perturbation seed {workloads.C5_SEED})", dt
     if cfg == "c2push":
         r = oracle.score_and_queue(od, w.dur, w.workers)
         dc = oracle.check_durations(w.dur, w.workers)
+        t0 = time.perf_counter()                  # scores precomputed (as in our arm)
         reps = 0
         while True:
             done = np.zeros(w.n, np.uint8)
@@ -194,7 +223,7 @@ def oracle_sample(cfg, w, budget_s, R):
             if time.perf_counter() - t0 >= budget_s:
                 break
         dt = time.perf_counter() - t0
-        return reps * w.n / dt, (f"1 DAG build + scores + {reps} whole c2 schedules, READY-mode queues rebuilt "
+        return reps * w.n / dt, (f"prebuilt DAG and scores, {reps} whole c2 schedules, READY-mode queues rebuilt "
                                  f"after every completion batch"), dt
     reps = 0
     if cfg == "c2n4":
@@ -213,7 +242,7 @@ def oracle_sample(cfg, w, budget_s, R):
         if time.perf_counter() - t0 >= budget_s:
             break
     dt = time.perf_counter() - t0
-    return reps * w.n / dt, f"1 DAG build + {reps} full score+queue passes of {cfg}", dt
+    return reps * w.n / dt, f"prebuilt DAG, {reps} full score+queue passes of {cfg}", dt
 
 
 def host_cores():
@@ -230,8 +259,8 @@ def oracle_c5_parallel(w, budget_s, R, threads=None):
     import threading
     import oracle
     threads = threads or host_cores()
+    od = oracle_dag(w)
     t0 = time.perf_counter()
-    od = oracle.build_dag(w.n, w.src, w.dst)
     nxt = [0]
     lock = threading.Lock()
     done = [0]
@@ -254,7 +283,7 @@ def oracle_c5_parallel(w, budget_s, R, threads=None):
         t.join()
     dt = time.perf_counter() - t0
     return (done[0] * w.n / dt,
-            f"1 DAG build + {done[0]} of {R} replicas of c2 on {threads} threads (perturbation seed {workloads.C5_SEED})",
+            f"prebuilt DAG, {done[0]} of {R} replicas of c2 on {threads} threads (perturbation seed {workloads.C5_SEED})",
             dt, threads)
 
 
@@ -265,7 +294,7 @@ def run_reference(args):
     import oracle
     oracle.build()
     cfg = args.config
-    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc", "c2n4") else cfg)
+    w = base_workload(cfg)
     per_step_budget = 3.0 if cfg != "c4" else 10.0
     times, tasks = [], []
     cores = 1
@@ -282,7 +311,7 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC_SIM if cfg in ("c5sim", "c5loc") else METRIC, "value": value, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
             "scaling": "none", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": CONFIG_TEXT[cfg], "name": cfg,
+            "config": {"workload": workload_text(cfg), "name": cfg,
                        "step": "bounded sample: " + sample},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -336,6 +365,16 @@ def measured_traffic(kernel, cfg):
         return None, None
 
 
+def base_workload(cfg):
+    """The DAG + base durations a config runs on (replica configs: the c2 DAG)."""
+    return workloads.config("c2" if cfg in REPLICA_CFGS + ("c2push", "c2n4") else cfg)
+
+
+def workload_text(cfg):
+    """config.workload, identical in both arms (the driver compares them)."""
+    return CONFIG_TEXT[cfg]
+
+
 def run_ours(args):
     import paper_conf_ipps_tayebbfg24_b200 as mp
     from paper_conf_ipps_tayebbfg24_b200 import dist as mpd
@@ -351,7 +390,8 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=dev)
     cfg = args.config
     sim = cfg in ("c5sim", "c5loc")
-    w = workloads.config("c2" if cfg in ("c5", "c5sim", "c5loc", "c2push", "c2n4") else cfg)
+    rep = cfg in REPLICA_CFGS
+    w = base_workload(cfg)
     A = w.n_arch
     n = w.n
     src_h = torch.from_numpy(w.src).pin_memory()
@@ -363,8 +403,9 @@ def run_ours(args):
     dag = mp.build_dag(n, src_d, dst_d)
     E = dag.n_edges
     stream = torch.cuda.current_stream()
+    gather_ev = []          # (start, end) events around the allgather of each timed step
 
-    if cfg in ("c5", "c5sim", "c5loc"):
+    if rep:
         # replicas are independent problems keyed by their GLOBAL id (world-size invariant results)
         R = args.replicas * world if args.scaling == "weak" else args.replicas
         r0, cnt = mpd.shard_range(R, world, rank)
@@ -383,9 +424,11 @@ def run_ours(args):
         gathered = torch.empty((world * slots, rb), dtype=torch.uint8, device=dev)
         result_h = torch.empty((world * slots, rb), dtype=torch.uint8).pin_memory()
         tasks_per_step = R * n
+        units_per_step = R
 
-        def step():
-            mp.dag_rebuild(dag, n, src_d, dst_d)
+        def step(rebuild=False, gev=None):
+            if rebuild:
+                mp.dag_rebuild(dag, n, src_d, dst_d)
             mp.replicas_run(dag, dur_d, workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out=out)
             if sim:
                 mp.simulate(dag, dur_d, workers, workloads.C5_SEED, workloads.C5_SIGMA, r0, cnt, out["qtask"],
@@ -393,13 +436,20 @@ def run_ours(args):
             mpd.pack_records(out["cp"], out["summary"], cnt, A, slots, out=local_rec,
                              extra=sim_out["stats"] if sim else None)
             if world > 1:
+                if gev is not None:
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
                 mpd.gather_records(local_rec, out=gathered)
+                if gev is not None:
+                    e1.record(stream)
+                    gev.append((e0, e1))
             else:
                 gathered.copy_(local_rec)
             return gathered
     elif cfg == "c2push":
         R, cnt = 1, 1
         tasks_per_step = n
+        units_per_step = 1
         full = mp.score_and_queue(dag, dur_d, w.workers)            # whole-DAG scores + ALL-mode queues
         flags_d = full["flags"]
         qptr_all, qtask_all = full["qptr"], full["qtask"]
@@ -412,7 +462,9 @@ def run_ours(args):
         qhost = torch.empty(A + 1, dtype=torch.int64).pin_memory()
         result_h = torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8).pin_memory()
 
-        def step():
+        def step(rebuild=False, gev=None):
+            if rebuild:
+                mp.dag_rebuild(dag, n, src_d, dst_d)
             mp.ready_init(dag, rem)
             done.zero_()
             mp.queues_push_all(dag, qptr_all, qtask_all, flags_d, dur_d, empty, rem, done, out=bufs[0])
@@ -428,6 +480,7 @@ def run_ours(args):
     elif cfg == "c2n4":
         R, cnt = 1, 1
         tasks_per_step = n
+        units_per_step = 1
         done_h = np.zeros(n, np.uint8)
         done_h[dag.arrays()["level_order"].cpu().numpy()[: n // 2]] = 1
         done_d = torch.from_numpy(done_h).to(dev)
@@ -444,8 +497,9 @@ def run_ours(args):
                         summary=torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=dev)))
         result_h = torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8).pin_memory()
 
-        def step():
-            mp.dag_rebuild(dag, n, src_d, dst_d)
+        def step(rebuild=False, gev=None):
+            if rebuild:
+                mp.dag_rebuild(dag, n, src_d, dst_d)
             bl, cp = mp.bottom_level_w(dag, dur_d, w.workers, mp.MP_WEIGHT_MEAN, out=o["bl"])
             gain, hd, flags = mp.affinity_prefix(dag, dur_d, w.workers, None, out=o["aff"])
             mp.nod_remaining(dag, dur_d, w.workers, done_d, out=o["nod"])
@@ -456,11 +510,12 @@ def run_ours(args):
         R, cnt = 1, 1
         outs = {}
         tasks_per_step = n
+        units_per_step = 1
         result_h = torch.empty(A * mp.SUMMARY_BYTES + 4, dtype=torch.uint8).pin_memory()
 
         cur = {"dag": dag, "src": src_d, "dst": dst_d}   # the depth probe swaps in its own DAG
 
-        def step(rebuild=True):
+        def step(rebuild=False, gev=None):
             dag_ = cur["dag"]
             if rebuild:
                 mp.dag_rebuild(dag_, n, cur["src"], cur["dst"])
@@ -489,6 +544,29 @@ def run_ours(args):
         if world > 1:
             dist.barrier()
 
+    def timed(fn, K, sync_ranks=True):
+        """K calls of fn, each bracketed by CUDA events on the launch stream, L2 flushed
+        before each (outside the events); barrier + synchronize on both sides."""
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+        torch.cuda.synchronize()
+        if sync_ranks:
+            barrier()
+        for i in range(K):
+            flush.zero_()
+            evs[i][0].record(stream)
+            fn()
+            evs[i][1].record(stream)
+        torch.cuda.synchronize()
+        if sync_ranks:
+            barrier()
+        return [a.elapsed_time(b) for a, b in evs]
+
+    def max_over_ranks(x):
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
     # ---- warm-up ----
     for _ in range(max(args.warmup, 0)):
         step()
@@ -496,55 +574,46 @@ def run_ours(args):
     torch.cuda.synchronize()
     barrier()
 
-    # ---- timed region (device time per step, L2 flushed between steps) ----
+    # ---- headline timed region: K steps, libmp profiling OFF ----
     clocks = Clocks(dev)
     clocks.start()
+    l0 = mp.launch_count()
+    step_ms = timed(lambda: step(gev=gather_ev), args.steps)
+    launches = mp.launch_count() - l0
+    ck = clocks.stop()
+    ms_per_step = max_over_ranks(sum(step_ms)) / args.steps
+    value = tasks_per_step / (ms_per_step * 1e-3)
+    allgather = None
+    if world > 1:
+        g_ms = max_over_ranks(sum(a.elapsed_time(b) for a, b in gather_ev)) / args.steps
+        allgather = {"ms_per_step": g_ms, "bytes_per_rank": int(local_rec.numel()),
+                     "bytes_gathered": int(gathered.numel()), "share_of_step": g_ms / ms_per_step,
+                     "how": "CUDA events around all_gather_into_tensor inside the timed steps, max over ranks"}
+
+    # ---- ingest (mp_dag_rebuild, a1+a2) timed on its own, then build + score ----
+    build_ms = max_over_ranks(sum(timed(lambda: mp.dag_rebuild(dag, n, src_d, dst_d), args.steps))) / args.steps
+    mp.check(dag)
+
+    # ---- profiled pass (per-kernel CUDA events inside libmp), same steps ----
     mp.prof_reset()
     mp.prof_enable(True)
-    l0 = mp.launch_count()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    torch.cuda.synchronize()
-    barrier()
-    for i in range(args.steps):
-        flush.zero_()
-        evs[i][0].record(stream)
-        step()
-        evs[i][1].record(stream)
-    torch.cuda.synchronize()
-    barrier()
-    launches = mp.launch_count() - l0
+    prof_ms = sum(timed(step, args.steps, sync_ranks=False)) / args.steps
     mp.prof_enable(False)
-    ck = clocks.stop()
-    step_ms = [a.elapsed_time(b) for a, b in evs]
-    tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
-    ms_per_step = float(tot.item()) / args.steps
-    value = tasks_per_step / (ms_per_step * 1e-3)
     prof = {k: mp.prof_query(k) for k in mp.prof_names()}
 
-    # ---- single DAGs: the score + queue path alone on the prebuilt DAG (t covers
-    #      bottom_level -> affinity -> score -> build_queues; the ingest is reported separately) ----
+    # ---- single DAGs: depth probe (SURVEY §8(d) two-term roofline) ----
     score_only = None
-    if cfg in ("c1", "c2", "c3", "c4", "lu64"):
-        sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-        torch.cuda.synchronize()
-        for i in range(args.steps):
-            flush.zero_()
-            sev[i][0].record(stream)
-            step(rebuild=False)
-            sev[i][1].record(stream)
-        torch.cuda.synchronize()
-        sc_ms = sum(a.elapsed_time(b) for a, b in sev) / args.steps
+    if cfg in SINGLE_CFGS:
         Q = int(np.isfinite(w.dur).sum())      # queue entries (every arch enabled by the workers)
         b_sc = 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 4 * n * A + 4 * Q
-        score_only = {"ms_per_dag": sc_ms, "tasks_per_s": n / (sc_ms * 1e-3), "build_ms": ms_per_step - sc_ms,
+        score_only = {"ms_per_dag": ms_per_step, "tasks_per_s": value, "build_ms": build_ms,
+                      "build_plus_score_ms": build_ms + ms_per_step,
                       "alg_bytes": b_sc, "hbm_frac_of_peak": None,
-                      "note": "bottom_level + affinity + score + build_queues on the prebuilt DAG, L2 flushed"}
-        # Depth probe (SURVEY §8(d) two-term roofline): the same calls on a DAG with the same n
-        # and the same depth L but no fan-in/fan-out -- a chain of L tasks plus n - L isolated
-        # tasks -- so the same kernels run; its time is the per-level latency floor plus the
-        # per-task (not per-edge) work.  probe / actual says how much of the time depth explains.
+                      "note": "bottom_level + affinity + score + build_queues on the prebuilt DAG, L2 flushed "
+                              "(= the headline value); the ingest is build_ms"}
+        # The same calls on a DAG with the same n and the same depth L but no fan-in/fan-out
+        # -- a chain of L tasks plus n - L isolated tasks -- so the same kernels run; its time
+        # is the per-level latency floor plus the per-task (not per-edge) work.
         Lv = dag.n_levels
         if not args.no_probe and Lv > 1:
             src_p = torch.arange(Lv - 1, dtype=torch.int32, device=dev)
@@ -553,19 +622,10 @@ def run_ours(args):
             assert dagp.n_levels == Lv
             cur.update(dag=dagp, src=src_p, dst=dst_p)
             pt = {}
-            for rb in (True, False):
+            for rb_ in (True, False):
                 for _ in range(2):
-                    step(rebuild=rb)
-                pev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-                       for _ in range(args.steps)]
-                torch.cuda.synchronize()
-                for i in range(args.steps):
-                    flush.zero_()
-                    pev[i][0].record(stream)
-                    step(rebuild=rb)
-                    pev[i][1].record(stream)
-                torch.cuda.synchronize()
-                pt[rb] = sum(a.elapsed_time(b) for a, b in pev) / args.steps
+                    step(rebuild=rb_)
+                pt[rb_] = sum(timed(lambda: step(rebuild=rb_), args.steps, sync_ranks=False)) / args.steps
             mp.check(dagp)
             cur.update(dag=dag, src=src_d, dst=dst_d)
             dagp.free()
@@ -573,7 +633,7 @@ def run_ours(args):
                 "dag": f"chain of L = {Lv} tasks + {n - Lv} isolated tasks (same n, same depth, E = {Lv - 1})",
                 "ms_score_only": pt[False], "ms_with_ingest": pt[True],
                 "t_level_us_score": pt[False] / Lv * 1e3, "t_level_us_with_ingest": pt[True] / Lv * 1e3,
-                "frac_of_score_only": pt[False] / sc_ms, "frac_of_step": pt[True] / ms_per_step,
+                "frac_of_score_only": pt[False] / ms_per_step, "frac_of_build_plus_score": pt[True] / (build_ms + ms_per_step),
                 "note": "two-term roofline: max(bytes floor, depth probe); the probe is a measured lower "
                         "bound for this n and L through the same calls"}
     step_dev_ms = {k: v[0] / args.steps for k, v in prof.items() if v[1] > 0}
@@ -581,31 +641,26 @@ def run_ours(args):
     dom_ms, dom_launches = prof[dom]
     mp.check(dag)
 
-    # ---- e2e: host buffers in, records out, through the public API ----
+    # ---- e2e: host buffers in, results out, through the public API (ingest included) ----
     e2e = None
     if not args.no_e2e:
-        eev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-        torch.cuda.synchronize()
-        barrier()
-        for i in range(args.steps):
-            flush.zero_()
-            eev[i][0].record(stream)
+        res_box = []
+
+        def e2e_step():
             src_d.copy_(src_h, non_blocking=True)
             dst_d.copy_(dst_h, non_blocking=True)
             dur_d.copy_(dur_h, non_blocking=True)
-            res = step()
+            res = step(rebuild=True)
             result_h[: res.numel()].view(-1).copy_(res.view(-1), non_blocking=True)
-            eev[i][1].record(stream)
-        torch.cuda.synchronize()
-        barrier()
-        et = torch.tensor([sum(a.elapsed_time(b) for a, b in eev)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(et, op=dist.ReduceOp.MAX)
-        e2e_ms = float(et.item()) / args.steps
+            res_box[:] = [res]
+
+        e2e_ms = max_over_ranks(sum(timed(e2e_step, args.steps))) / args.steps
+        res = res_box[0]
         h2d = src_h.numel() * 4 + dst_h.numel() * 4 + dur_h.numel() * 4
         d2h = res.numel() * res.element_size()
         e2e = {"value": tasks_per_step / (e2e_ms * 1e-3), "unit": UNIT, "ms_per_step": e2e_ms,
-               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "note": "per step: H2D of edges + durations, mp_dag_rebuild, the step, D2H of the results"}
 
     if rank != 0:
         if world > 1:
@@ -619,7 +674,7 @@ def run_ours(args):
     except Exception:
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
     ctx = dict(n=n, E=E, A=A)
-    if cfg in ("c5", "c5sim", "c5loc"):
+    if rep:
         ctx["replicas_per_launch"] = cnt      # one k_rep2_bl / k_rep2_sort launch covers the rank's block
         ctx["sort_entries_per_launch"] = cnt * A * n
     else:
@@ -633,13 +688,15 @@ def run_ours(args):
             **({"bound_note": "latency: each warp runs one instance's sequential event chain"} if dom.endswith("k_sim") else {}), "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": (achieved / peak) if achieved else None, "traffic": traffic, "traffic_source": traffic_src,
             "alg_bytes_per_launch": alg, "avg_launch_ms": avg_ms, "launches": dom_launches,
-            "share_of_step": (dom_ms / args.steps) / ms_per_step, "peak_source": peak_src,
+            "share_of_step": (dom_ms / args.steps) / prof_ms, "peak_source": peak_src,
+            "timing": "per-kernel CUDA events (libmp mp_prof) in a second pass of the same steps; "
+                      f"that pass: {prof_ms:.4f} ms per step vs {ms_per_step:.4f} ms unprofiled",
             "per_kernel_ms_per_step": {k: round(v, 4) for k, v in sorted(step_dev_ms.items(), key=lambda x: -x[1])}}
     # whole-step algorithmic bytes (SURVEY §8(d) B_alg) as context
-    if cfg in ("c5", "c5sim", "c5loc"):
-        b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + args.replicas * 4 * n * A / world  # CSR + dur + queues out
+    if rep:
+        b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + cnt * 4 * n * A   # CSR + dur + this rank's queues out
     else:
-        b_alg = 4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 4 * n * A + 4 * n * A
+        b_alg = score_only["alg_bytes"] if score_only else (4 * (n + 1) + 4 * E + 4 * n * A + 4 * n + 8 * n * A)
     roof["step_alg_bytes_per_gpu"] = b_alg
     roof["step_hbm_frac"] = b_alg / (ms_per_step * 1e-3) / 1e9 / peak
     if score_only is not None:
@@ -663,39 +720,33 @@ def run_ours(args):
             v, sample, dt = oracle_sample(cfg, w, args.cpu_budget_s, args.replicas)
             cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, "seconds": round(dt, 2)}
 
-    rep = cfg in ("c5", "c5sim")
-    line = {"metric": METRIC_SIM if cfg in ("c5sim", "c5loc") else METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+    step_text = {"c5": "mp_replicas_run (this rank's replica block) + allgather(68-byte records)",
+                 "c5sim": "mp_replicas_run + mp_simulate + allgather(records + sim stats)",
+                 "c5loc": "mp_replicas_run + mp_simulate (LS_SDH^2 pick) + allgather(records + sim stats)",
+                 "c2push": "mp_ready_init + mp_queues_push_all per completion batch (scores and ALL-mode "
+                           "queues precomputed)",
+                 "c2n4": "bottom_level_w(mean) + affinity_prefix + nod_remaining + score + build_queues"}.get(
+        cfg, "bottom_level + affinity + score + build_queues on the prebuilt DAG")
+    line = {"metric": METRIC_SIM if sim else METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
             "scaling": args.scaling if rep else "none", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic",
-            "config": {"workload": (CONFIG_TEXT[cfg] if not rep else
-                                    f"{R} duration-perturbed replicas of the 64x64 Cholesky DAG ({cnt} per GPU, "
-                                    f"{args.scaling} scaling; BASELINE config 5 = 4096 in total = --scaling strong)"
-                                    + ("; each scheduled by the N2 PUSH/POP simulation with eviction on "
-                                       f"{SIM_WORKERS[0]} CPU + {SIM_WORKERS[1]} GPU workers" if sim else "")
-                                    + ("; POP with the LS_SDH^2 locality pick (n = 10, eps = 0.8) on 960x960 tiles, "
-                                       "transfers at 2^-24 ms/byte" if cfg == "c5loc" else "")),
-                       "name": cfg, "tasks_per_dag": n, "edges": E,
+            "config": {"workload": workload_text(cfg), "name": cfg, "tasks_per_dag": n, "edges": E,
                        "levels": dag.n_levels, "archs": A,
                        "replicas": R if rep else 1, "replicas_per_gpu": cnt,
-                       "ms_per_dag": ms_per_step / (R if rep else 1) * world if rep else ms_per_step,
+                       "replica_sharding": (f"{args.scaling} scaling: {R} replicas in total, {cnt} on rank 0; "
+                                            "BASELINE config 5 = 4096 in total = --scaling strong") if rep else None,
                        "l2": f"flushed between timed steps ({L2_FLUSH_BYTES >> 20} MiB write)",
                        "queues": "materialised in HBM for every replica" if rep else "materialised",
-                       "step": ("mp_dag_rebuild + mp_replicas_run + allgather(records)" if cfg == "c5" else
-                                "mp_dag_rebuild + mp_replicas_run + mp_simulate + allgather(records + sim stats)"
-                                if sim else
-                                "mp_ready_init + mp_queues_push_all per completion batch (scores and ALL-mode queues "
-                                "precomputed)"
-                                if cfg == "c2push" else
-                                "mp_dag_rebuild + bottom_level_w(mean) + affinity_prefix + nod_remaining + score + "
-                                "build_queues" if cfg == "c2n4" else
-                                "mp_dag_rebuild + bottom_level + affinity + score + build_queues"),
-                       "parallelism": f"replica shards x{world}" if rep else "single DAG",
+                       "step": step_text,
+                       "parallelism": f"replica shards x{world}" if rep else "single DAG (replicas only)",
                        **({"sim_workers": list(SIM_WORKERS), "max_tries": SIM_MAX_TRIES, "eviction": True}
                           if sim else {}),
                        **({"locality": {"top_n": LOC["top_n"], "eps": LOC["eps"],
                                         "xfer_ms_per_byte": LOC["xfer_ms_per_byte"]}} if cfg == "c5loc" else {})},
-            "ms_per_dag": ms_per_step / (R / world) if rep else ms_per_step,
+            "ms_per_dag": ms_per_step * world / R if rep else ms_per_step,
+            "build_ms": build_ms, "build_plus_step_ms": build_ms + ms_per_step,
+            **({"allgather": allgather} if allgather else {}),
             "roofline": roof, **({"score_only": score_only} if score_only else {}),
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
             "gpu_launches_per_step": launches / args.steps, "clocks": ck,
@@ -705,10 +756,23 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+def spawn_ranks(args):
+    """--gpus N > 1 outside torchrun: re-launch this script as N ranks (one per GPU)."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
+    elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args))
     else:
         run_ours(args)
 

@@ -13,6 +13,7 @@ Configs (BASELINE.json order):
   c3  tiled QR 128x128 (split diagonal), 3 resource types        (A=3)
   c4  sparse-QR-like tree (G=42) U FMM octree (H=8, 2^19 parts)  (A=2)
   c5  replicas of c2 (R=4096, sigma=1/8, seed 20240311)
+  c4fmm  c4's FMM octree part alone (TBFMM-shaped)
 """
 from __future__ import annotations
 
@@ -159,6 +160,8 @@ def config(name: str) -> Workload:
         w = qr(128, split_diag=True)
     elif name == "c4":
         w = union(sparse_tree(42, 64, 32), fmm_tree(8, 1 << 19, 7), "c4")
+    elif name == "c4fmm":       # c4's FMM part alone (the 13-level single-DAG case)
+        w = fmm_tree(8, 1 << 19, 7)
     elif name == "lu64":
         w = lu(64)
     else:
