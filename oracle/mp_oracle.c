@@ -441,7 +441,8 @@ int or_score(int32_t n, int32_t A, int32_t kind, const float* crit, const float*
 /* summaries = Alg. 1 counters.  READY mode (done != NULL): only tasks     */
 /* t with !done(t) and all predecessors done (P:l.91, reading c18).        */
 /* --------------------------------------------------------------------- */
-static const uint64_t* g_sort_key;   /* qsort context (single-threaded oracle) */
+static _Thread_local const uint64_t* g_sort_key;   /* qsort context, per thread (tests and the
+                                                    cpu baseline call the oracle from threads) */
 static int cmp_entry(const void* pa, const void* pb) {
     int32_t a = *(const int32_t*)pa, b = *(const int32_t*)pb;
     uint64_t ka = g_sort_key[a], kb = g_sort_key[b];

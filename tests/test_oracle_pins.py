@@ -593,3 +593,17 @@ def test_error_paths():
     assert d0.n_levels == 0 and d0.n_edges == 0
     d1 = oracle.build_dag(5, [], [])
     assert d1.n_levels == 1
+
+
+def test_oracle_replicas_thread_safe():
+    """The GPU parity test and the cpu baseline run oracle.replica from threads: the
+    results must equal the sequential ones (no shared mutable state in the oracle)."""
+    from concurrent.futures import ThreadPoolExecutor
+    w = workloads.config("c2")
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    args = (workloads.C5_SEED, workloads.C5_SIGMA)
+    seq = [oracle.replica(od, w.dur, w.workers, *args, r) for r in range(16)]
+    with ThreadPoolExecutor(8) as ex:
+        par = list(ex.map(lambda r: oracle.replica(od, w.dur, w.workers, *args, r), range(16)))
+    for a, b in zip(seq, par):
+        assert a[0] == b[0] and a[1].tobytes() == b[1].tobytes() and np.array_equal(a[2], b[2])
