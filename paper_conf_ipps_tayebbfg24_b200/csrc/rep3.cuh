@@ -83,7 +83,7 @@ struct R4Args {
 // shared-memory layout (identical in both CTAs, so peer addresses map 1:1)
 struct R4Layout {
     uint32_t h, hpad, ew;
-    size_t o_ds, o_ps, o_cnt, o_coff, o_clog, o_e0, o_e1, o_list, o_sc, o_um, o_uo, o_crit, o_rb, bytes;
+    size_t o_ds, o_ps, o_cnt, o_coff, o_clog, o_e0, o_e1, o_list, o_sc, o_um, o_uo, o_crit, o_mpos, o_rb, bytes;
 };
 __host__ __device__ inline R4Layout r4_layout(int32_t n) {
     R4Layout L;
@@ -100,6 +100,7 @@ __host__ __device__ inline R4Layout r4_layout(int32_t n) {
     L.o_um = o;   o += (size_t)L.ew * 4;           // P5: members (either queue) per 32 positions
     L.o_uo = o;   o += (size_t)L.ew * 4;           // P5: exclusive prefix of their counts
     L.o_crit = o; o += (size_t)R4_LIST * 4;         // P5: critc of every member, in position order
+    L.o_mpos = o; o += (size_t)R4_LIST * 2;         // P5: their local positions
     L.o_rb = o;   o += (size_t)(R4_MAXR + 1) * 4;  // P3: round bounds
     L.o_ps = o;   o += (size_t)L.hpad * 2;           // task id in position order
     L.o_coff = o; o += (size_t)R4_NC * 2;
@@ -240,10 +241,71 @@ __global__ void __launch_bounds__(R4_THREADS, 1) k_rep3_sort(R4Args a) {
 #ifdef MP_PHASES
     long long k3_t = 0;
 #endif
+    // D(t) of replica r (a10: both perturbed durations, hashed once per pass)
+    auto D_task = [&](uint64_t cbase, int32_t t) -> uint32_t {
+        const float2 bb = __ldg(reinterpret_cast<const float2*>(a.base) + t);
+        const uint64_t xs = cbase + (uint64_t)(uint32_t)t * golden2;
+        bool dummy = false;
+        const float x0 = canon_dur(perturb_x(bb.x, xs, a.sigma), dummy);
+        const float x1 = canon_dur(perturb_x(bb.y, xs + SPLITMIX_GOLDEN, a.sigma), dummy);
+        return r4_D(x0, x1, a.emask);
+    };
+    auto cbase_of = [&](uint64_t r) -> uint64_t {
+        return a.seed + ((uint64_t)r * (uint64_t)n * 2u + 1u) * SPLITMIX_GOLDEN;
+    };
+    // ---- the launch's fine-bin geometry, built once from a reference replica (the call's
+    //      first) and shared by every replica (their D follow the same distribution):
+    //      every coarse bin of the range gets >= 1 fine bin (another replica may have keys
+    //      where the reference has none), the rest proportionally to the reference's
+    //      coarse counts -> fine bins hold ~3 entries ----
+    {
+        for (int32_t i = threadIdx.x; i < R4_NC; i += R4_THREADS) cnt[i] = 0u;
+        __syncthreads();
+        const uint64_t cb0 = cbase_of((uint64_t)a.r0);
+        for (int32_t t = own0 + threadIdx.x; t < own1; t += R4_THREADS)
+            atomicAdd(&cnt[r4_coarse(g, D_task(cb0, t))], 1u);
+        cl.sync();
+        const uint32_t ncb = (uint32_t)(((uint64_t)(g.hi - g.lo) >> g.cs) + 1);
+        constexpr int CPER = R4_NC / R4_THREADS;   // 4
+        uint32_t c[CPER], tc = 0;
+#pragma unroll
+        for (int j = 0; j < CPER; j++) {
+            const uint32_t b = threadIdx.x * CPER + j;
+            c[j] = cnt[b] + cntP[b];
+            tc += c[j];
+        }
+        uint32_t TOT;
+        r3_scan(tc, sc, TOT);
+        const uint64_t Fn = (uint64_t)R4_NF - ncb, Fd = TOT > 0 ? TOT : 1u;
+        uint32_t m[CPER], sm = 0;
+#pragma unroll
+        for (int j = 0; j < CPER; j++) {
+            const uint32_t b = threadIdx.x * CPER + j;
+            uint32_t v = 0;
+            if (b < ncb) {
+                v = (uint32_t)min(((uint64_t)c[j] * Fn + Fd - 1) / Fd, (uint64_t)255);
+                if (g.cs < 8) v = min(v, 1u << g.cs);
+                v = max(v, 1u);
+            }
+            m[j] = v;
+            sm += v;
+        }
+        uint32_t ftot;
+        uint32_t e = r3_scan(sm, sc, ftot);
+#pragma unroll
+        for (int j = 0; j < CPER; j++) {
+            const uint32_t b = threadIdx.x * CPER + j;
+            coff[b] = (uint16_t)e;
+            clog[b] = (uint8_t)m[j];
+            e += m[j];
+        }
+        cl.sync();   // the peer is done reading cnt
+    }
 
     uint32_t* um = reinterpret_cast<uint32_t*>(r4s + L.o_um);
     uint32_t* uo = reinterpret_cast<uint32_t*>(r4s + L.o_uo);
     uint32_t* mcrit = reinterpret_cast<uint32_t*>(r4s + L.o_crit);
+    uint16_t* mpos = reinterpret_cast<uint16_t*>(r4s + L.o_mpos);
     int32_t* rb = reinterpret_cast<int32_t*>(r4s + L.o_rb);
     __shared__ uint32_t s_nmem, s_bpair;
 
@@ -261,78 +323,25 @@ __global__ void __launch_bounds__(R4_THREADS, 1) k_rep3_sort(R4Args a) {
         if (rl >= a.R) break;
         K3_PHASE(0);
         const int64_t r = a.r0 + rl;
-        // ---- P1: D(t) of the own tasks (both perturbed durations hashed once, a10) into
-        //      Ds (id order for now), coarse histogram; clear the e-bits ----
-        for (int32_t i = threadIdx.x; i < R4_NC; i += R4_THREADS) cnt[i] = 0u;
-        for (int32_t i = threadIdx.x; i < (int32_t)L.ew; i += R4_THREADS) { e0[i] = 0u; e1[i] = 0u; }
+        // ---- P1: D(t) of the own tasks into Ds (id order for now) and the fine histogram
+        //      (16-bit counters in pairs) ----
+        for (int32_t i = threadIdx.x; i < R4_NF / 2; i += R4_THREADS) cnt[i] = 0u;
         if (threadIdx.x == 0) { s_nbig = 0u; s_nmem = 0u; s_bpair = 0u; }
         __syncthreads();
         {
-            const uint64_t cbase = a.seed + ((uint64_t)r * (uint64_t)n * 2u + 1u) * SPLITMIX_GOLDEN;
+            const uint64_t cbase = cbase_of((uint64_t)r);
             bool outside = false;
             for (int32_t t = own0 + threadIdx.x; t < own1; t += R4_THREADS) {
-                const float2 bb = __ldg(reinterpret_cast<const float2*>(a.base) + t);
-                const uint64_t xs = cbase + (uint64_t)(uint32_t)t * golden2;
-                bool dummy = false;
-                const float x0 = canon_dur(perturb_x(bb.x, xs, a.sigma), dummy);
-                const float x1 = canon_dur(perturb_x(bb.y, xs + SPLITMIX_GOLDEN, a.sigma), dummy);
-                const uint32_t D = r4_D(x0, x1, a.emask);
+                const uint32_t D = D_task(cbase, t);
                 Ds[t - own0] = D;
                 outside |= D < g.lo || D > g.hi;
-                atomicAdd(&cnt[r4_coarse(g, D)], 1u);
+                const uint32_t f = r4_fine(g, coff, clog, D);
+                atomicAdd(&cnt[f >> 1], 1u << ((f & 1u) * 16u));
             }
             if (__any_sync(0xffffffffu, outside) && lane == 0) atomicOr(flag0, 1u);
         }
         cl.sync();                                                          // S1
         K3_PHASE(1);
-        // ---- G: proportional sub-bin geometry (both CTAs, same result) ----
-        {
-            constexpr int CPER = R4_NC / R4_THREADS;   // 4
-            uint32_t c[CPER], ne = 0, tc = 0;
-#pragma unroll
-            for (int j = 0; j < CPER; j++) {
-                const uint32_t b = threadIdx.x * CPER + j;
-                c[j] = cnt[b] + cntP[b];
-                ne += c[j] > 0u ? 1u : 0u;
-                tc += c[j];
-            }
-            uint32_t NE, TOT;
-            r3_scan(ne, sc, NE);
-            r3_scan(tc, sc, TOT);
-            const uint64_t Fn = (uint64_t)R4_NF - NE, Fd = TOT > 0 ? TOT : 1u;
-            uint32_t m[CPER], sm = 0;
-#pragma unroll
-            for (int j = 0; j < CPER; j++) {
-                uint32_t v = 0;
-                if (c[j] > 0u) {
-                    v = (uint32_t)min(((uint64_t)c[j] * Fn + Fd - 1) / Fd, (uint64_t)255);
-                    if (g.cs < 8) v = min(v, 1u << g.cs);
-                    v = max(v, 1u);
-                }
-                m[j] = v;
-                sm += v;
-            }
-            uint32_t ftot;
-            uint32_t e = r3_scan(sm, sc, ftot);
-#pragma unroll
-            for (int j = 0; j < CPER; j++) {
-                const uint32_t b = threadIdx.x * CPER + j;
-                coff[b] = (uint16_t)e;
-                clog[b] = (uint8_t)m[j];
-                e += m[j];
-            }
-        }
-        cl.sync();                                                          // S2 (peer done reading cnt)
-        K3_PHASE(2);
-        // ---- P1b: fine histogram (16-bit counters in pairs) ----
-        for (int32_t i = threadIdx.x; i < R4_NF / 2; i += R4_THREADS) cnt[i] = 0u;
-        __syncthreads();
-        for (int32_t i = threadIdx.x; i < hk; i += R4_THREADS) {
-            const uint32_t f = r4_fine(g, coff, clog, Ds[i]);
-            atomicAdd(&cnt[f >> 1], 1u << ((f & 1u) * 16u));
-        }
-        cl.sync();                                                          // S3
-        K3_PHASE(3);
         // ---- S: global starts; own cursors = start + (CTA 1: CTA 0's count) ----
         uint32_t Dr[R4_PER];   // P2: the own D values leave Ds (the peer scatters into it)
         {
@@ -368,6 +377,7 @@ __global__ void __launch_bounds__(R4_THREADS, 1) k_rep3_sort(R4Args a) {
                 Dr[j] = i < hk ? Ds[i] : 0u;
             }
             cl.sync();                                                      // S4 (peer done reading cnt; own D in registers)
+            K3_PHASE(2);
 #pragma unroll
             for (int j = 0; j < WPER; j++) cnt[threadIdx.x * WPER + j] = cur[j];
         }
@@ -569,10 +579,25 @@ __global__ void __launch_bounds__(R4_THREADS, 1) k_rep3_sort(R4Args a) {
                 while (m) {
                     const int b = __ffs(m) - 1;
                     m &= m - 1u;
+                    mpos[idx] = (uint16_t)(wq * 32 + b);
                     mcrit[idx++] = critc_of(Ps[wq * 32 + b]);
                 }
             }
             __syncthreads();
+            // non-members: straight to both queues (coalesced, no divergence)
+            for (int32_t lp = threadIdx.x; lp < hk; lp += R4_THREADS) {
+                if ((um[lp >> 5] >> (lp & 31)) & 1u) continue;
+                const int32_t p = own0 + lp;
+                const uint32_t t = Ps[lp];
+                if (p < cG) {
+                    if (p == 0) *head1p = t;
+                    if (q1) __stcs(q1 + p, (int32_t)t);
+                }
+                if (p >= n1only) {
+                    if (p == n - 1) *head0p = t;
+                    if (q0) __stcs(q0 + (n - 1 - p), (int32_t)t);
+                }
+            }
             // critc of the member at position p (own and listed; else from HBM)
             auto crit_at = [&](int32_t p) -> uint32_t {
                 if (mfit && p >= own0 && p < own1) {
@@ -581,13 +606,16 @@ __global__ void __launch_bounds__(R4_THREADS, 1) k_rep3_sort(R4Args a) {
                 }
                 return critc_of(*Pp(p));
             };
+            // members: one thread each, rank inside their runs
             bool longrun = false;
-            for (int32_t lp = threadIdx.x; lp < hk; lp += R4_THREADS) {
+            const int32_t nmem = mfit ? (int32_t)mtot : hk;
+            for (int32_t mi = threadIdx.x; mi < nmem; mi += R4_THREADS) {
+                const int32_t lp = mfit ? (int32_t)mpos[mi] : mi;
+                if (!mfit && !((um[lp >> 5] >> (lp & 31)) & 1u)) continue;
                 const int32_t p = own0 + lp;
                 const uint32_t t = Ps[lp];
-                const bool mem = (um[lp >> 5] >> (lp & 31)) & 1u;
                 int32_t pos1 = p, pos0 = n - 1 - p;
-                if (mem) {
+                {
                     if (member1(p)) {   // queue 1: runs of equal gain_1 by (critc, id)
                         int32_t lo = p, hi = p;
                         while (lo > 0 && p - lo <= R4_RUN && ebit(1, lo - 1)) lo--;

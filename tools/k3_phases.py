@@ -25,7 +25,7 @@ for it in range(3):
     mp.replicas_run(dag, dur, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, 0, R)
     torch.cuda.synchronize()
 L.mp_debug_k2_phases(buf.ctypes.data, 1)
-names = {17: "P1 hash+coarse", 18: "G geometry", 19: "P1b fine hist", 20: "S scan + P2 scatter", 21: "P3 bin sort", 22: "P3b same-gain bits", 23: "P5 emission"}
+names = {17: "P1 hash+fine hist", 18: "S scan", 20: "P2 scatter", 21: "P3 bin sort", 22: "P3b same-gain bits", 23: "P5 emission"}
 
 tot = buf[16:].sum()
 for i in sorted(names):  # cycles of CTA 0 of each cluster
