@@ -72,9 +72,6 @@ struct Rep2Args {
     int32_t* qtask;              // [R][n*A] or null
     mp_queue_summary* sum;       // [R][A]
     uint32_t* ticket;
-    int32_t* fb_list;            // [R] K3's fallback list (two archs)
-    const int32_t* rlist;        // K2 list mode: process replicas rlist[0 .. *rlist_n) only
-    const uint32_t* rlist_n;
 };
 
 template <int A>
@@ -1063,8 +1060,6 @@ MP_INLINE bool r2_same_q(float xa, float xb, float den, float lim) {
 template <int A>
 __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     extern __shared__ __align__(16) unsigned char r3s[];
-    const uint32_t rtotal = a.rlist ? __ldcg(a.rlist_n) : (uint32_t)a.R;
-    if (rtotal == 0u) return;                  // list mode with nothing left to do
     R3Smem S;
     S.starts = reinterpret_cast<uint32_t*>(r3s);
     S.bkraw = r3s + (size_t)(R3_NF + 64) * 4;
@@ -1140,10 +1135,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             s_max[threadIdx.x] = 0ull;
         }
         __syncthreads();
-        const uint32_t tick = s_tick;
+        const int64_t rl = s_tick;
         __syncthreads();
-        if (tick >= rtotal) break;
-        const int64_t rl = a.rlist ? (int64_t)__ldcg(a.rlist + tick) : (int64_t)tick;
+        if (rl >= a.R) break;
         K2_PHASE(0);
         const int64_t r = a.r0 + rl;
         const float CP = a.cp[rl];
@@ -1705,8 +1699,6 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
 
 }  // namespace mpk
 
-#include "rep3.cuh"   // K3 (uses the helpers above; its launch is used by rep2_launch below)
-
 namespace mph {
 
 template <int A>
@@ -1719,8 +1711,7 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
                    align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 8) +
-                   align256((size_t)grid2 * ((n + 15) & ~15) * 4) + align256((size_t)grid2 * R3_GEO_BYTES) +
-                   align256((size_t)R * 4);
+                   align256((size_t)grid2 * ((n + 15) & ~15) * 4) + align256((size_t)grid2 * R3_GEO_BYTES);
     MP_TRY(ensure_ws(dag, bytes, st));
     Arena ar{dag->ws, dag->ws_cap};
     Rep2Args a{};
@@ -1753,7 +1744,6 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     a.qtask = qtask;
     a.sum = sum;
     a.ticket = dag->tickets + 56;
-    a.fb_list = A == 2 ? ar.take<int32_t>((size_t)R) : nullptr;
     static std::atomic<uint64_t> attr{0};
     const int smem1 = 32 * 32 * 33 * 4;
     const int smem2 = (int)r3_smem_bytes();
@@ -1799,32 +1789,6 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         if (cs == 1) return fail(MP_ERR_CUDA, "k_rep2_bl launch: %s", cudaGetErrorString(e));
     }
     MP_CUDA(cudaMemsetAsync(a.ticket, 0, 4, st));
-    if (A == 2 && r4_fits(dag)) {
-        // K3: the on-chip two-arch sort (rep3.cuh); replicas it cannot take go to K2's list
-        R4Args b{};
-        b.n = n;
-        b.R = R;
-        b.r0 = r0;
-        b.base = base;
-        b.emask = emask;
-        b.seed = seed;
-        b.sigma = sigma;
-        b.cp = cp;
-        b.hd = a.hd;
-        b.counts = a.counts;
-        b.brw = a.brw;
-        b.bl32 = a.bl32;
-        b.qof = dag->qof;
-        b.qtask = qtask;
-        b.sum = sum;
-        b.ticket = dag->tickets + 57;
-        b.fb_list = a.fb_list;
-        b.fb_count = reinterpret_cast<uint32_t*>(dag->tickets + 58);
-        MP_CUDA(cudaMemsetAsync(dag->tickets + 57, 0, 8, st));
-        MP_TRY(rep3_launch(dag, b, st));
-        a.rlist = b.fb_list;
-        a.rlist_n = b.fb_count;
-    }
     {
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3((unsigned)grid2);
