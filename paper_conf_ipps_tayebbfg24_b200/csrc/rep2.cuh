@@ -1763,8 +1763,11 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     MP_CUDA(cudaMemsetAsync(a.counts, 0, (size_t)R * A * 4, st));
     MP_CUDA(cudaMemsetAsync(a.brw, 0, (size_t)R * A * 16, st));
     // cluster size: enough CTAs per 32-replica group to cover the SMs (strong scaling keeps K1 short)
+    // (8-CTA clusters and a cross-CTA dataflow mode -- bl lines as ready flags polled from L2 --
+    // measured slower: R = 512 K1 0.98 ms (4-CTA, level barriers) vs 1.58 ms (8-CTA) and
+    // 1.06 ms (4-CTA dataflow); the per-group time is a latency floor of ~5 us per level)
     int cs = 1;
-    while (cs < 4 && groups * (cs * 2) <= dag->num_sms) cs *= 2;   // 8-CTA clusters measured slower
+    while (cs < 4 && groups * (cs * 2) <= dag->num_sms) cs *= 2;
     for (;; cs /= 2) {
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3((unsigned)(groups * cs));
