@@ -67,6 +67,8 @@ CONFIG_TEXT = {
              "960x960-double tiles, per-node residency, transfers at 2^-24 ms/byte (~16.8 GB/s)",
     "c4fmm": "the FMM octree part of c4 alone (depth 8, 2^19 particles, 1,099,435 tasks, 24,008,280 edges, "
              "13 levels; TBFMM-shaped, PAPER.md l.263-270), 2 resource types",
+    "hier": "N4 workload: tiled Cholesky with hierarchical tasks (PAPER.md l.318), 48x48 coarse tiles, each task "
+            "expanded into its 2x2-sub-tile sub-graph with probability 1/2 (85,673 tasks), 2 resource types",
     "lu64": "N4 workload: tiled LU without pivoting 64x64 tiles (getrf, PAPER.md l.251; 89,440 tasks), 2 resource types",
     "c2n4": "N4 variants on the 64x64 Cholesky DAG: mean-cost (HEFT) bottom-level, hd as a running max along the "
             "push order (id order), NOD on the remaining graph (first half of the level order completed), "
@@ -76,7 +78,7 @@ CONFIG_TEXT = {
 }
 L2_FLUSH_BYTES = 256 << 20
 REPLICA_CFGS = ("c5", "c5sim", "c5loc")
-SINGLE_CFGS = ("c1", "c2", "c3", "c4", "c4fmm", "lu64")
+SINGLE_CFGS = ("c1", "c2", "c3", "c4", "c4fmm", "lu64", "hier")
 KERNELS = ("k_rep_main", "k_rep_out", "k_sort_pass", "k_sort_hist", "k_sort_plan", "k_kahn", "k_csr_count",
            "k_csr_fill", "k_csr_rowsort", "k_csr_emit", "k_scan_excl", "k_iota_level_keys", "k_level_order", "k_qmaps",
            "k_qcols", "k_bl_small", "k_bl_flow", "k_aff_hd", "k_aff_gain", "k_crit_max", "k_score",

@@ -114,3 +114,51 @@ def test_lu64_full_path_bit_exact():
     Q = int(orr["qptr"][-1])
     assert np.array_equal(r["qtask"].cpu().numpy()[:Q], orr["qtask"])
     assert r["summary"].cpu().numpy().tobytes() == orr["summary"].tobytes()
+
+
+def _full_compare(w, kind=oracle.CRIT_BL):
+    """The whole a1-a9 path on the GPU vs the oracle, every output bit-exact."""
+    g, o = _dags(w.n, w.src, w.dst)
+    r = mp.score_and_queue(g, to_dev(w.dur), w.workers, kind)
+    mp.check(g)
+    orr = oracle.score_and_queue(o, w.dur, w.workers, kind)
+    ga = {k: v.cpu().numpy() for k, v in g.arrays().items()}
+    assert g.n_levels == o.n_levels and g.n_edges == o.n_edges
+    for k in ("row_ptr", "col", "indeg", "level", "level_ptr", "level_order"):
+        assert np.array_equal(ga[k], getattr(o, k)), k
+    assert np.array_equal(bits(r["bl"].cpu().numpy()), bits(orr["bl"]))
+    assert np.array_equal(bits(r["gain"].cpu().numpy()), bits(orr["gain"]))
+    assert np.array_equal(bits(r["crit_norm"].cpu().numpy()), bits(orr["crit_norm"]))
+    assert np.array_equal(r["key"].cpu().numpy().view(np.uint64), orr["key"])
+    Q = int(orr["qptr"][-1])
+    assert np.array_equal(r["qptr"].cpu().numpy(), orr["qptr"])
+    assert np.array_equal(r["qtask"].cpu().numpy()[:Q], orr["qtask"])
+    assert r["summary"].cpu().numpy().tobytes() == orr["summary"].tobytes()
+    return g, o
+
+
+@pytest.mark.parametrize("N,p,seed", [(6, 0.5, 1), (12, 0.3, 2), (16, 1.0, 3), (16, 0.0, 4)])
+def test_hier_small_full_path_bit_exact(N, p, seed):
+    """N4 hierarchical-task Cholesky (P:l.318): mixed granularity, no / full expansion."""
+    w = workloads.hier(N, 2, p, seed)
+    _full_compare(w)
+    _full_compare(w, oracle.CRIT_NOD)
+
+
+def test_hier_config_full_path_and_replicas():
+    """The bench's hier config (48 x 48 coarse tiles, half expanded: 85,673 tasks) through
+    a1-a9, then 40 duration-perturbed replicas of it (a10; n >= 65,536: the general path) against
+    the oracle, every replica."""
+    w = workloads.config("hier")
+    g, o = _full_compare(w)
+    R = 40
+    cp, summ, q = mp.replicas_run(g, to_dev(w.dur), w.workers, workloads.C5_SEED, workloads.C5_SIGMA, 5, R)
+    mp.check(g)
+    cp = cp.cpu().numpy()
+    gs = mp.summaries(summ).reshape(R, w.n_arch)
+    q = q.cpu().numpy()
+    for i in range(R):
+        ocp, osum, oq, _ = oracle.replica(o, w.dur, w.workers, workloads.C5_SEED, workloads.C5_SIGMA, 5 + i)
+        assert bits(cp[i:i + 1])[0] == bits(np.float32(ocp)), i
+        assert gs[i].tobytes() == osum.tobytes(), i
+        assert np.array_equal(q[i, :len(oq)], oq), i

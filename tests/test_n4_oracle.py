@@ -178,3 +178,80 @@ def test_nod_remaining_against_fractions(seed):
             assert abs(float(nod[t, a]) - float(exact)) <= tol
     assert np.array_equal(oracle.nod_remaining(dag, dur, [1, 1], np.zeros(n, np.uint8)),
                           oracle.nod(dag, dur, [1, 1]))
+
+
+# ---------------------------------------------------------------- hierarchical tasks (P:l.318)
+
+def _chol_counts(M):
+    """Closed forms of the M x M tiled Cholesky (SURVEY §8(c) a1/a2 pins)."""
+    from math import comb
+    return M + M * (M - 1) + comb(M, 3), (M - 1) * M * (M + 1) // 2, 3 * M - 2
+
+
+@pytest.mark.parametrize("N,s", [(3, 2), (5, 2), (4, 3)])
+def test_hier_extremes_are_the_plain_tilings(N, s):
+    """Hierarchical tasks (reading h1): expanding no task gives the N x N tiled Cholesky,
+    expanding every task the (N s) x (N s) one -- n, E, depth from the closed forms, and
+    (small case) the same DAG up to relabelling, kernel kinds matched."""
+    import networkx as nx
+    from workloads import dense
+    for p, M in ((0.0, N), (1.0, N * s)):
+        rec = dense.hier_cholesky(N, s, p)
+        src, dst = rec.edges()
+        dag = oracle.build_dag(rec.n, src, dst)
+        assert (dag.n, dag.n_edges, dag.n_levels) == _chol_counts(M)
+    if N * s <= 8:
+        def graph(rec, fine):
+            src, dst = rec.edges()
+            G = nx.DiGraph()
+            for t, kd in enumerate(rec.kinds().tolist()):
+                G.add_node(t, kind=kd - 4 if fine else kd)
+            G.add_edges_from(zip(src.tolist(), dst.tolist()))
+            return G
+        Gh = graph(dense.hier_cholesky(N, s, 1.0), True)
+        Gf = graph(dense.cholesky(N * s), False)
+        assert nx.is_isomorphic(Gh, Gf, node_match=lambda x, y: x["kind"] == y["kind"])
+
+
+def test_hier_full_expansion_cp_closed_form():
+    """Every task expanded: the DAG is the (N s)-tile Cholesky with the fine-task weights,
+    so CP = p + (M-1) t + (M-2) max(g, s+p) + s + p (SURVEY §8(c) a4, M = N s) with
+    w = min(CPU, GPU) of HIER_MODEL's fine kernels (dyadic: exact in binary32)."""
+    import workloads
+    from workloads import dense
+    N, s = 6, 2
+    w = workloads.hier(N, s, 1.0)
+    assert set(np.unique(w.kind).tolist()) == {dense.POTRF_F, dense.TRSM_F, dense.SYRK_F, dense.GEMM_F}
+    mn = {k: min(v) for k, v in workloads.HIER_MODEL.items()}
+    P, T, S, G = mn[dense.POTRF_F], mn[dense.TRSM_F], mn[dense.SYRK_F], mn[dense.GEMM_F]
+    M = N * s
+    dag = oracle.build_dag(w.n, w.src, w.dst)
+    bl, cp = oracle.bottom_level(dag, w.dur, w.workers)
+    assert float(cp) == P + (M - 1) * T + (M - 2) * max(G, S + P) + S + P
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_hier_partial_levels_and_cp_against_networkx(seed):
+    """Partly expanded DAGs (mixed granularity): levels = networkx generations, CP = the
+    networkx longest path with w = min over archs (dyadic weights: exact)."""
+    import networkx as nx
+    import workloads
+    w = workloads.hier(6, 2, 0.5, seed)
+    assert 0 < int((w.kind >= 4).sum()) < w.n          # both granularities present
+    dag = oracle.build_dag(w.n, w.src, w.dst)
+    G = nx.DiGraph()
+    G.add_nodes_from(range(w.n))
+    G.add_edges_from(zip(w.src.tolist(), w.dst.tolist()))
+    gens = list(nx.topological_generations(G))
+    assert dag.n_levels == len(gens)
+    for lv, g in enumerate(gens):
+        assert sorted(g) == sorted(np.where(dag.level == lv)[0].tolist())
+    wt = w.dur.min(axis=1)
+    for v in G:
+        G.nodes[v]["w"] = float(wt[v])
+    longest = {}
+    for v in reversed(list(nx.topological_sort(G))):
+        longest[v] = G.nodes[v]["w"] + max((longest[u] for u in G.successors(v)), default=0.0)
+    bl, cp = oracle.bottom_level(dag, w.dur, w.workers)
+    assert float(cp) == max(longest.values())
+    assert all(float(bl[v]) == longest[v] for v in G)

@@ -14,6 +14,7 @@ Configs (BASELINE.json order):
   c4  sparse-QR-like tree (G=42) U FMM octree (H=8, 2^19 parts)  (A=2)
   c5  replicas of c2 (R=4096, sigma=1/8, seed 20240311)
   c4fmm  c4's FMM octree part alone (TBFMM-shaped)
+  hier   N4: Cholesky with hierarchical tasks
 """
 from __future__ import annotations
 
@@ -48,6 +49,17 @@ SPQR_MODEL = {  # (CPU, GPU): QR tile kernels use the QR CPU/GPU columns; ASM is
     sparse_qr.TSMQR: (48.0, 3.0),
     sparse_qr.ASM: (0.125, np.inf),
 }
+# Hierarchical Cholesky: coarse tasks keep CHOL_MODEL; a
+# fine sub-task (tile s = 2 times smaller: 1/8 of the flops) costs 1/8 on a CPU and, GPUs
+# being far less efficient on small tiles, 4/8 of the coarse GPU time (reading h3) -- so the
+# DAG mixes large GPU-friendly tasks with small CPU-friendly ones, as §VII describes.
+HIER_MODEL = dict(CHOL_MODEL)
+HIER_MODEL.update({
+    dense.POTRF_F: (0.75, 1.5),
+    dense.TRSM_F: (1.5, 0.5),
+    dense.SYRK_F: (1.5, 0.375),
+    dense.GEMM_F: (3.75, 0.75),
+})
 LU_MODEL = {  # (CPU, GPU), SURVEY §8(f) N4
     dense.GETRF: (12.0, 6.0),
     dense.TRSM_L: (12.0, 1.0),
@@ -115,6 +127,14 @@ def qr(N: int, split_diag: bool = True) -> Workload:
                      tiles=N, split_diag=split_diag)
 
 
+def hier(N: int, s: int = 2, p_expand: float = 0.5, seed: int = 31) -> Workload:
+    """Cholesky with hierarchical tasks (N4): N x N coarse tiles, expanded tasks at s x s
+    sub-tiles (dense.hier_cholesky).  Durations: HIER_MODEL (defined for s = 2)."""
+    assert s == 2, "HIER_MODEL's fine-task durations are defined for s = 2"
+    return _from_stf(f"hier{N}", dense.hier_cholesky(N, s, p_expand, seed), HIER_MODEL, ("CPU", "GPU"),
+                     tiles=N, split=s, p_expand=p_expand, seed=seed)
+
+
 def lu(N: int) -> Workload:
     return _from_stf(f"lu{N}", dense.lu(N), LU_MODEL, ("CPU", "GPU"), tiles=N)
 
@@ -162,6 +182,8 @@ def config(name: str) -> Workload:
         w = union(sparse_tree(42, 64, 32), fmm_tree(8, 1 << 19, 7), "c4")
     elif name == "c4fmm":       # c4's FMM part alone (the 13-level single-DAG case)
         w = fmm_tree(8, 1 << 19, 7)
+    elif name == "hier":        # N4: hierarchical tasks (48 x 48 coarse tiles, half expanded)
+        w = hier(48, 2, 0.5, 31)
     elif name == "lu64":
         w = lu(64)
     else:

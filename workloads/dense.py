@@ -74,3 +74,78 @@ def lu(N: int) -> STFRecorder:
             for j in range(k + 1, N):
                 s.submit(GEMM_LU, reads=(A(i, k), A(k, j)), writes=(A(i, j),))
     return s
+
+
+# fine-granularity kernel kinds of the hierarchical Cholesky (sub-tasks of an expanded task)
+POTRF_F, TRSM_F, SYRK_F, GEMM_F = 4, 5, 6, 7
+
+
+def hier_cholesky(N: int, s: int = 2, p_expand: float = 0.5, seed: int = 31) -> STFRecorder:
+    """Tiled Cholesky with hierarchical tasks (§VII:
+    "hierarchical tasks ... submit subgraphs at runtime ... expos[ing] different task
+    sizes in the DAG").  Reading h1: the matrix has N x N coarse tiles,
+    each split into s x s fine tiles (the handles); a coarse task that is *expanded*
+    (each independently with probability p_expand, seeded -- reading h2) submits, in its
+    place, the fine-tile tasks of the same operation restricted to its tiles, in
+    right-looking order; a task that is not expanded accesses every fine tile of its
+    coarse tiles (the lower triangle of a diagonal tile).  Dependencies are then
+    inferred by the STF rules at fine-tile granularity, so an expanded sub-graph
+    inherits exactly the predecessors and successors of the data its sub-tasks touch.
+    p_expand = 0 gives cholesky(N) (coarse tasks only); p_expand = 1 gives the same
+    DAG as cholesky(N * s) (every task at fine granularity)."""
+    import numpy as np
+    rng = np.random.default_rng(seed)
+    rec = STFRecorder()
+    M = N * s
+    F = lambda I, J: I * M + J  # noqa: E731  fine tile handle
+
+    def tile(i, j):   # fine handles of coarse tile (i, j); lower triangle of a diagonal tile
+        return tuple(F(I, J) for I in range(i * s, (i + 1) * s) for J in range(j * s, (j + 1) * s)
+                     if i != j or I >= J)
+
+    def expand():
+        return p_expand >= 1.0 or (p_expand > 0.0 and rng.random() < p_expand)
+
+    for k in range(N):
+        K = range(k * s, (k + 1) * s)
+        if expand():                                   # POTRF(k): fine Cholesky of tile (k, k)
+            for Kf in K:
+                rec.submit(POTRF_F, writes=(F(Kf, Kf),))
+                for I in range(Kf + 1, (k + 1) * s):
+                    rec.submit(TRSM_F, reads=(F(Kf, Kf),), writes=(F(I, Kf),))
+                for I in range(Kf + 1, (k + 1) * s):
+                    rec.submit(SYRK_F, reads=(F(I, Kf),), writes=(F(I, I),))
+                    for J in range(Kf + 1, I):
+                        rec.submit(GEMM_F, reads=(F(I, Kf), F(J, Kf)), writes=(F(I, J),))
+        else:
+            rec.submit(POTRF, writes=tile(k, k))
+        for i in range(k + 1, N):
+            Ii = range(i * s, (i + 1) * s)
+            if expand():                               # TRSM(k, i): X L^T = B, column by column
+                for Kf in K:
+                    for I in Ii:
+                        rec.submit(TRSM_F, reads=(F(Kf, Kf),), writes=(F(I, Kf),))
+                    for J in range(Kf + 1, (k + 1) * s):
+                        for I in Ii:
+                            rec.submit(GEMM_F, reads=(F(I, Kf), F(J, Kf)), writes=(F(I, J),))
+            else:
+                rec.submit(TRSM, reads=tile(k, k), writes=tile(i, k))
+        for i in range(k + 1, N):
+            Ii = range(i * s, (i + 1) * s)
+            if expand():                               # SYRK(k, i): A(i,i) -= A(i,k) A(i,k)^T
+                for Kf in K:
+                    for I in Ii:
+                        rec.submit(SYRK_F, reads=(F(I, Kf),), writes=(F(I, I),))
+                        for J in range(i * s, I):
+                            rec.submit(GEMM_F, reads=(F(I, Kf), F(J, Kf)), writes=(F(I, J),))
+            else:
+                rec.submit(SYRK, reads=tile(i, k), writes=tile(i, i))
+            for j in range(k + 1, i):
+                if expand():                           # GEMM(k, i, j): A(i,j) -= A(i,k) A(j,k)^T
+                    for Kf in K:
+                        for I in Ii:
+                            for J in range(j * s, (j + 1) * s):
+                                rec.submit(GEMM_F, reads=(F(I, Kf), F(J, Kf)), writes=(F(I, J),))
+                else:
+                    rec.submit(GEMM, reads=tile(i, k) + tile(j, k), writes=tile(i, j))
+    return rec
