@@ -354,17 +354,19 @@ def kernel_alg_bytes(name, ctx):
     return None
 
 
-TRAFFIC_FILE = os.path.join(ROOT, "profiles", "r01", "traffic.json")
+TRAFFIC_FILES = [os.path.join(ROOT, "profiles", r, "traffic.json") for r in ("r02", "r01")]   # newest first
 
 
 def measured_traffic(kernel, cfg):
-    """dram read+write bytes per launch from a committed `ncu --set full` capture, if any."""
-    try:
-        t = json.load(open(TRAFFIC_FILE))
-        e = t.get(cfg, {}).get(kernel)
-        return (e["dram_bytes_per_launch"], e["source"]) if e else (None, None)
-    except Exception:
-        return None, None
+    """dram read+write bytes per launch from the newest committed `ncu --set full` capture, if any."""
+    for f in TRAFFIC_FILES:
+        try:
+            e = json.load(open(f)).get(cfg, {}).get(kernel)
+        except Exception:
+            continue
+        if e:
+            return e["dram_bytes_per_launch"], e["source"]
+    return None, None
 
 
 def base_workload(cfg):
@@ -603,6 +605,28 @@ def run_ours(args):
     mp.prof_enable(False)
     prof = {k: mp.prof_query(k) for k in mp.prof_names()}
 
+    # ---- per-level latency microbenchmarks (independent of the product kernels) ----
+    def t_level_us():
+        Lm = 2000
+        sink = torch.zeros(1, dtype=torch.int32, device=dev)
+        M = 1 << 20                                            # 4 MB pointer cycle: L2 resident
+        perm = np.random.default_rng(1).permutation(M).astype(np.uint32)
+        nxt = np.empty(M, np.uint32)
+        nxt[perm] = np.roll(perm, -1)
+        chain = torch.from_numpy(nxt.view(np.int32)).to(dev)
+        out = {}
+        for name, kind, arg in (("syncthreads", mp.MB_SYNC, 0), ("cluster2", mp.MB_CLUSTER, 2),
+                                ("cluster4", mp.MB_CLUSTER, 4), ("cluster8", mp.MB_CLUSTER, 8),
+                                ("grid", mp.MB_GRID, 0), ("l2_chain", mp.MB_CHAIN, 0)):
+            fn = (lambda k=kind, a=arg: mp.microbench(k, Lm, sink, a, chain))
+            for _ in range(2):
+                fn()
+            ms = timed(fn, 5, sync_ranks=False)
+            out[name + "_us"] = statistics.median(ms) * 1e3 / Lm
+        return out
+
+    tlev = t_level_us()
+
     # ---- single DAGs: depth probe (SURVEY §8(d) two-term roofline) ----
     score_only = None
     if cfg in SINGLE_CFGS:
@@ -708,6 +732,12 @@ def run_ours(args):
             dp["bytes_floor_ms"] = score_only["alg_bytes"] / 1e9 / peak * 1e3
             dp["two_term_floor_ms"] = max(dp["bytes_floor_ms"], dp["ms_score_only"])
             dp["frac_of_two_term"] = dp["two_term_floor_ms"] / score_only["ms_per_dag"]
+        # microbenchmark floor of one level-synchronous bottom-level pass: per level one
+        # block barrier + two dependent L2 round trips (successor ids, then their bl)
+        Lv = dag.n_levels
+        score_only["level_floor_ms"] = Lv * (tlev["syncthreads_us"] + 2 * tlev["l2_chain_us"]) * 1e-3
+        score_only["two_term_floor_ms"] = max(score_only["alg_bytes"] / 1e9 / peak * 1e3, score_only["level_floor_ms"])
+        score_only["frac_of_two_term_floor"] = score_only["two_term_floor_ms"] / score_only["ms_per_dag"]
 
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
@@ -750,6 +780,11 @@ def run_ours(args):
             "build_ms": build_ms, "build_plus_step_ms": build_ms + ms_per_step,
             **({"allgather": allgather} if allgather else {}),
             "roofline": roof, **({"score_only": score_only} if score_only else {}),
+            "t_level": {**{k: round(v, 4) for k, v in tlev.items()},
+                        "how": "mp_microbench: 2000 level boundaries per launch (empty __syncthreads loop in one "
+                               "CTA, cluster barrier loop, cooperative grid barrier loop on every SM, one "
+                               "thread's dependent ld.global.cg chain over a 4 MB L2-resident cycle), median "
+                               "of 5 CUDA-event-timed launches, microseconds per level"},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
             "gpu_launches_per_step": launches / args.steps, "clocks": ck,
             "device": torch.cuda.get_device_name(dev)}

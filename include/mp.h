@@ -362,6 +362,22 @@ const char* mp_last_error(void);
 /* Library introspection for tests: "sm_100a", version string. */
 const char* mp_build_info(void);
 
+/*
+ * Per-level latency microbenchmarks (SURVEY §8(d) two-term roofline): a level-
+ * synchronous pass over a depth-L DAG costs at least L x t_level.  Launches one
+ * microkernel on `stream` that performs L level boundaries of the given kind and
+ * nothing else (the caller times it):
+ *   MP_MB_SYNC     one CTA of 1024 threads, L __syncthreads
+ *   MP_MB_CLUSTER  one cluster of `arg` (2..8) CTAs, L cluster barriers
+ *   MP_MB_GRID     one CTA per SM (cooperative launch), L grid barriers
+ *   MP_MB_CHAIN    one thread, L dependent L2 loads p = d_next[p] (d_next: a
+ *                  permutation cycle of uint32 indices, device, caller-owned)
+ * d_sink: one uint32 of device scratch (keeps the work observable).
+ */
+enum { MP_MB_SYNC = 0, MP_MB_CLUSTER = 1, MP_MB_GRID = 2, MP_MB_CHAIN = 3 };
+mp_status mp_microbench(int32_t kind, int32_t L, int32_t arg, const uint32_t* d_next, uint32_t* d_sink,
+                        void* stream);
+
 /* Diagnostics.  mp_launch_count: kernels libmp has launched in this process.
  * mp_prof_enable(1): bracket every launch with CUDA events on its stream;
  * mp_prof_query synchronises on those events and returns the summed device

@@ -393,6 +393,16 @@ def build_info() -> str:
     return _lib.lib().mp_build_info().decode()
 
 
+MB_SYNC, MB_CLUSTER, MB_GRID, MB_CHAIN = 0, 1, 2, 3
+
+
+def microbench(kind: int, L: int, sink: torch.Tensor, arg: int = 0, chain: torch.Tensor | None = None):
+    """mp_microbench: launch one per-level latency microkernel (L level boundaries of `kind`)
+    on the current stream; the caller times it (bench.py's t_level)."""
+    _lib.check(_lib.lib().mp_microbench(int(kind), int(L), int(arg), _ptr(chain) if chain is not None else None,
+                                        _ptr(sink), _stream()), "mp_microbench")
+
+
 def launch_count() -> int:
     """Kernels libmp has launched in this process (mp_launch_count)."""
     return int(_lib.lib().mp_launch_count())

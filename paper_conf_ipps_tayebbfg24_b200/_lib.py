@@ -20,6 +20,7 @@ EXPORTS = (
     "mp_build_queues", "mp_replicas_run", "mp_ready_init", "mp_queues_push", "mp_simulate", "mp_simulate_cfg",
     "mp_bottom_level_w", "mp_affinity_prefix", "mp_nod_remaining", "mp_queues_push_all",
     "mp_check", "mp_free", "mp_status_str", "mp_last_error", "mp_build_info", "mp_launch_count", "mp_prof_enable", "mp_prof_reset", "mp_prof_query", "mp_prof_names",
+    "mp_microbench",
 )
 
 
@@ -74,6 +75,7 @@ def lib():
     L.mp_nod_remaining.argtypes = [P, i32, P, P, P, P, P]
     L.mp_queues_push_all.argtypes = [P, i32, P, P, P, P, P, i32, P, P, P, P, P, P]
     L.mp_check.argtypes = [P, P]
+    L.mp_microbench.argtypes = [i32, i32, i32, P, P, P]
     L.mp_free.argtypes = [P]
     L.mp_free.restype = None
     L.mp_status_str.argtypes = [C.c_int]

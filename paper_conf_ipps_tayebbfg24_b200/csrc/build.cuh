@@ -753,8 +753,8 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
     ALLOC(dag->level_ptr, nn + 1);
     ALLOC(dag->level_order, nn);
     ALLOC(dag->qof, nn);
-    ALLOC(dag->nodeq, nn);
-    ALLOC(dag->rowq, nn + 1);
+    ALLOC(dag->nodeq, nn + 4);        // + 4: k_bl_small's 16-byte aligned bulk copies read past the end
+    ALLOC(dag->rowq, nn + 1 + 4);
     CK(cudaMemsetAsync(dag->err, 0, 16, st));
     CK(cudaMemsetAsync(dag->tickets, 0, 64 * 4, st));
     CK(cudaMemsetAsync(dag->row_ptr, 0, (nn + 1) * 4, st));
@@ -954,7 +954,7 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
         ALLOC(dag->lvlp, L + 1);
         ALLOC(dag->nodep, P);
         ALLOC(dag->rowp, P + 1);
-        ALLOC(dag->colq, dag->E > 0 ? dag->E : 1);
+        ALLOC(dag->colq, (dag->E > 0 ? dag->E : 1) + 4);
         ALLOC(dag->colp, dag->E > 0 ? dag->E : 1);
         ALLOC(dag->b_pof, nn);
         int32_t* pof = dag->b_pof;
@@ -983,7 +983,7 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
         ALLOC(dag->lvlp, 1);
         ALLOC(dag->nodep, 1);
         ALLOC(dag->rowp, 1);
-        ALLOC(dag->colq, 1);
+        ALLOC(dag->colq, 1 + 4);
         ALLOC(dag->colp, 1);
         CK(cudaMemsetAsync(dag->lvlq, 0, 4, st));
         CK(cudaMemsetAsync(dag->lvlp, 0, 4, st));

@@ -46,19 +46,90 @@ MP_INLINE float task_weight(const DurView& d, int32_t v, bool& bad) {
 // __syncthreads per level; bl(v) = w(v) + max bl(succ) with a single RN add.
 // Nothing but the successors' bl depends on the previous level, so it is taken off
 // the per-level chain: a prologue writes every w(v) into its slot sbl[q] (all loads
-// in flight at once), and each thread's first row range of the next level is loaded
-// one level ahead.  A level then costs the colq round trip + the shared-memory max +
-// the barrier (max is exact and order-free, so the bits are unchanged).
+// in flight at once), and the next level's CSR slice -- its row offsets (rowq), node
+// ids (nodeq) and successor positions (colq), contiguous ranges of q-space -- is
+// copied into a shared-memory staging buffer by a TMA bulk copy (cp.async.bulk,
+// mbarrier completion) while the current level computes: a staged level reads only
+// shared memory, so it costs the shared-memory gathers + the barrier.  A level whose
+// slice does not fit the buffer reads the CSR from L2 (prefetched there at start).
+// (max is exact and order-free, so the bits are unchanged.)
+MP_INLINE void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(bar)), "r"(count)
+                 : "memory");
+}
+MP_INLINE void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(
+                     (uint32_t)__cvta_generic_to_shared(bar)), "r"(bytes)
+                 : "memory");
+}
+MP_INLINE void mbar_wait(uint64_t* bar, uint32_t phase) {
+    const uint32_t a = (uint32_t)__cvta_generic_to_shared(bar);
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(a), "r"(phase)
+            : "memory");
+    }
+}
+// bulk copy global -> shared (16-byte aligned, size a multiple of 16), completion on bar
+MP_INLINE void tma_bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     (uint32_t)__cvta_generic_to_shared(dst)),
+                 "l"(src), "r"(bytes), "r"((uint32_t)__cvta_generic_to_shared(bar))
+                 : "memory");
+}
+
+struct BlStage {          // one staging buffer: a level's CSR slice in shared memory
+    int32_t qa, qb;       // the level's q range
+    int32_t e0;           // rowq[qa]
+    int32_t ok;           // staged (else read from global)
+    int32_t orow, onod, ocol;   // element offsets of the slices inside their 16-byte aligned copies
+};
+
 __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
                                                    const int32_t* __restrict__ nodeq,
                                                    const int32_t* __restrict__ rowq,
                                                    const int32_t* __restrict__ colq, DurView d, float* bl,
-                                                   float* cp, uint32_t* err) {
-    extern __shared__ float sbl[];
+                                                   float* cp, uint32_t* err, int32_t stage_words) {
+    extern __shared__ __align__(16) float sbl[];
+    __shared__ __align__(8) uint64_t bars[2];
+    __shared__ BlStage stg[2];
     bool bad = false;
     float cpm = 0.0f;
     const int32_t t = (int32_t)threadIdx.x;
     const int32_t nq = __ldg(lvlq + L);
+    // staging buffers after sbl (16-byte aligned), stage_words int32 each (0: no staging)
+    int32_t* sbuf[2];
+    sbuf[0] = reinterpret_cast<int32_t*>(sbl + ((nq + 3) & ~3));
+    sbuf[1] = sbuf[0] + stage_words;
+    const int32_t prod = (int32_t)blockDim.x - 1;   // producer thread: the last one
+    // producer: stage level r's slice into buffer b (called one level ahead)
+    auto stage = [&](int32_t r, int b) {
+        BlStage& S = stg[b];
+        S.ok = 0;
+        if (r >= L || stage_words <= 0) return;
+        const int32_t qa = __ldg(lvlq + r), qb = __ldg(lvlq + r + 1);
+        const int32_t e0 = __ldg(rowq + qa), e1 = __ldg(rowq + qb);
+        S.qa = qa;
+        S.qb = qb;
+        S.e0 = e0;
+        // three aligned copies: rowq[qa .. qb] (qb-qa+1), nodeq[qa .. qb), colq[e0 .. e1)
+        const int32_t ra = qa & ~3, rn = ((qb + 1 + 3) & ~3) - ra;
+        const int32_t na = qa & ~3, nn = ((qb + 3) & ~3) - na;
+        const int32_t ca = e0 & ~3, cn = ((e1 + 3) & ~3) - ca;
+        if (rn + nn + cn > stage_words) return;
+        S.orow = qa - ra;
+        S.onod = rn + (qa - na);
+        S.ocol = rn + nn + (e0 - ca);
+        int32_t* dst = sbuf[b];
+        mbar_expect_tx(&bars[b], (uint32_t)(rn + nn + cn) * 4u);
+        tma_bulk_g2s(dst, rowq + ra, (uint32_t)rn * 4u, &bars[b]);
+        tma_bulk_g2s(dst + rn, nodeq + na, (uint32_t)nn * 4u, &bars[b]);
+        if (cn > 0) tma_bulk_g2s(dst + rn + nn, colq + ca, (uint32_t)cn * 4u, &bars[b]);
+        S.ok = 1;
+    };
     {
         // the level walk reads every successor id and row bound once, a level at a time:
         // pull them into L2 now (one prefetch per 128-byte line) so no level waits on HBM
@@ -66,45 +137,60 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
         for (int32_t e = t * 32; e < E; e += blockDim.x * 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(colq + e));
         for (int32_t q = t * 32; q <= nq; q += blockDim.x * 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(rowq + q));
     }
-    for (int32_t q = t; q < nq; q += blockDim.x) sbl[q] = task_weight(d, __ldg(nodeq + q), bad);
-    int32_t qa = __ldg(lvlq), qb = L > 0 ? __ldg(lvlq + 1) : qa;
-    int32_t pe0 = 0, pe1 = 0;
-    if (qa + t < qb) {
-        pe0 = __ldg(rowq + qa + t);
-        pe1 = __ldg(rowq + qa + t + 1);
+    if (t == prod) {
+        mbar_init(&bars[0], 1);
+        mbar_init(&bars[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+    for (int32_t q = t; q < nq; q += blockDim.x) sbl[q] = task_weight(d, __ldg(nodeq + q), bad);
     __syncthreads();
+    if (t == prod) stage(0, 0);
+    uint32_t ph[2] = {0u, 0u};
     for (int32_t r = 0; r < L; r++) {
-        const int32_t qc = r + 2 <= L ? __ldg(lvlq + r + 2) : qb;
-        int32_t ne0 = 0, ne1 = 0;
-        if (qb + t < qc) {
-            ne0 = __ldg(rowq + qb + t);
-            ne1 = __ldg(rowq + qb + t + 1);
-        }
-        for (int32_t q = qa + t; q < qb; q += blockDim.x) {
-            int32_t e = pe0, e1 = pe1;
-            if (q != qa + t) {
-                e = __ldg(rowq + q);
-                e1 = __ldg(rowq + q + 1);
+        const int b = r & 1;
+        // the next level's slice goes into the other buffer (free: its level ended at the
+        // previous barrier) while this level computes
+        if (t == prod) stage(r + 1, b ^ 1);
+        const BlStage S = stg[b];
+        const int32_t qa = __ldg(lvlq + r), qb = __ldg(lvlq + r + 1);
+        if (S.ok) {
+            mbar_wait(&bars[b], ph[b]);
+            const int32_t* srow = sbuf[b] + S.orow - qa;       // srow[q] = rowq[q]
+            const int32_t* snod = sbuf[b] + S.onod - qa;       // snod[q] = nodeq[q]
+            const int32_t* scol = sbuf[b] + S.ocol - S.e0;     // scol[e] = colq[e]
+            for (int32_t q = qa + t; q < qb; q += blockDim.x) {
+                int32_t e = srow[q];
+                const int32_t e1 = srow[q + 1];
+                const int32_t v = snod[q];
+                float m = 0.0f;  // bl >= 0, and w + 0 = w: same as "bl = w without successors"
+                for (; e + 4 <= e1; e += 4)
+                    m = fmaxf(m, fmaxf(fmaxf(sbl[scol[e]], sbl[scol[e + 1]]), fmaxf(sbl[scol[e + 2]], sbl[scol[e + 3]])));
+                for (; e < e1; e++) m = fmaxf(m, sbl[scol[e]]);
+                const float bb = __fadd_rn(sbl[q], m);
+                sbl[q] = bb;
+                bl[v] = bb;
+                cpm = fmaxf(cpm, bb);
             }
-            const int32_t v = __ldg(nodeq + q);
-            float m = 0.0f;  // bl >= 0, and w + 0 = w: same as "bl = w without successors"
-            for (; e + 4 <= e1; e += 4) {
-                const int32_t c0 = __ldg(colq + e), c1 = __ldg(colq + e + 1);
-                const int32_t c2 = __ldg(colq + e + 2), c3 = __ldg(colq + e + 3);
-                m = fmaxf(m, fmaxf(fmaxf(sbl[c0], sbl[c1]), fmaxf(sbl[c2], sbl[c3])));
+        } else {
+            for (int32_t q = qa + t; q < qb; q += blockDim.x) {
+                int32_t e = __ldg(rowq + q);
+                const int32_t e1 = __ldg(rowq + q + 1);
+                const int32_t v = __ldg(nodeq + q);
+                float m = 0.0f;
+                for (; e + 4 <= e1; e += 4) {
+                    const int32_t c0 = __ldg(colq + e), c1 = __ldg(colq + e + 1);
+                    const int32_t c2 = __ldg(colq + e + 2), c3 = __ldg(colq + e + 3);
+                    m = fmaxf(m, fmaxf(fmaxf(sbl[c0], sbl[c1]), fmaxf(sbl[c2], sbl[c3])));
+                }
+                for (; e < e1; e++) m = fmaxf(m, sbl[__ldg(colq + e)]);
+                const float bb = __fadd_rn(sbl[q], m);
+                sbl[q] = bb;
+                bl[v] = bb;
+                cpm = fmaxf(cpm, bb);
             }
-            for (; e < e1; e++) m = fmaxf(m, sbl[__ldg(colq + e)]);
-            const float b = __fadd_rn(sbl[q], m);
-            sbl[q] = b;
-            bl[v] = b;
-            cpm = fmaxf(cpm, b);
         }
+        if (S.ok) ph[b] ^= 1u;
         __syncthreads();
-        qa = qb;
-        qb = qc;
-        pe0 = ne0;
-        pe1 = ne1;
     }
     cpm = warp_max(cpm);
     if ((threadIdx.x & 31) == 0) atomicMax((uint32_t*)cp, f2u(cpm));
@@ -492,11 +578,18 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
     const int32_t n = dag->n;
     if (n == 0) return MP_OK;
     if (n <= SMALL_CAP) {
+        // bl in shared memory; what is left of the opt-in maximum holds two CSR staging buffers
+        int optin = 0;
+        MP_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dag->device));
+        const size_t sbytes = (size_t)((n + 3) & ~3) * 4;
+        const int64_t avail = (int64_t)optin - (int64_t)sbytes - 1024;   // static smem + slack
+        const int32_t stage_words = avail >= 2 * 1024 ? (int32_t)((avail / 2 / 4) & ~3) : 0;
+        const size_t smem = sbytes + (size_t)2 * stage_words * 4;
         static std::atomic<uint64_t> attr{0};
-        size_t smem = (size_t)n * 4;
         if (first_on_device(attr))
-            MP_CUDA(cudaFuncSetAttribute(k_bl_small, cudaFuncAttributeMaxDynamicSharedMemorySize, SMALL_CAP * 4));
-        MP_LAUNCH(k_bl_small, 1, 1024, smem, st, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp, dag->err);
+            MP_CUDA(cudaFuncSetAttribute(k_bl_small, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - 1024));
+        MP_LAUNCH(k_bl_small, 1, 1024, smem, st, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp, dag->err,
+                  stage_words);
     } else {
         size_t need = align256((size_t)dag->P * 4);
         MP_TRY(ensure_ws(dag, need, st));
