@@ -88,30 +88,35 @@ struct BlStage {          // one staging buffer: a level's CSR slice in shared m
     int32_t orow, onod, ocol;   // element offsets of the slices inside their 16-byte aligned copies
 };
 
+constexpr int BL_NB = 8;        // k_bl_small: staging ring (levels in flight ahead of the walk)
+constexpr int BL_LTAB = 4096;   // level-bound table in shared memory for L < BL_LTAB
+
 __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
                                                    const int32_t* __restrict__ nodeq,
                                                    const int32_t* __restrict__ rowq,
                                                    const int32_t* __restrict__ colq, DurView d, float* bl,
                                                    float* cp, uint32_t* err, int32_t stage_words) {
     extern __shared__ __align__(16) float sbl[];
-    __shared__ __align__(8) uint64_t bars[2];
-    __shared__ BlStage stg[2];
+    __shared__ __align__(8) uint64_t bars[BL_NB];
+    __shared__ BlStage stg[BL_NB];
     bool bad = false;
     float cpm = 0.0f;
     const int32_t t = (int32_t)threadIdx.x;
     const int32_t nq = __ldg(lvlq + L);
-    // staging buffers after sbl (16-byte aligned), stage_words int32 each (0: no staging)
-    int32_t* sbuf[2];
-    sbuf[0] = reinterpret_cast<int32_t*>(sbl + ((nq + 3) & ~3));
-    sbuf[1] = sbuf[0] + stage_words;
+    // after sbl: the level-bound table (q start and edge start of every level, when L is
+    // small enough) and BL_NB staging buffers of stage_words int32 each (0: no staging)
+    const bool tab = L < BL_LTAB;
+    int32_t* lq = reinterpret_cast<int32_t*>(sbl + ((nq + 3) & ~3));      // [L + 1] q starts
+    int32_t* le = lq + (tab ? ((L + 1 + 3) & ~3) : 0);                      // [L + 1] edge starts
+    int32_t* sbase = le + (tab ? ((L + 1 + 3) & ~3) : 0);
     const int32_t prod = (int32_t)blockDim.x - 1;   // producer thread: the last one
-    // producer: stage level r's slice into buffer b (called one level ahead)
+    // producer: stage level r's slice into buffer b
     auto stage = [&](int32_t r, int b) {
         BlStage& S = stg[b];
         S.ok = 0;
         if (r >= L || stage_words <= 0) return;
-        const int32_t qa = __ldg(lvlq + r), qb = __ldg(lvlq + r + 1);
-        const int32_t e0 = __ldg(rowq + qa), e1 = __ldg(rowq + qb);
+        const int32_t qa = tab ? lq[r] : __ldg(lvlq + r), qb = tab ? lq[r + 1] : __ldg(lvlq + r + 1);
+        const int32_t e0 = tab ? le[r] : __ldg(rowq + qa), e1 = tab ? le[r + 1] : __ldg(rowq + qb);
         S.qa = qa;
         S.qb = qb;
         S.e0 = e0;
@@ -123,7 +128,7 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
         S.orow = qa - ra;
         S.onod = rn + (qa - na);
         S.ocol = rn + nn + (e0 - ca);
-        int32_t* dst = sbuf[b];
+        int32_t* dst = sbase + (int64_t)b * stage_words;
         mbar_expect_tx(&bars[b], (uint32_t)(rn + nn + cn) * 4u);
         tma_bulk_g2s(dst, rowq + ra, (uint32_t)rn * 4u, &bars[b]);
         tma_bulk_g2s(dst + rn, nodeq + na, (uint32_t)nn * 4u, &bars[b]);
@@ -138,26 +143,33 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
         for (int32_t q = t * 32; q <= nq; q += blockDim.x * 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(rowq + q));
     }
     if (t == prod) {
-        mbar_init(&bars[0], 1);
-        mbar_init(&bars[1], 1);
+        for (int b = 0; b < BL_NB; b++) mbar_init(&bars[b], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+    if (tab)
+        for (int32_t r = t; r <= L; r += blockDim.x) {
+            const int32_t q = __ldg(lvlq + r);
+            lq[r] = q;
+            le[r] = __ldg(rowq + q);
+        }
     for (int32_t q = t; q < nq; q += blockDim.x) sbl[q] = task_weight(d, __ldg(nodeq + q), bad);
     __syncthreads();
-    if (t == prod) stage(0, 0);
-    uint32_t ph[2] = {0u, 0u};
+    if (t == prod)
+        for (int32_t r = 0; r < BL_NB - 1; r++) stage(r, r % BL_NB);
+    __syncthreads();   // stg[] visible to every thread
+    uint32_t ph = 0u;  // bit b: parity of buffer b's next phase
     for (int32_t r = 0; r < L; r++) {
-        const int b = r & 1;
-        // the next level's slice goes into the other buffer (free: its level ended at the
-        // previous barrier) while this level computes
-        if (t == prod) stage(r + 1, b ^ 1);
+        const int b = r % BL_NB;
+        // level r + BL_NB - 1 goes into the buffer level r - 1 used (free since the last barrier)
+        if (t == prod) stage(r + BL_NB - 1, (r + BL_NB - 1) % BL_NB);
         const BlStage S = stg[b];
-        const int32_t qa = __ldg(lvlq + r), qb = __ldg(lvlq + r + 1);
+        const int32_t qa = tab ? lq[r] : __ldg(lvlq + r), qb = tab ? lq[r + 1] : __ldg(lvlq + r + 1);
         if (S.ok) {
-            mbar_wait(&bars[b], ph[b]);
-            const int32_t* srow = sbuf[b] + S.orow - qa;       // srow[q] = rowq[q]
-            const int32_t* snod = sbuf[b] + S.onod - qa;       // snod[q] = nodeq[q]
-            const int32_t* scol = sbuf[b] + S.ocol - S.e0;     // scol[e] = colq[e]
+            mbar_wait(&bars[b], (ph >> b) & 1u);
+            const int32_t* buf = sbase + (int64_t)b * stage_words;
+            const int32_t* srow = buf + S.orow - qa;       // srow[q] = rowq[q]
+            const int32_t* snod = buf + S.onod - qa;       // snod[q] = nodeq[q]
+            const int32_t* scol = buf + S.ocol - S.e0;     // scol[e] = colq[e]
             for (int32_t q = qa + t; q < qb; q += blockDim.x) {
                 int32_t e = srow[q];
                 const int32_t e1 = srow[q + 1];
@@ -171,6 +183,7 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
                 bl[v] = bb;
                 cpm = fmaxf(cpm, bb);
             }
+            ph ^= 1u << b;
         } else {
             for (int32_t q = qa + t; q < qb; q += blockDim.x) {
                 int32_t e = __ldg(rowq + q);
@@ -189,7 +202,6 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
                 cpm = fmaxf(cpm, bb);
             }
         }
-        if (S.ok) ph[b] ^= 1u;
         __syncthreads();
     }
     cpm = warp_max(cpm);
@@ -582,9 +594,10 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
         int optin = 0;
         MP_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dag->device));
         const size_t sbytes = (size_t)((n + 3) & ~3) * 4;
-        const int64_t avail = (int64_t)optin - (int64_t)sbytes - 1024;   // static smem + slack
-        const int32_t stage_words = avail >= 2 * 1024 ? (int32_t)((avail / 2 / 4) & ~3) : 0;
-        const size_t smem = sbytes + (size_t)2 * stage_words * 4;
+        const size_t tbytes = dag->L < BL_LTAB ? (size_t)2 * (((dag->L + 1) + 3) & ~3) * 4 : 0;   // level table
+        const int64_t avail = (int64_t)optin - (int64_t)sbytes - (int64_t)tbytes - 1024;   // static smem + slack
+        const int32_t stage_words = avail >= BL_NB * 1024 ? (int32_t)((avail / BL_NB / 4) & ~3) : 0;
+        const size_t smem = sbytes + tbytes + (size_t)BL_NB * stage_words * 4;
         static std::atomic<uint64_t> attr{0};
         if (first_on_device(attr))
             MP_CUDA(cudaFuncSetAttribute(k_bl_small, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - 1024));
