@@ -100,6 +100,7 @@ def parse():
                    help="c5 sharding: strong = --replicas in total split across ranks (BASELINE config 5), "
                         "weak = every rank scores its own block of --replicas replicas (global ids rank*R..)")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-tlevel", action="store_true", help="skip the t_level microbenchmarks")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-budget-s", type=float, default=12.0)
     return p.parse_args()
@@ -625,7 +626,7 @@ def run_ours(args):
             out[name + "_us"] = statistics.median(ms) * 1e3 / Lm
         return out
 
-    tlev = t_level_us()
+    tlev = t_level_us() if not args.no_tlevel else {"syncthreads_us": 0.0, "l2_chain_us": 0.0}
 
     # ---- single DAGs: depth probe (SURVEY §8(d) two-term roofline) ----
     score_only = None

@@ -81,21 +81,22 @@ MP_INLINE void tma_bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t
                  : "memory");
 }
 
-struct BlStage {          // one staging buffer: a level's CSR slice in shared memory
+struct BlStage {          // one staged level: its CSR slice in the shared-memory arena
     int32_t qa, qb;       // the level's q range
     int32_t e0;           // rowq[qa]
     int32_t ok;           // staged (else read from global)
-    int32_t orow, onod, ocol;   // element offsets of the slices inside their 16-byte aligned copies
+    int32_t orow, onod, ocol;   // arena offsets (int32 words) of rowq[qa], nodeq[qa], colq[e0]
+    int32_t charge;       // arena words the level holds (its copies + any wrap-around gap)
 };
 
-constexpr int BL_NB = 8;        // k_bl_small: staging ring (levels in flight ahead of the walk)
+constexpr int BL_NB = 16;       // k_bl_small: levels staged ahead of the walk, at most
 constexpr int BL_LTAB = 4096;   // level-bound table in shared memory for L < BL_LTAB
 
 __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
                                                    const int32_t* __restrict__ nodeq,
                                                    const int32_t* __restrict__ rowq,
                                                    const int32_t* __restrict__ colq, DurView d, float* bl,
-                                                   float* cp, uint32_t* err, int32_t stage_words) {
+                                                   float* cp, uint32_t* err, int32_t arena_words) {
     extern __shared__ __align__(16) float sbl[];
     __shared__ __align__(8) uint64_t bars[BL_NB];
     __shared__ BlStage stg[BL_NB];
@@ -104,36 +105,54 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
     const int32_t t = (int32_t)threadIdx.x;
     const int32_t nq = __ldg(lvlq + L);
     // after sbl: the level-bound table (q start and edge start of every level, when L is
-    // small enough) and BL_NB staging buffers of stage_words int32 each (0: no staging)
+    // small enough), then the staging arena (arena_words int32, a ring: levels are staged
+    // in order and released in order; 0: no staging)
     const bool tab = L < BL_LTAB;
     int32_t* lq = reinterpret_cast<int32_t*>(sbl + ((nq + 3) & ~3));      // [L + 1] q starts
     int32_t* le = lq + (tab ? ((L + 1 + 3) & ~3) : 0);                      // [L + 1] edge starts
-    int32_t* sbase = le + (tab ? ((L + 1 + 3) & ~3) : 0);
+    int32_t* arena = le + (tab ? ((L + 1 + 3) & ~3) : 0);
+    const int32_t A = arena_words & ~3;
     const int32_t prod = (int32_t)blockDim.x - 1;   // producer thread: the last one
-    // producer: stage level r's slice into buffer b
-    auto stage = [&](int32_t r, int b) {
-        BlStage& S = stg[b];
-        S.ok = 0;
-        if (r >= L || stage_words <= 0) return;
-        const int32_t qa = tab ? lq[r] : __ldg(lvlq + r), qb = tab ? lq[r + 1] : __ldg(lvlq + r + 1);
-        const int32_t e0 = tab ? le[r] : __ldg(rowq + qa), e1 = tab ? le[r + 1] : __ldg(rowq + qb);
-        S.qa = qa;
-        S.qb = qb;
-        S.e0 = e0;
-        // three aligned copies: rowq[qa .. qb] (qb-qa+1), nodeq[qa .. qb), colq[e0 .. e1)
-        const int32_t ra = qa & ~3, rn = ((qb + 1 + 3) & ~3) - ra;
-        const int32_t na = qa & ~3, nn = ((qb + 3) & ~3) - na;
-        const int32_t ca = e0 & ~3, cn = ((e1 + 3) & ~3) - ca;
-        if (rn + nn + cn > stage_words) return;
-        S.orow = qa - ra;
-        S.onod = rn + (qa - na);
-        S.ocol = rn + nn + (e0 - ca);
-        int32_t* dst = sbase + (int64_t)b * stage_words;
-        mbar_expect_tx(&bars[b], (uint32_t)(rn + nn + cn) * 4u);
-        tma_bulk_g2s(dst, rowq + ra, (uint32_t)rn * 4u, &bars[b]);
-        tma_bulk_g2s(dst + rn, nodeq + na, (uint32_t)nn * 4u, &bars[b]);
-        if (cn > 0) tma_bulk_g2s(dst + rn + nn, colq + ca, (uint32_t)cn * 4u, &bars[b]);
-        S.ok = 1;
+    int32_t rn = 0, head = 0, used = 0;             // producer state: next level, ring head, words held
+    // producer: decide (and, space permitting, stage) levels ahead; every level <= r + 1
+    // must be decided before this returns (the walk reads its record after the next barrier)
+    auto advance = [&](int32_t r) {
+        while (rn < L && rn <= r + BL_NB - 1) {
+            const int b = rn % BL_NB;
+            BlStage& S = stg[b];
+            const int32_t qa = tab ? lq[rn] : __ldg(lvlq + rn), qb = tab ? lq[rn + 1] : __ldg(lvlq + rn + 1);
+            const int32_t e0 = tab ? le[rn] : __ldg(rowq + qa), e1 = tab ? le[rn + 1] : __ldg(rowq + qb);
+            // three 16-byte aligned copies: rowq[qa .. qb], nodeq[qa .. qb), colq[e0 .. e1)
+            const int32_t ra = qa & ~3, rw = ((qb + 1 + 3) & ~3) - ra;
+            const int32_t na = qa & ~3, nw = ((qb + 3) & ~3) - na;
+            const int32_t ca = e0 & ~3, cw = ((e1 + 3) & ~3) - ca;
+            const int32_t sz = rw + nw + cw;
+            S.qa = qa;
+            S.qb = qb;
+            S.e0 = e0;
+            S.ok = 0;
+            S.charge = 0;
+            if (sz > A) { rn++; continue; }                         // never fits: read from L2
+            const int32_t start = head + sz <= A ? head : 0;
+            const int32_t charge = head + sz <= A ? sz : (A - head) + sz;
+            if (used + charge > A) {
+                if (rn <= r + 1) { rn++; continue; }                 // due now: read from L2
+                break;                                               // wait for space
+            }
+            head = start + sz;
+            used += charge;
+            S.charge = charge;
+            S.orow = start + (qa - ra);
+            S.onod = start + rw + (qa - na);
+            S.ocol = start + rw + nw + (e0 - ca);
+            int32_t* dst = arena + start;
+            mbar_expect_tx(&bars[b], (uint32_t)sz * 4u);
+            tma_bulk_g2s(dst, rowq + ra, (uint32_t)rw * 4u, &bars[b]);
+            tma_bulk_g2s(dst + rw, nodeq + na, (uint32_t)nw * 4u, &bars[b]);
+            if (cw > 0) tma_bulk_g2s(dst + rw + nw, colq + ca, (uint32_t)cw * 4u, &bars[b]);
+            S.ok = 1;
+            rn++;
+        }
     };
     {
         // the level walk reads every successor id and row bound once, a level at a time:
@@ -154,22 +173,24 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
         }
     for (int32_t q = t; q < nq; q += blockDim.x) sbl[q] = task_weight(d, __ldg(nodeq + q), bad);
     __syncthreads();
-    if (t == prod)
-        for (int32_t r = 0; r < BL_NB - 1; r++) stage(r, r % BL_NB);
+    if (t == prod && A > 0) advance(-1);
+    if (t == prod && A <= 0)
+        for (int b = 0; b < BL_NB; b++) stg[b].ok = 0;
     __syncthreads();   // stg[] visible to every thread
     uint32_t ph = 0u;  // bit b: parity of buffer b's next phase
     for (int32_t r = 0; r < L; r++) {
         const int b = r % BL_NB;
-        // level r + BL_NB - 1 goes into the buffer level r - 1 used (free since the last barrier)
-        if (t == prod) stage(r + BL_NB - 1, (r + BL_NB - 1) % BL_NB);
+        if (t == prod && A > 0) {
+            if (r > 0) used -= stg[(r - 1) % BL_NB].charge;   // level r - 1 is done (barrier passed)
+            advance(r);
+        }
         const BlStage S = stg[b];
         const int32_t qa = tab ? lq[r] : __ldg(lvlq + r), qb = tab ? lq[r + 1] : __ldg(lvlq + r + 1);
-        if (S.ok) {
+        if (A > 0 && S.ok) {
             mbar_wait(&bars[b], (ph >> b) & 1u);
-            const int32_t* buf = sbase + (int64_t)b * stage_words;
-            const int32_t* srow = buf + S.orow - qa;       // srow[q] = rowq[q]
-            const int32_t* snod = buf + S.onod - qa;       // snod[q] = nodeq[q]
-            const int32_t* scol = buf + S.ocol - S.e0;     // scol[e] = colq[e]
+            const int32_t* srow = arena + S.orow - qa;       // srow[q] = rowq[q]
+            const int32_t* snod = arena + S.onod - qa;       // snod[q] = nodeq[q]
+            const int32_t* scol = arena + S.ocol - S.e0;     // scol[e] = colq[e]
             for (int32_t q = qa + t; q < qb; q += blockDim.x) {
                 int32_t e = srow[q];
                 const int32_t e1 = srow[q + 1];
@@ -596,13 +617,13 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
         const size_t sbytes = (size_t)((n + 3) & ~3) * 4;
         const size_t tbytes = dag->L < BL_LTAB ? (size_t)2 * (((dag->L + 1) + 3) & ~3) * 4 : 0;   // level table
         const int64_t avail = (int64_t)optin - (int64_t)sbytes - (int64_t)tbytes - 1024;   // static smem + slack
-        const int32_t stage_words = avail >= BL_NB * 1024 ? (int32_t)((avail / BL_NB / 4) & ~3) : 0;
-        const size_t smem = sbytes + tbytes + (size_t)BL_NB * stage_words * 4;
+        const int32_t arena_words = avail >= 4096 ? (int32_t)((avail / 4) & ~3) : 0;
+        const size_t smem = sbytes + tbytes + (size_t)arena_words * 4;
         static std::atomic<uint64_t> attr{0};
         if (first_on_device(attr))
             MP_CUDA(cudaFuncSetAttribute(k_bl_small, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - 1024));
         MP_LAUNCH(k_bl_small, 1, 1024, smem, st, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp, dag->err,
-                  stage_words);
+                  arena_words);
     } else {
         size_t need = align256((size_t)dag->P * 4);
         MP_TRY(ensure_ws(dag, need, st));
