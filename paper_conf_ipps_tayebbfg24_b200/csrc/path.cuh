@@ -171,7 +171,18 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
             lq[r] = q;
             le[r] = __ldg(rowq + q);
         }
-    for (int32_t q = t; q < nq; q += blockDim.x) sbl[q] = task_weight(d, __ldg(nodeq + q), bad);
+    {   // weights: the ids of 8 positions per thread first, then their durations (loads in flight)
+        constexpr int U = 8;
+        const int32_t stride = (int32_t)blockDim.x;
+        for (int32_t q0 = t; q0 < nq; q0 += U * stride) {
+            int32_t vv[U];
+#pragma unroll
+            for (int u = 0; u < U; u++) vv[u] = q0 + u * stride < nq ? __ldg(nodeq + q0 + u * stride) : -1;
+#pragma unroll
+            for (int u = 0; u < U; u++)
+                if (vv[u] >= 0) sbl[q0 + u * stride] = task_weight(d, vv[u], bad);
+        }
+    }
     __syncthreads();
     if (t == prod && A > 0) advance(-1);
     if (t == prod && A <= 0)
