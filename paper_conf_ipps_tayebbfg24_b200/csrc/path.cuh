@@ -89,39 +89,30 @@ struct BlStage {          // one staged level: its CSR slice in the shared-memor
     int32_t charge;       // arena words the level holds (its copies + any wrap-around gap)
 };
 
-constexpr int BL_NB = 16;       // k_bl_small: levels staged ahead of the walk, at most
-constexpr int BL_LTAB = 4096;   // level-bound table in shared memory for L < BL_LTAB
-
-__global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
-                                                   const int32_t* __restrict__ nodeq,
-                                                   const int32_t* __restrict__ rowq,
-                                                   const int32_t* __restrict__ colq, DurView d, float* bl,
-                                                   float* cp, uint32_t* err, int32_t arena_words) {
-    extern __shared__ __align__(16) float sbl[];
-    __shared__ __align__(8) uint64_t bars[BL_NB];
-    __shared__ BlStage stg[BL_NB];
-    bool bad = false;
-    float cpm = 0.0f;
-    const int32_t t = (int32_t)threadIdx.x;
-    const int32_t nq = __ldg(lvlq + L);
-    // after sbl: the level-bound table (q start and edge start of every level, when L is
-    // small enough), then the staging arena (arena_words int32, a ring: levels are staged
-    // in order and released in order; 0: no staging)
-    const bool tab = L < BL_LTAB;
-    int32_t* lq = reinterpret_cast<int32_t*>(sbl + ((nq + 3) & ~3));      // [L + 1] q starts
-    int32_t* le = lq + (tab ? ((L + 1 + 3) & ~3) : 0);                      // [L + 1] edge starts
-    int32_t* arena = le + (tab ? ((L + 1 + 3) & ~3) : 0);
-    const int32_t A = arena_words & ~3;
-    const int32_t prod = (int32_t)blockDim.x - 1;   // producer thread: the last one
-    int32_t rn = 0, head = 0, used = 0;             // producer state: next level, ring head, words held
-    // producer: decide (and, space permitting, stage) levels ahead; every level <= r + 1
-    // must be decided before this returns (the walk reads its record after the next barrier)
-    auto advance = [&](int32_t r) {
-        while (rn < L && rn <= r + BL_NB - 1) {
-            const int b = rn % BL_NB;
+// Producer side of a level-by-level walk that stages each level's CSR slice (rowq, nodeq,
+// colq: contiguous q-space ranges) into a shared-memory ring arena with TMA bulk copies,
+// up to BL_NB levels ahead (k_bl_small, k_rep2_bl's level mode).  One thread calls
+// advance(r) at the start of level r (after the barrier that ended level r - 1): it
+// releases level r - 1's space, then decides -- and, space permitting, stages -- the
+// levels ahead; every level <= r + 1 is decided before it returns (the walk reads that
+// level's record after the next barrier).  A level that does not fit is read from L2.
+struct CsrStager {
+    int32_t* arena;
+    int32_t A;                       // arena words
+    BlStage* stg;                    // [BL_NB]
+    uint64_t* bars;                  // [BL_NB] mbarriers
+    const int32_t* lq;               // level q starts (shared, when tab) else null
+    const int32_t* le;               // level edge starts (shared, when tab) else null
+    int32_t L;
+    const int32_t *lvlq, *rowq, *nodeq, *colq;
+    int32_t rn, head, used;          // producer state
+    MP_INLINE void advance(int32_t r, int nb) {
+        if (r > 0) used -= stg[(r - 1) % nb].charge;      // level r - 1 is done
+        while (rn < L && rn <= r + nb - 1) {
+            const int b = rn % nb;
             BlStage& S = stg[b];
-            const int32_t qa = tab ? lq[rn] : __ldg(lvlq + rn), qb = tab ? lq[rn + 1] : __ldg(lvlq + rn + 1);
-            const int32_t e0 = tab ? le[rn] : __ldg(rowq + qa), e1 = tab ? le[rn + 1] : __ldg(rowq + qb);
+            const int32_t qa = lq ? lq[rn] : __ldg(lvlq + rn), qb = lq ? lq[rn + 1] : __ldg(lvlq + rn + 1);
+            const int32_t e0 = le ? le[rn] : __ldg(rowq + qa), e1 = le ? le[rn + 1] : __ldg(rowq + qb);
             // three 16-byte aligned copies: rowq[qa .. qb], nodeq[qa .. qb), colq[e0 .. e1)
             const int32_t ra = qa & ~3, rw = ((qb + 1 + 3) & ~3) - ra;
             const int32_t na = qa & ~3, nw = ((qb + 3) & ~3) - na;
@@ -153,7 +144,34 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
             S.ok = 1;
             rn++;
         }
-    };
+    }
+};
+
+constexpr int BL_NB = 16;       // k_bl_small: levels staged ahead of the walk, at most
+constexpr int BL_LTAB = 4096;   // level-bound table in shared memory for L < BL_LTAB
+
+__global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
+                                                   const int32_t* __restrict__ nodeq,
+                                                   const int32_t* __restrict__ rowq,
+                                                   const int32_t* __restrict__ colq, DurView d, float* bl,
+                                                   float* cp, uint32_t* err, int32_t arena_words) {
+    extern __shared__ __align__(16) float sbl[];
+    __shared__ __align__(8) uint64_t bars[BL_NB];
+    __shared__ BlStage stg[BL_NB];
+    bool bad = false;
+    float cpm = 0.0f;
+    const int32_t t = (int32_t)threadIdx.x;
+    const int32_t nq = __ldg(lvlq + L);
+    // after sbl: the level-bound table (q start and edge start of every level, when L is
+    // small enough), then the staging arena (arena_words int32, a ring: levels are staged
+    // in order and released in order; 0: no staging)
+    const bool tab = L < BL_LTAB;
+    int32_t* lq = reinterpret_cast<int32_t*>(sbl + ((nq + 3) & ~3));      // [L + 1] q starts
+    int32_t* le = lq + (tab ? ((L + 1 + 3) & ~3) : 0);                      // [L + 1] edge starts
+    int32_t* arena = le + (tab ? ((L + 1 + 3) & ~3) : 0);
+    const int32_t A = arena_words & ~3;
+    const int32_t prod = (int32_t)blockDim.x - 1;   // producer thread: the last one
+    CsrStager stager{arena, A, stg, bars, tab ? lq : nullptr, tab ? le : nullptr, L, lvlq, rowq, nodeq, colq, 0, 0, 0};
     {
         // the level walk reads every successor id and row bound once, a level at a time:
         // pull them into L2 now (one prefetch per 128-byte line) so no level waits on HBM
@@ -184,17 +202,14 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
         }
     }
     __syncthreads();
-    if (t == prod && A > 0) advance(-1);
+    if (t == prod && A > 0) stager.advance(-1, BL_NB);
     if (t == prod && A <= 0)
         for (int b = 0; b < BL_NB; b++) stg[b].ok = 0;
     __syncthreads();   // stg[] visible to every thread
     uint32_t ph = 0u;  // bit b: parity of buffer b's next phase
     for (int32_t r = 0; r < L; r++) {
         const int b = r % BL_NB;
-        if (t == prod && A > 0) {
-            if (r > 0) used -= stg[(r - 1) % BL_NB].charge;   // level r - 1 is done (barrier passed)
-            advance(r);
-        }
+        if (t == prod && A > 0) stager.advance(r, BL_NB);
         const BlStage S = stg[b];
         const int32_t qa = tab ? lq[r] : __ldg(lvlq + r), qb = tab ? lq[r + 1] : __ldg(lvlq + r + 1);
         if (A > 0 && S.ok) {
