@@ -1766,9 +1766,34 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     // (8-CTA clusters and a cross-CTA dataflow mode -- bl lines as ready flags polled from L2 --
     // measured slower: R = 512 K1 0.98 ms (4-CTA, level barriers) vs 1.58 ms (8-CTA) and
     // 1.06 ms (4-CTA dataflow); the per-group time is a latency floor of ~5 us per level)
+    // the largest cluster (<= 8 CTAs) with which every group's cluster is resident at once
+    // (a second wave of clusters would double K1); 1 when the groups alone fill the SMs
     int cs = 1;
-    while (cs < 4 && groups * (cs * 2) <= dag->num_sms) cs *= 2;
-    for (;; cs /= 2) {
+    for (int c = 8; c >= 2; c--) {
+        if (groups * c > dag->num_sms) continue;
+        cudaLaunchConfig_t q = {};
+        q.gridDim = dim3((unsigned)(groups * c));
+        q.blockDim = dim3(R2_THREADS);
+        q.dynamicSmemBytes = (size_t)smem1;
+        q.stream = st;
+        cudaLaunchAttribute qa[1];
+        qa[0].id = cudaLaunchAttributeClusterDimension;
+        qa[0].val.clusterDim.x = (unsigned)c;
+        qa[0].val.clusterDim.y = 1;
+        qa[0].val.clusterDim.z = 1;
+        q.attrs = qa;
+        q.numAttrs = 1;
+        int mac = 0;
+        if (cudaOccupancyMaxActiveClusters(&mac, k_rep2_bl<A>, &q) != cudaSuccess) {
+            cudaGetLastError();
+            continue;
+        }
+        if (mac >= groups) {
+            cs = c;
+            break;
+        }
+    }
+    for (;; cs = cs > 1 ? cs - 1 : 1) {
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3((unsigned)(groups * cs));
         cfg.blockDim = dim3(R2_THREADS);
