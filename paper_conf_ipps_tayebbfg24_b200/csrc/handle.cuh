@@ -44,8 +44,6 @@ struct mp_dag {
     unsigned long long* scan_status = nullptr;
     size_t scan_status_cap = 0;
     uint32_t* tickets = nullptr; // [64]
-    uint32_t sort_epoch = 0;
-    uint32_t scan_epoch = 0;
     int num_sms = 148;
     // build scratch (grow-only, reused by mp_dag_rebuild)
     int32_t* b_rem = nullptr;
@@ -165,8 +163,10 @@ inline mp_status ensure_scan_status(mp_dag* dag, size_t entries, cudaStream_t st
 inline mp_status scan(mp_dag* dag, const int32_t* in, int32_t* out, int64_t n, int32_t* d_total,
                       cudaStream_t st) {
     MP_TRY(ensure_scan_status(dag, (size_t)((n + mpk::SCAN_TILE - 1) / mpk::SCAN_TILE) + 1, st));
-    mpk::ScanWs w{dag->scan_status, dag->tickets + 63};
-    MP_CUDA(mpk::scan_excl(in, out, n, d_total, w, dag->scan_epoch, st));
+    // the last status word is the device epoch counter (zeroed with the array)
+    mpk::ScanWs w{dag->scan_status, dag->tickets + 63,
+                  reinterpret_cast<uint32_t*>(dag->scan_status + dag->scan_status_cap - 1)};
+    MP_CUDA(mpk::scan_excl(in, out, n, d_total, w, st));
     return MP_OK;
 }
 
@@ -206,7 +206,8 @@ inline mp_status run_sort(mp_dag* dag, mpk::SortArgs& a, cudaStream_t st) {
     int64_t tps = (a.seg_len + mpk::SORT_TILE - 1) / mpk::SORT_TILE;
     MP_TRY(ensure_sort_status(dag, (size_t)(tps * a.nseg) * 256, st));
     a.status = dag->sort_status;
-    MP_CUDA(mpk::sort_launch(a, dag->sort_epoch, st));
+    a.depoch = reinterpret_cast<uint32_t*>(dag->sort_status + dag->sort_status_cap - 1);   // zeroed with it
+    MP_CUDA(mpk::sort_launch(a, st));
     return MP_OK;
 }
 

@@ -669,11 +669,11 @@ __global__ void k_q_scatter(int32_t n, int32_t A, const uint64_t* key, const int
     }
 }
 
-__global__ void k_q_out(const SortPlan* plan, uint32_t* const* vb, const int32_t* total, int32_t A,
+__global__ void k_q_out(const SortPlan* plan, const uint32_t* vb0, const uint32_t* vb1, const int32_t* total, int32_t A,
                         const int32_t* counts, const unsigned long long* brw, int64_t* qptr, int32_t* qtask,
                         mp_queue_summary* sum) {
     const int32_t Q = *total;
-    const uint32_t* v = Q > 0 ? vb[plan->final_sel] : nullptr;
+    const uint32_t* v = Q > 0 ? (plan->final_sel ? vb1 : vb0) : nullptr;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < Q; i += (int64_t)gridDim.x * blockDim.x)
         qtask[i] = (int32_t)v[i];
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -837,13 +837,10 @@ inline mp_status build_queues(mp_dag* dag, int32_t A, const uint64_t* key, const
     int32_t* counts = ar.take<int32_t>(MAX_ARCH);
     unsigned long long* brw = ar.take<unsigned long long>(2 * MAX_ARCH);
     int32_t* total = ar.take<int32_t>(2);
-    uint32_t** vb = ar.take<uint32_t*>(2);
     int64_t* dlen = ar.take<int64_t>(1);
     MP_CUDA(cudaMemsetAsync(counts, 0, 4 * MAX_ARCH, st));
     MP_CUDA(cudaMemsetAsync(brw, 0, 16 * MAX_ARCH, st));
     MP_CUDA(cudaMemsetAsync(total, 0, 8, st));
-    uint32_t* hv[2] = {sa.vals[0], sa.vals[1]};
-    MP_CUDA(cudaMemcpyAsync(vb, hv, sizeof(hv), cudaMemcpyHostToDevice, st));
     if (n > 0) {
         if (done) {
             MP_CUDA(cudaMemsetAsync(blocked, 0, (size_t)n, st));
@@ -859,7 +856,8 @@ inline mp_status build_queues(mp_dag* dag, int32_t A, const uint64_t* key, const
         MP_LAUNCH(k_copy_len, 1, 1, 0, st, total, dlen);
         MP_TRY(run_sort(dag, sa, st));
     }
-    MP_LAUNCH(k_q_out, grid_for(nA > 0 ? nA : 1), 256, 0, st, sa.plans, vb, total, A, counts, brw, qptr, qtask, sum);
+    MP_LAUNCH(k_q_out, grid_for(nA > 0 ? nA : 1), 256, 0, st, sa.plans, sa.vals[0], sa.vals[1], total, A, counts, brw,
+              qptr, qtask, sum);
     MP_CUDA(cudaGetLastError());
     return MP_OK;
 }

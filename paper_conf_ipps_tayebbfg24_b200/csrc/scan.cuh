@@ -13,10 +13,18 @@ constexpr int SCAN_TILE = SCAN_THREADS * SCAN_IPT;
 struct ScanWs {
     unsigned long long* status;   // [ntiles], zeroed once
     uint32_t* ticket;             // [1]
+    uint32_t* depoch;             // device scan counter (status tags; graph-replay safe)
 };
 
+// before a scan: reset the tile ticket and bump the epoch (one thread)
+__global__ void k_scan_prep(ScanWs ws) {
+    *ws.ticket = 0u;
+    *ws.depoch = *ws.depoch + 1u;
+}
+
 __global__ void __launch_bounds__(SCAN_THREADS)
-k_scan_excl(const int32_t* in, int32_t* out, int64_t n, int32_t* total, ScanWs ws, uint32_t epoch) {
+k_scan_excl(const int32_t* in, int32_t* out, int64_t n, int32_t* total, ScanWs ws) {
+    const uint32_t epoch = *(volatile uint32_t*)ws.depoch & 0x3fffffffu;
     __shared__ uint32_t tile_sh;
     __shared__ int32_t wsum[SCAN_THREADS / 32];
     __shared__ int64_t excl_sh;
@@ -78,16 +86,14 @@ k_scan_excl(const int32_t* in, int32_t* out, int64_t n, int32_t* total, ScanWs w
 }
 
 inline cudaError_t scan_excl(const int32_t* in, int32_t* out, int64_t n, int32_t* d_total, ScanWs ws,
-                             uint32_t& epoch, cudaStream_t st) {
+                             cudaStream_t st) {
     if (n <= 0) {
         if (d_total) return cudaMemsetAsync(d_total, 0, sizeof(int32_t), st);
         return cudaSuccess;
     }
-    cudaError_t e = cudaMemsetAsync(ws.ticket, 0, sizeof(uint32_t), st);
-    if (e) return e;
-    epoch++;
+    MP_LAUNCH(k_scan_prep, 1, 1, 0, st, ws);
     int64_t ntiles = (n + SCAN_TILE - 1) / SCAN_TILE;
-    MP_LAUNCH(k_scan_excl, (unsigned)ntiles, SCAN_THREADS, 0, st, in, out, n, d_total, ws, epoch & 0x3fffffffu);
+    MP_LAUNCH(k_scan_excl, (unsigned)ntiles, SCAN_THREADS, 0, st, in, out, n, d_total, ws);
     return cudaGetLastError();
 }
 

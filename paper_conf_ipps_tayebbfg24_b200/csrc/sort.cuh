@@ -45,6 +45,7 @@ struct SortArgs {
     unsigned long long* status;        // [nseg*tiles_per_seg][256]
     uint32_t* tickets;                 // [npass]
     const int64_t* d_len;              // optional device-side length (<= seg_len), all segments
+    uint32_t* depoch;                  // device sort counter (the status tags; graph-replay safe)
 };
 
 MP_INLINE int64_t eff_len(const SortArgs& a) {
@@ -83,6 +84,7 @@ __global__ void k_sort_plan(SortArgs a) {
     int s = blockIdx.x;
     int d = threadIdx.x;
     if (s == 0 && d < a.npass) a.tickets[d] = 0;
+    if (s == 0 && d == 0) *a.depoch = *a.depoch + 1u;   // this sort's epochs: depoch * 8 + pass
     int sel = 0;
     const int64_t len = eff_len(a);
     for (int p = 0; p < a.npass; p++) {
@@ -111,7 +113,10 @@ __global__ void k_sort_plan(SortArgs a) {
 constexpr uint64_t ST_AGG = 1ull << 32;
 constexpr uint64_t ST_PRE = 2ull << 32;
 
-__global__ void __launch_bounds__(SORT_THREADS) k_sort_pass(SortArgs a, int pass, uint32_t epoch) {
+__global__ void __launch_bounds__(SORT_THREADS) k_sort_pass(SortArgs a, int pass) {
+    // status tags come from a device counter bumped once per sort by k_sort_plan, so a
+    // replayed CUDA graph never meets its previous replay's tags
+    const uint32_t epoch = (*(volatile uint32_t*)a.depoch * (uint32_t)SORT_MAX_PASS + (uint32_t)pass) & 0x3fffffffu;
     __shared__ uint32_t whist[SORT_WARPS][256];
     __shared__ uint32_t tstart[256];       // digit start within the tile
     __shared__ int64_t gdelta[256];        // global position = gdelta[d] + tile-local index
@@ -250,10 +255,10 @@ __global__ void __launch_bounds__(SORT_THREADS) k_sort_pass(SortArgs a, int pass
 
 inline size_t sort_plan_bytes(int nseg) { return (size_t)nseg * sizeof(SortPlan); }
 
-// Launch the whole sort. hist must be zeroed (done here); status must be
-// zero-initialised once at allocation; epoch is a per-workspace counter that
-// grows by npass per call.
-inline cudaError_t sort_launch(SortArgs a, uint32_t& epoch, cudaStream_t st) {
+// Launch the whole sort. hist must be zeroed (done here); status (and the device epoch
+// counter a.depoch) must be zero-initialised once at allocation.  No host state: the
+// launch sequence can be captured in a CUDA graph and replayed.
+inline cudaError_t sort_launch(SortArgs a, cudaStream_t st) {
     if (a.seg_len <= 0 || a.nseg <= 0 || a.npass <= 0) return cudaSuccess;
     a.tiles_per_seg = (int32_t)((a.seg_len + SORT_TILE - 1) / SORT_TILE);
     cudaError_t e = cudaMemsetAsync(a.hist, 0, (size_t)a.nseg * a.npass * 256 * sizeof(uint32_t), st);
@@ -269,10 +274,7 @@ inline cudaError_t sort_launch(SortArgs a, uint32_t& epoch, cudaStream_t st) {
         e = cudaFuncSetAttribute(k_sort_pass, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
         if (e) return e;
     }
-    for (int p = 0; p < a.npass; p++) {
-        epoch++;
-        MP_LAUNCH(k_sort_pass, (unsigned)ntiles, SORT_THREADS, dyn, st, a, p, epoch & 0x3fffffffu);
-    }
+    for (int p = 0; p < a.npass; p++) MP_LAUNCH(k_sort_pass, (unsigned)ntiles, SORT_THREADS, dyn, st, a, p);
     return cudaGetLastError();
 }
 

@@ -592,3 +592,46 @@ def test_random_sweep_single_dag_and_replicas():
         R = int(rng.integers(1, 70))
         _replica_check(W, R, int(rng.integers(0, 10000)), sorted(set([0, R - 1, R // 2])),
                        sigma=float(rng.choice([0.0, 0.0625, 0.125, 0.25])), seed=int(rng.integers(0, 2**62)))
+
+
+@pytest.mark.parametrize("name", ["c1", "c2", "c4fmm", "hier"])
+def test_score_path_cuda_graph_replay(name):
+    """The single-DAG score path has no host state across calls (device-side sort / scan
+    epochs), so bench.py captures it in a CUDA graph: every replay must give the oracle's
+    bytes (k_bl_small / k_bl_wide / k_bl_flow, the queue sort, the scans)."""
+    w = workloads.config(name)
+    dag = mp.build_dag(w.n, to_dev(w.src, torch.int32), to_dev(w.dst, torch.int32))
+    dur = to_dev(w.dur)
+    n, A = w.dur.shape
+    o = dict(bl=dict(bl=torch.empty(n, dtype=torch.float32, device=DEV), cp=torch.empty(1, dtype=torch.float32, device=DEV),
+                     nod=None),
+             aff=dict(gain=torch.empty((n, A), dtype=torch.float32, device=DEV), hd=torch.empty(A, dtype=torch.float32, device=DEV),
+                      flags=torch.empty((n, A), dtype=torch.uint8, device=DEV)),
+             sc=dict(crit_norm=torch.empty(n, dtype=torch.float32, device=DEV), key=torch.empty((n, A), dtype=torch.int64, device=DEV)),
+             q=dict(qptr=torch.empty(A + 1, dtype=torch.int64, device=DEV), qtask=torch.empty(n * A, dtype=torch.int32, device=DEV),
+                    summary=torch.empty(A * mp.SUMMARY_BYTES, dtype=torch.uint8, device=DEV)))
+
+    def step():
+        bl, cp, _ = mp.bottom_level(dag, dur, w.workers, out=o["bl"])
+        gain, hd, flags = mp.affinity(dag, dur, w.workers, out=o["aff"])
+        cn, key = mp.score(dag, 0, bl, gain, flags, out=o["sc"])
+        mp.build_queues(dag, key, flags, dur, out=o["q"])
+
+    for _ in range(2):
+        step()
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        step()
+    od = oracle.build_dag(w.n, w.src, w.dst)
+    ref = oracle.score_and_queue(od, w.dur, w.workers)
+    Q = int(ref["qptr"][-1])
+    for _ in range(3):
+        o["q"]["qtask"].fill_(-1)
+        g.replay()
+        torch.cuda.synchronize()
+        mp.check(dag)
+        assert np.array_equal(bits(o["bl"]["bl"].cpu().numpy()), bits(ref["bl"]))
+        assert np.array_equal(o["q"]["qptr"].cpu().numpy(), ref["qptr"])
+        assert np.array_equal(o["q"]["qtask"].cpu().numpy()[:Q], ref["qtask"])
+        assert o["q"]["summary"].cpu().numpy().tobytes() == ref["summary"].tobytes()
