@@ -17,6 +17,8 @@
 //                   there; ranges with one key value are streamed in order.
 // Bit-exact with the oracle: same RN ops as path.cuh / replicas.cuh.
 #pragma once
+#include <map>
+#include <mutex>
 #include "replicas.cuh"
 
 namespace mpk {
@@ -1768,8 +1770,20 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     // 1.06 ms (4-CTA dataflow); the per-group time is a latency floor of ~5 us per level)
     // the largest cluster (<= 8 CTAs) with which every group's cluster is resident at once
     // (a second wave of clusters would double K1); 1 when the groups alone fill the SMs
+    // (memoised per device and group count: the occupancy queries cost host time every call)
+    static std::mutex cs_mu;
+    static std::map<std::pair<int, int64_t>, int> cs_memo;
     int cs = 1;
-    for (int c = 8; c >= 2; c--) {
+    bool memo_hit = false;
+    {
+        std::lock_guard<std::mutex> lk(cs_mu);
+        auto it = cs_memo.find({dag->device, groups * 8 + A});
+        if (it != cs_memo.end()) {
+            cs = it->second;
+            memo_hit = true;
+        }
+    }
+    for (int c = 8; c >= 2 && !memo_hit; c--) {
         if (groups * c > dag->num_sms) continue;
         cudaLaunchConfig_t q = {};
         q.gridDim = dim3((unsigned)(groups * c));
@@ -1792,6 +1806,10 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
             cs = c;
             break;
         }
+    }
+    if (!memo_hit) {
+        std::lock_guard<std::mutex> lk(cs_mu);
+        cs_memo[{dag->device, groups * 8 + A}] = cs;
     }
     for (;; cs = cs > 1 ? cs - 1 : 1) {
         cudaLaunchConfig_t cfg = {};
