@@ -150,12 +150,18 @@ struct CsrStager {
 constexpr int BL_NB = 16;       // k_bl_small: levels staged ahead of the walk, at most
 constexpr int BL_LTAB = 4096;   // level-bound table in shared memory for L < BL_LTAB
 
+// GBL = false: bl of every position in shared memory (n <= SMALL_CAP).  GBL = true
+// (k_bl_one, medium DAGs with moderate edge counts): the same single-CTA walk with bl in
+// a q-indexed global array `blg` (L2-resident; the block barrier orders a level's stores
+// before the next level's loads), so the whole shared memory holds the staging arena.
+template <bool GBL>
 __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __restrict__ lvlq,
                                                    const int32_t* __restrict__ nodeq,
                                                    const int32_t* __restrict__ rowq,
                                                    const int32_t* __restrict__ colq, DurView d, float* bl,
-                                                   float* cp, uint32_t* err, int32_t arena_words) {
-    extern __shared__ __align__(16) float sbl[];
+                                                   float* cp, uint32_t* err, int32_t arena_words, float* blg) {
+    extern __shared__ __align__(16) float sdyn[];
+    float* sbl = GBL ? blg : sdyn;
     __shared__ __align__(8) uint64_t bars[BL_NB];
     __shared__ BlStage stg[BL_NB];
     bool bad = false;
@@ -166,7 +172,7 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
     // small enough), then the staging arena (arena_words int32, a ring: levels are staged
     // in order and released in order; 0: no staging)
     const bool tab = L < BL_LTAB;
-    int32_t* lq = reinterpret_cast<int32_t*>(sbl + ((nq + 3) & ~3));      // [L + 1] q starts
+    int32_t* lq = reinterpret_cast<int32_t*>(GBL ? sdyn : sdyn + ((nq + 3) & ~3));   // [L + 1] q starts
     int32_t* le = lq + (tab ? ((L + 1 + 3) & ~3) : 0);                      // [L + 1] edge starts
     int32_t* arena = le + (tab ? ((L + 1 + 3) & ~3) : 0);
     const int32_t A = arena_words & ~3;
@@ -270,6 +276,10 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
 #endif
 constexpr int32_t BL_WIDE_MIN = MP_BL_WIDE_MIN;   // mean level width (n / L) that selects k_bl_wide
 constexpr int BL_WIDE_THREADS = 512;
+#ifndef MP_BL_ONE_MAX_E
+#define MP_BL_ONE_MAX_E (1 << 20)
+#endif
+constexpr int64_t BL_ONE_MAX_E = MP_BL_ONE_MAX_E;   // k_bl_one: one SM's issue budget for the edges
 
 __global__ void __launch_bounds__(BL_WIDE_THREADS) k_bl_wide(int32_t L, const int32_t* __restrict__ lvlq,
                                                               const int32_t* __restrict__ nodeq,
@@ -727,9 +737,25 @@ inline mp_status bottom_level(mp_dag* dag, int32_t A, const float* dur, const in
         const size_t smem = sbytes + tbytes + (size_t)arena_words * 4;
         static std::atomic<uint64_t> attr{0};
         if (first_on_device(attr))
-            MP_CUDA(cudaFuncSetAttribute(k_bl_small, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - 1024));
-        MP_LAUNCH(k_bl_small, 1, 1024, smem, st, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp, dag->err,
-                  arena_words);
+            MP_CUDA(cudaFuncSetAttribute(k_bl_small<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - 1024));
+        MP_LAUNCH(k_bl_small<false>, 1, 1024, smem, st, dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp,
+                  dag->err, arena_words, (float*)nullptr);
+    } else if (dag->E <= BL_ONE_MAX_E && (int64_t)n < (int64_t)BL_WIDE_MIN * dag->L) {
+        // medium DAG, moderate edge count: one CTA, bl in L2, CSR staged in shared memory
+        int optin = 0;
+        MP_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dag->device));
+        MP_TRY(ensure_ws(dag, align256((size_t)n * 4), st));
+        float* blg = (float*)dag->ws;
+        const size_t tbytes = dag->L < BL_LTAB ? (size_t)2 * (((dag->L + 1) + 3) & ~3) * 4 : 0;
+        const int64_t avail = (int64_t)optin - (int64_t)tbytes - 1024;
+        const int32_t arena_words = avail >= 4096 ? (int32_t)((avail / 4) & ~3) : 0;
+        const size_t smem = tbytes + (size_t)arena_words * 4;
+        static std::atomic<uint64_t> attr1{0};
+        if (first_on_device(attr1))
+            MP_CUDA(cudaFuncSetAttribute(k_bl_small<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - 1024));
+        mph::ProfScope ps("k_bl_one", st);
+        k_bl_small<true><<<1, 1024, smem, st>>>(dag->L, dag->lvlq, dag->nodeq, dag->rowq, dag->colq, d, bl, cp, dag->err,
+                                               arena_words, blg);
     } else if (dag->L > 0 && (int64_t)n >= (int64_t)BL_WIDE_MIN * dag->L) {
         // few, wide levels: level-synchronous edge-parallel cooperative kernel
         const int32_t nq = n;
