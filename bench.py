@@ -585,6 +585,9 @@ def run_ours(args):
     #      libmp keeps no host state across the calls: device-side sort/scan epochs) ----
     graph = None
     if cfg in SINGLE_CFGS and not args.eager:
+        if args.warmup < 1:   # one eager pass first: workspaces grow outside the capture
+            step()
+            torch.cuda.synchronize()
         l0 = mp.launch_count()
         graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(graph):
