@@ -100,6 +100,11 @@ MP_INLINE void r2_durs(const Rep2Args& a, int64_t r, int32_t t, float (&x)[A], u
 // ---------------------------------------------------------------------------------------
 // K1
 // ---------------------------------------------------------------------------------------
+#ifndef MP_K1_PF
+#define MP_K1_PF 8
+#endif
+constexpr int K1_PF = MP_K1_PF;   // successor-line gathers in flight per lane
+
 template <int A>
 // A 32-replica group is run by a cluster of `cs` CTAs (cs = 1 when there are enough
 // groups to fill the GPU; up to 8 for small per-GPU replica counts): the nodes of a
@@ -253,29 +258,29 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_bl(Rep2Args a) {
             }
             if (!k) wt = 0.0f;
             }
-            // successors: 32 positions per coalesced load, broadcast by shuffles, gathers 8 at a time
+            // successors: 32 positions per coalesced load, broadcast by shuffles, gathers K1_PF at a time
             float m = 0.0f;
             for (int32_t eb = e0; eb < e1; eb += 32) {
                 const int32_t cb = min(32, e1 - eb);
                 const int32_t s32 = eb == e0 ? sv : (lane < cb ? __ldg(a.colq + eb + lane) : 0);
                 int32_t j = 0;
-                for (; j + 8 <= cb; j += 8) {
-                    float t8[8];
+                for (; j + K1_PF <= cb; j += K1_PF) {
+                    float t8[K1_PF];
                     if (flow) {
 #pragma unroll
-                        for (int u = 0; u < 8; u++) {
+                        for (int u = 0; u < K1_PF; u++) {
                             const int32_t sp = __shfl_sync(0xffffffffu, s32, j + u);
                             while (rdy[sp] == 0) {}
                         }
                         __threadfence_block();
                     }
 #pragma unroll
-                    for (int u = 0; u < 8; u++) {
+                    for (int u = 0; u < K1_PF; u++) {
                         const int32_t sp = __shfl_sync(0xffffffffu, s32, j + u);
                         t8[u] = bll[sp * 32];
                     }
 #pragma unroll
-                    for (int u = 0; u < 8; u++) m = fmaxf(m, t8[u]);
+                    for (int u = 0; u < K1_PF; u++) m = fmaxf(m, t8[u]);
                 }
                 for (; j < cb; j++) {
                     const int32_t sp = __shfl_sync(0xffffffffu, s32, j);

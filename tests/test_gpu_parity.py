@@ -164,6 +164,19 @@ def test_layered_skewed_fanin():
     compare(n, s, d, random_dags.dyadic_durations(n, 2, 9, tiny_set=True), np.ones(2, np.int32))
 
 
+def test_medium_dags_many_edges():
+    """Medium DAGs past k_bl_one's edge budget (1 Mi < E <= 8 Mi, the dataflow kernel):
+    levels narrower than a warp next to 30,000-wide levels with up to 60 predecessors per
+    task, and a random deep DAG (39,108 levels) with three archs and ties."""
+    n, s, d = random_dags.layered_dag([1, 3, 30000, 2, 30000, 30000, 30000, 1, 16, 9000, 17, 5], fan=60, seed=41)
+    g = compare(n, s, d, random_dags.dyadic_durations(n, 2, 41, tiny_set=True), np.ones(2, np.int32))
+    assert 1 << 20 < g["dag"].n_edges <= 8 << 20
+    n = 300000
+    s, d = random_dags.random_dag(n, 5.0, 42, dup=0.1, max_span=64)
+    g = compare(n, s, d, random_dags.dyadic_durations(n, 3, 42, p_inf=0.2, tiny_set=True), np.ones(3, np.int32))
+    assert 1 << 20 < g["dag"].n_edges <= 8 << 20
+
+
 def test_empty_and_edgeless():
     compare(0, np.zeros(0, np.int32), np.zeros(0, np.int32), np.zeros((0, 2), np.float32), np.ones(2, np.int32))
     n = 5000
