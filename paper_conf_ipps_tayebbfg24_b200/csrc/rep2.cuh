@@ -1509,6 +1509,9 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             }
             __syncthreads();
             const bool mfit = s_mtot <= ccap;
+#ifdef MP_PHASES
+            if (threadIdx.x == 0) atomicAdd(&g_k2_phase[20], (unsigned long long)s_mtot);
+#endif
             if (mfit) {
 #pragma unroll
                 for (int h = 0; h < 2; h++) {
@@ -1547,18 +1550,40 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 return crs[mp[i >> 5] + __popc(m & ((1u << (i & 31)) - 1u))];
             };
             auto bit = [&](const uint32_t* e, int32_t i) -> bool { return (e[i >> 5] >> (i & 31)) & 1u; };
-            if (mfit) {   // positions in no equal-gain run go straight to both queues (coalesced)
-                for (int32_t p = threadIdx.x; p < a.n; p += R2_THREADS) {
-                    if ((mw[p >> 5] >> (p & 31)) & 1u) continue;
-                    const uint32_t t = Ps[p];
-                    if (p < cG) {
-                        if (p == 0) s_h1 = t;
-                        if (q1) __stcs(q1 + p, (int32_t)t);
+            if (mfit) {   // positions in no equal-gain run go straight to both queues (coalesced):
+                          // 4 consecutive positions per thread, 16-byte stores where aligned
+                const bool v1 = q1 && ((reinterpret_cast<uintptr_t>(q1) & 15u) == 0u);
+                const bool v0 = q0 && ((a.n & 3) == 0) && ((reinterpret_cast<uintptr_t>(q0) & 15u) == 0u);
+                for (int32_t p4 = 4 * (int32_t)threadIdx.x; p4 < a.n; p4 += 4 * R2_THREADS) {
+                    const uint32_t mb = (mw[p4 >> 5] >> (p4 & 31)) & 0xFu;
+                    uint32_t tt[4];
+                    if (p4 + 4 <= a.n) {
+                        const uint2 v = *reinterpret_cast<const uint2*>(Ps + p4);
+                        tt[0] = v.x & 0xFFFFu; tt[1] = v.x >> 16; tt[2] = v.y & 0xFFFFu; tt[3] = v.y >> 16;
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 4; j++) tt[j] = p4 + j < a.n ? Ps[p4 + j] : 0u;
                     }
-                    if (p >= n1only) {
-                        if (p == a.n - 1) s_h0 = t;
-                        if (q0) __stcs(q0 + (a.n - 1 - p), (int32_t)t);
+                    if (p4 == 0 && !(mb & 1u) && cG > 0) s_h1 = tt[0];
+                    if (v1 && mb == 0u && p4 + 4 <= cG) {
+                        __stcs(reinterpret_cast<int4*>(q1 + p4), make_int4((int)tt[0], (int)tt[1], (int)tt[2], (int)tt[3]));
+                    } else if (q1) {
+#pragma unroll
+                        for (int j = 0; j < 4; j++)
+                            if (p4 + j < cG && !((mb >> j) & 1u)) __stcs(q1 + p4 + j, (int32_t)tt[j]);
                     }
+                    if (v0 && mb == 0u && p4 >= n1only && p4 + 4 <= a.n) {
+                        __stcs(reinterpret_cast<int4*>(q0 + (a.n - 4 - p4)), make_int4((int)tt[3], (int)tt[2], (int)tt[1], (int)tt[0]));
+                    } else if (q0) {
+#pragma unroll
+                        for (int j = 0; j < 4; j++) {
+                            const int32_t p = p4 + j;
+                            if (p < a.n && p >= n1only && !((mb >> j) & 1u)) __stcs(q0 + (a.n - 1 - p), (int32_t)tt[j]);
+                        }
+                    }
+#pragma unroll
+                    for (int j = 0; j < 4; j++)
+                        if (p4 + j == a.n - 1 && !((mb >> j) & 1u)) s_h0 = tt[j];
                 }
             }
             // members (all positions when they did not fit): rank inside their runs

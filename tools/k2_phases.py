@@ -30,3 +30,4 @@ names = {1: "P0 hash+D+minmax", 2: "pass1 coarse hist", 3: "sub-bins", 4: "pass2
 tot = buf.sum()
 for i in sorted(names):
     print(f"{names[i]:28s} {100.0 * buf[i] / tot:5.1f}%  {buf[i] / R / 1.965e3:8.2f} us/replica")
+print(f"deferred positions per replica {buf[20] / R:8.1f}   near-tie pairs per replica {buf[21] / R:8.1f}")
