@@ -1090,12 +1090,16 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     // With one fixed range every replica has the same coarse bins, and the sub-bin geometry
     // built for this CTA's first replica is reused: later replicas bin their keys while
     // hashing (P0) and skip the sorter's two histogram passes.
-    __shared__ uint32_t s_flo, s_fhi, s_geo_ok, s_geo_nfb, s_out;
+    __shared__ uint32_t s_flo, s_fhi, s_geo_ok, s_geo_nfb, s_out, s_fast;
     unsigned char* geo = a.s_geo ? a.s_geo + (int64_t)blockIdx.x * R3_GEO_BYTES : nullptr;
     if constexpr (A == 2) {
-        if (threadIdx.x == 0) { s_flo = ~0u; s_fhi = 0u; s_geo_ok = 0u; s_geo_nfb = 0u; }
+        if (threadIdx.x == 0) {
+            s_flo = ~0u; s_fhi = 0u; s_geo_ok = 0u; s_geo_nfb = 0u;
+            s_fast = (a.emask == 3u && (reinterpret_cast<uintptr_t>(a.base) & 15u) == 0u) ? 1u : 0u;
+        }
         __syncthreads();
         uint32_t lo = ~0u, hi = 0u;
+        bool dom = true;   // every extreme a nonzero finite domain value (K1's fast-path rule)
         for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
             float xl[2], xh[2];
             uint32_t enl = 0, enh = 0;
@@ -1107,6 +1111,8 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 const float e1 = canon_dur(perturb_u(bv, a.sigma, 0xFFFFFFu), dummy);
                 xl[b] = e0 < e1 ? e0 : e1;
                 xh[b] = e0 < e1 ? e1 : e0;
+                const uint32_t ul = f2u(xl[b]), uh = f2u(xh[b]);
+                if (!(ul >= 0x2B000000u && ul < 0x49800000u && uh >= 0x2B000000u && uh < 0x49800000u)) dom = false;
                 if (((a.emask >> b) & 1u) && !is_inf(xl[b])) enl |= 1u << b;
                 if (((a.emask >> b) & 1u) && !is_inf(xh[b])) enh |= 1u << b;
             }
@@ -1125,9 +1131,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         }
         lo = __reduce_min_sync(0xffffffffu, lo);
         hi = __reduce_max_sync(0xffffffffu, hi);
+        dom = __all_sync(0xffffffffu, dom);
         if ((threadIdx.x & 31) == 0) {
             atomicMin(&s_flo, lo);
             atomicMax(&s_fhi, hi);
+            if (!dom) atomicAnd(&s_fast, 0u);
         }
         __syncthreads();
         if (threadIdx.x == 0 && s_flo > s_fhi) { s_flo = 0u; s_fhi = 0xFFFFFFFFu; }
@@ -1208,7 +1216,51 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             };
             const bool al = (reinterpret_cast<uintptr_t>(a.base) & 15u) == 0;
             const int32_t n2 = al ? (a.n & ~1) : 0;
-            for (int32_t t0 = 2 * threadIdx.x; t0 < n2; t0 += 4 * R2_THREADS) {
+            if (s_fast) {
+                // fast path (decided per launch, as K1's): both archs enabled everywhere and no
+                // perturbed duration can be 0, inf or outside the domain, so canonicalisation,
+                // enabled masks and sentinels drop out; the splitmix64 state of (r, t, arch 0),
+                // seed + ((r n + t) 2 + 1) golden, is walked by additions
+                auto onef = [&](int32_t t, float b0v, float b1v, uint64_t X) {
+                    const float x0 = perturb_x(b0v, X, a.sigma), x1 = perturb_x(b1v, X + SPLITMIX_GOLDEN, a.sigma);
+                    const uint32_t db = f2u(__fsub_rn(x1, x0));
+                    const uint32_t D = (db >> 31) ? ~db : (db | 0x80000000u);
+                    dkey[t] = D;
+                    dmn = min(dmn, D);
+                    dmx = max(dmx, D);
+                    if (pre) {
+                        const uint64_t key = (uint64_t)D << 32;
+                        uint32_t f = 0xFFFFu;
+                        if (key < gf.lo || key > gf.hi) {
+                            outside = true;
+                        } else {
+                            f = r3_bin32(S, gf, D);
+                            atomicAdd(&S.starts[f], 1u);
+                        }
+                        fbuf[t] = (uint16_t)f;
+                    }
+                };
+                constexpr uint64_t G2 = 2ull * SPLITMIX_GOLDEN;
+                uint64_t X = a.seed + ((uint64_t)r * (uint64_t)a.n * 2u + 1u) * SPLITMIX_GOLDEN +
+                             (uint64_t)(2 * threadIdx.x) * G2;
+                for (int32_t t0 = 2 * threadIdx.x; t0 < n2; t0 += 4 * R2_THREADS, X += (uint64_t)(4 * R2_THREADS) * G2) {
+                    const int32_t t1 = t0 + 2 * R2_THREADS;
+                    const float4 v0 = __ldg(reinterpret_cast<const float4*>(a.base) + (t0 >> 1));
+                    float4 v1 = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (t1 < n2) v1 = __ldg(reinterpret_cast<const float4*>(a.base) + (t1 >> 1));
+                    onef(t0, v0.x, v0.y, X);
+                    onef(t0 + 1, v0.z, v0.w, X + G2);
+                    if (t1 < n2) {
+                        const uint64_t X1 = X + (uint64_t)(2 * R2_THREADS) * G2;
+                        onef(t1, v1.x, v1.y, X1);
+                        onef(t1 + 1, v1.z, v1.w, X1 + G2);
+                    }
+                }
+                for (int32_t t = n2 + threadIdx.x; t < a.n; t += R2_THREADS)
+                    onef(t, __ldg(a.base + 2 * (int64_t)t), __ldg(a.base + 2 * (int64_t)t + 1),
+                         a.seed + (((uint64_t)r * (uint64_t)a.n + (uint64_t)t) * 2u + 1u) * SPLITMIX_GOLDEN);
+            }
+            for (int32_t t0 = 2 * threadIdx.x; !s_fast && t0 < n2; t0 += 4 * R2_THREADS) {
                 const int32_t t1 = t0 + 2 * R2_THREADS;
                 const float4 v0 = __ldg(reinterpret_cast<const float4*>(a.base) + (t0 >> 1));
                 float4 v1 = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -1220,7 +1272,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                     one(t1 + 1, v1.z, v1.w);
                 }
             }
-            for (int32_t t = n2 + threadIdx.x; t < a.n; t += R2_THREADS)
+            for (int32_t t = n2 + threadIdx.x; !s_fast && t < a.n; t += R2_THREADS)
                 one(t, __ldg(a.base + 2 * (int64_t)t), __ldg(a.base + 2 * (int64_t)t + 1));
             mn[A] = (unsigned long long)dmn << 32;
             mx[A] = (unsigned long long)dmx << 32;
@@ -1366,10 +1418,14 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
                 const bool one_arch = cC != a.n || cG != a.n;   // some D are the one-arch sentinels
                 constexpr int32_t CH = 128, STEP = CH * R2_WARPS;
-                for (int32_t cb0 = w * CH; cb0 < a.n; cb0 += 2 * STEP) {
-                    uint32_t Dv[2][4], nx[2];
+#ifndef MP_EQ_H
+#define MP_EQ_H 2
+#endif
+                constexpr int EQ_H = MP_EQ_H;   // 128-position chunks per warp in flight
+                for (int32_t cb0 = w * CH; cb0 < a.n; cb0 += EQ_H * STEP) {
+                    uint32_t Dv[EQ_H][4], nx[EQ_H];
 #pragma unroll
-                    for (int h = 0; h < 2; h++) {
+                    for (int h = 0; h < EQ_H; h++) {
                         const int32_t p4 = cb0 + h * STEP + lane * 4;
                         if (p4 + 4 <= a.n) {
                             const uint4 v = __ldcg(reinterpret_cast<const uint4*>(dsorted + p4));
@@ -1381,7 +1437,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                         nx[h] = (lane == 31 && p4 + 4 < a.n) ? __ldcg(dsorted + p4 + 4) : 0u;
                     }
 #pragma unroll
-                    for (int h = 0; h < 2; h++) {
+                    for (int h = 0; h < EQ_H; h++) {
                         const int32_t cb = cb0 + h * STEP;
                         if (cb >= a.n) break;
                         const int32_t p4 = cb + lane * 4;

@@ -1,10 +1,3 @@
-mkdir -p gpurun_out/s16
-cp ab/libmp_kid0.so paper_conf_ipps_tayebbfg24_b200/libmp.so
-timeout 2400 python -m pytest tests -m gpu -q -x > gpurun_out/s16/gpu_tests_kid0.log 2>&1; echo tests_kid0=$?; tail -2 gpurun_out/s16/gpu_tests_kid0.log
-cp ab/libmp_kid.so paper_conf_ipps_tayebbfg24_b200/libmp.so
-timeout 2400 python -m pytest tests -m gpu -q -x > gpurun_out/s16/gpu_tests_kid.log 2>&1; echo tests_kid=$?; tail -2 gpurun_out/s16/gpu_tests_kid.log
-for v in flow2 kid kid0 kidb8; do
-  cp ab/libmp_$v.so paper_conf_ipps_tayebbfg24_b200/libmp.so
-  for c in c2 lu64 c3 c4; do echo "== $v"; timeout 300 python tools/ingest_breakdown.py $c 5 2>&1 | head -1 | cut -c1-200; done
-done
-cp ab/libmp_kid.so paper_conf_ipps_tayebbfg24_b200/libmp.so
+mkdir -p gpurun_out/s17
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -m gpu -k "replica or c5" > gpurun_out/s17/rep_tests.log 2>&1; echo tests=$?; tail -2 gpurun_out/s17/rep_tests.log
+VARS="eq2 k2fast" RS="4096 512" bash tools/ab.sh
