@@ -54,6 +54,8 @@ struct mp_dag {
     int32_t* b_pof = nullptr;
     int32_t* b_bar = nullptr;   // grid barrier: arrivals [0], release flag [32]
     int4* b_colr = nullptr;     // one-block Kahn: per edge {target, its row start, row end, 0}
+    int32_t* b_rrow = nullptr;  // k_lvl_flow: predecessor CSR offsets [n+1]
+    int32_t* b_rcol = nullptr;  // k_lvl_flow: predecessor ids [E]
     std::map<const void*, size_t> caps;  // capacity (bytes) of every grow-only field
 };
 

@@ -173,7 +173,7 @@ void mp_free(mp_dag* dag) {
                     dag->qof,     dag->nodeq, dag->rowq, dag->colq,  dag->lvlq,      dag->nodep,
                     dag->rowp,    dag->colp, dag->lvlp,  dag->err,   dag->ws,        dag->sort_status,
                     dag->scan_status, dag->tickets, dag->b_rem, dag->b_f0, dag->b_f1, dag->b_counts,
-                    dag->b_kout, dag->b_pof, dag->b_bar, dag->b_colr};
+                    dag->b_kout, dag->b_pof, dag->b_bar, dag->b_colr, dag->b_rrow, dag->b_rcol};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     delete dag;

@@ -127,6 +127,30 @@ def test_deep_chain_and_wide_star():
     compare(n, s2, d2, random_dags.dyadic_durations(n, 2, 4), np.ones(2, np.int32))
 
 
+@pytest.mark.parametrize("seed,n,deg,span", [
+    (11, 3000, 3.0, 8),          # chains inside 32-id chunks
+    (12, 60000, 6.0, 16),
+    (13, 200000, 4.0, None),     # long-range edges
+    (14, 100000, 40.0, 4096),    # ~1,280 predecessors per chunk: pending list full -> in-place waits
+])
+def test_id_order_dags(seed, n, deg, span):
+    """Id order is topological (every edge to a larger id, as in a sequential task flow):
+    the levels come from the pull dataflow k_lvl_flow instead of the level-synchronous Kahn;
+    levels, level order, q-space and the whole score path bit-exact with the oracle."""
+    src, dst = random_dags.random_dag(n, deg, seed, dup=0.2, permute=False, max_span=span)
+    assert (src < dst).all()
+    compare(n, src, dst, random_dags.dyadic_durations(n, 2, seed, p_inf=0.1, tiny_set=True), np.ones(2, np.int32))
+
+
+def test_id_order_fan_in():
+    """One sink with 99,999 predecessors, id order topological (k_lvl_flow, one chunk waiting
+    on a full pending list)."""
+    n = 100000
+    s = np.arange(n - 1, dtype=np.int32)
+    d = np.full(n - 1, n - 1, np.int32)
+    compare(n, s, d, random_dags.dyadic_durations(n, 2, 5), np.ones(2, np.int32))
+
+
 def test_one_block_kahn_frontier_spill():
     """a2 ingest, one-block Kahn (n <= 48K): the first sfcap (<= 8192) entries of a frontier
     live in shared memory, the rest spill to the global list -- levels narrower than, equal
