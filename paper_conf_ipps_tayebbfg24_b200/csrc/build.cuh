@@ -393,6 +393,9 @@ __global__ void k_rcsr_fill(int32_t n, const int32_t* __restrict__ row_ptr, cons
 constexpr int LVL_THREADS = 256;
 constexpr int LVL_PCAP = 1024;   // pending-predecessor list per warp (4 B id + 1 B owner lane)
 constexpr int LVL_PPL = 8;
+#ifndef MP_LVL_BACKOFF_MAX
+#define MP_LVL_BACKOFF_MAX 256
+#endif
 constexpr uint32_t LVL_NOT_READY = 0xFFFFFFFFu;
 MP_INLINE uint32_t lvl_ld(const uint32_t* p) {
     uint32_t v;
@@ -490,8 +493,9 @@ __global__ void __launch_bounds__(LVL_THREADS, 4) k_lvl_flow(int32_t n, const in
         // rounds: poll every unresolved list entry once, then publish the lanes with nothing
         // pending (this is what resolves the entries that point inside the chunk)
         bool done = v >= n;
-        uint32_t rounds = 0;
+        uint32_t rounds = 0, backoff = 32;
         while (true) {
+            bool prog = false;
             for (uint32_t i0 = 0; i0 < npend; i0 += 32 * LVL_PPL) {
                 int32_t ent[LVL_PPL];
 #pragma unroll
@@ -510,6 +514,7 @@ __global__ void __launch_bounds__(LVL_THREADS, 4) k_lvl_flow(int32_t n, const in
                         atomicMax(&smax[w][ow], xv[k] + 1u);
                         atomicSub(&scnt[w][ow], 1);
                         spend[w][i] = -1;
+                        prog = true;
                     }
             }
             __syncwarp();
@@ -518,8 +523,17 @@ __global__ void __launch_bounds__(LVL_THREADS, 4) k_lvl_flow(int32_t n, const in
                 asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(level + v), "r"(lv) : "memory");
                 lmax = max(lmax, lv);
                 done = true;
+                prog = true;
             }
             if (__all_sync(0xffffffffu, done)) break;
+            // a round without progress: back off, so waiting warps leave the issue slots to the
+            // warps that have work (the kernel is issue-bound on c4 without it)
+            if (__any_sync(0xffffffffu, prog)) {
+                backoff = 32;
+            } else {
+                __nanosleep(backoff);
+                backoff = min(backoff * 2u, (uint32_t)MP_LVL_BACKOFF_MAX);
+            }
             if (++rounds >= (1u << 20)) {   // no progress possible (cannot happen on a DAG)
                 stuck = true;
                 break;

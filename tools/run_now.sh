@@ -1,6 +1,8 @@
-mkdir -p gpurun_out/s21
-timeout 1500 python -m pytest tests -m gpu -q -x > gpurun_out/s21/gpu_tests.log 2>&1; echo tests=$?; tail -2 gpurun_out/s21/gpu_tests.log
-timeout 300 python bench.py --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/s21/bench_c5.json 2>gpurun_out/s21/bench_c5.err; python -c "
-import json; d=json.loads(open('gpurun_out/s21/bench_c5.json').read().strip().splitlines()[-1]); print('c5', round(d['ms_per_step'],3), d.get('build_ms'), d['e2e']['value'])"
-for c in c2 c3 c4; do timeout 300 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/s21/bench_$c.json 2>/dev/null; python -c "
-import json; d=json.loads(open('gpurun_out/s21/bench_$c.json').read().strip().splitlines()[-1]); print('$c', round(d['ms_per_step'],3), 'build', round(d['build_ms'],3))"; done
+mkdir -p gpurun_out/s26
+timeout 300 python -m pytest tests/test_gpu_parity.py -m gpu -q -x -k "configs_bit_exact or c4_bit or id_order" > gpurun_out/s26/quick.log 2>&1; rc=$?; echo quick=$rc; tail -2 gpurun_out/s26/quick.log
+if [ $rc -ne 0 ]; then exit 0; fi
+for rep in 1 2; do for v in head bo64 bo256 bo1024; do
+  cp ab/libmp_$v.so paper_conf_ipps_tayebbfg24_b200/libmp.so
+  for c in c2 hier c3 c4 c4fmm; do echo "== $v $(timeout 120 python tools/ingest_breakdown.py $c 10 2>&1 | head -1 | cut -c1-60)"; done
+done; done
+cp ab/libmp_bo256.so paper_conf_ipps_tayebbfg24_b200/libmp.so
