@@ -376,16 +376,40 @@ struct KahnArgs {
 // a level's grid barrier plus its chain of dependent loads.
 
 // predecessor CSR: rcol[rrow[v] ...] = predecessors of v (any order: only their max is used);
-// a warp per run of rows, lanes over a row's successors
+// a warp takes rpw consecutive rows and spreads their edges over its lanes (warp scan of the
+// row lengths + a 5-step shuffle search for each edge's row, as k_csr_emit)
 __global__ void k_rcsr_fill(int32_t n, const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                            const int32_t* __restrict__ rrow, int32_t* fillc, int32_t* rcol) {
+                            const int32_t* __restrict__ rrow, int32_t* fillc, int32_t* rcol, int rpw) {
     const int lane = threadIdx.x & 31;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t u = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; u < n; u += nw) {
-        const int32_t e0 = __ldg(row_ptr + u), e1 = __ldg(row_ptr + u + 1);
-        for (int32_t e = e0 + lane; e < e1; e += 32) {
-            const int32_t v = __ldg(col + e);
-            rcol[__ldg(rrow + v) + atomicAdd(fillc + v, 1)] = (int32_t)u;
+    for (int64_t r0 = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5) * rpw; r0 < n; r0 += nw * rpw) {
+        const int64_t r = r0 + lane;
+        int32_t sb = 0, c = 0;
+        if (lane < rpw && r < n) {
+            sb = __ldg(row_ptr + r);
+            c = __ldg(row_ptr + r + 1) - sb;
+        }
+        int32_t inc = c;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const int32_t y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        const int32_t exc = inc - c;
+        const int32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+        const int32_t e0 = __shfl_sync(0xffffffffu, sb, 0);   // the rows' edges are contiguous
+        for (int32_t kb = 0; kb < tot; kb += 32) {
+            const int32_t k = kb + lane;
+            int lo = 0;
+#pragma unroll
+            for (int step = 16; step >= 1; step >>= 1) {
+                const int32_t ev = __shfl_sync(0xffffffffu, exc, lo + step);
+                if (ev <= k) lo += step;
+            }
+            if (k < tot) {
+                const int32_t v = __ldg(col + e0 + k);
+                rcol[__ldg(rrow + v) + atomicAdd(fillc + v, 1)] = (int32_t)(r0 + lo);
+            }
         }
     }
 }
@@ -1037,7 +1061,7 @@ inline mp_status build_into(mp_dag* dag, int32_t n, int64_t m, const int32_t* d_
         }
         CK(cudaMemsetAsync(rem, 0, (size_t)n * 4, st));
         MP_LAUNCH(k_rcsr_fill, grid_for((int64_t)n * 32), 256, 0, st, n, dag->row_ptr, dag->col, dag->b_rrow, rem,
-                  dag->b_rcol);
+                  dag->b_rcol, rows_per_warp(n, (int64_t)grid_for((int64_t)n * 32) * 8));
         CK(cudaMemsetAsync(dag->level, 0xff, (size_t)n * 4, st));
         CK(cudaMemsetAsync(dag->tickets + 60, 0, 4, st));
         int bps = 0;
