@@ -57,6 +57,8 @@ struct mp_dag {
     int32_t* b_rrow = nullptr;  // k_lvl_flow: predecessor CSR offsets [n+1]
     int32_t* b_rcol = nullptr;  // k_lvl_flow: predecessor ids [E]
     std::map<const void*, size_t> caps;  // capacity (bytes) of every grow-only field
+    cudaStream_t side = nullptr;         // replica path: K2's pre-sort pass beside K1
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr;
 };
 
 namespace mph {
@@ -80,6 +82,16 @@ inline mp_status fail(mp_status s, const char* fmt, ...) {
             return mph::fail(e__ == cudaErrorMemoryAllocation ? MP_ERR_NOMEM : MP_ERR_CUDA, \
                              "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e__)); \
     } while (0)
+
+// side stream + two events of a handle (created on first use, on the handle's device)
+inline mp_status ensure_side_stream(mp_dag* dag) {
+    if (dag->side) return MP_OK;
+    if (cudaStreamCreateWithFlags(&dag->side, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&dag->ev_a, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&dag->ev_b, cudaEventDisableTiming) != cudaSuccess)
+        return fail(MP_ERR_CUDA, "side stream: %s", cudaGetErrorString(cudaGetLastError()));
+    return MP_OK;
+}
 
 #define MP_TRY(expr)                   \
     do {                               \

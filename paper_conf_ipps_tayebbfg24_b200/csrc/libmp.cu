@@ -176,6 +176,9 @@ void mp_free(mp_dag* dag) {
                     dag->b_kout, dag->b_pof, dag->b_bar, dag->b_colr, dag->b_rrow, dag->b_rcol};
     for (void* p : ptrs)
         if (p) cudaFree(p);
+    if (dag->ev_a) cudaEventDestroy(dag->ev_a);
+    if (dag->ev_b) cudaEventDestroy(dag->ev_b);
+    if (dag->side) cudaStreamDestroy(dag->side);
     delete dag;
 }
 

@@ -74,6 +74,14 @@ struct Rep2Args {
     int32_t* qtask;              // [R][n*A] or null
     mp_queue_summary* sum;       // [R][A]
     uint32_t* ticket;
+    // two archs: K2 split for overlap with K1 (rep2_launch).  mode 1 = pre-sort pass (hash +
+    // sort of replicas [0, pre_R) into pp_pos / pp_ds, launched beside K1 on the SMs K1
+    // leaves idle); mode 2 = the main pass, replicas < pre_R start after their sort.
+    int mode;
+    int32_t pre_R;
+    uint16_t* pp_pos;            // [pre_R][npad] sorted positions
+    uint32_t* pp_ds;             // [pre_R][npad] D in sorted order
+    uint32_t* ticket_pre;
 };
 
 template <int A>
@@ -1143,8 +1151,10 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
     }
     const uint64_t kfl = (uint64_t)s_flo << 32, kfh = (uint64_t)s_fhi << 32;
     const R3Geo gf = r3_geo(kfl, kfh > kfl ? kfh : kfl + (1ull << 32));
+    const bool presort = A == 2 && a.mode == 1;
+    const int64_t Rlim = presort ? a.pre_R : a.R;
     while (true) {
-        if (threadIdx.x == 0) s_tick = atomicAdd(a.ticket, 1u);
+        if (threadIdx.x == 0) s_tick = atomicAdd(presort ? a.ticket_pre : a.ticket, 1u);
         if (threadIdx.x <= A) {
             s_min[threadIdx.x] = ~0ull;
             s_max[threadIdx.x] = 0ull;
@@ -1152,8 +1162,17 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         __syncthreads();
         const int64_t rl = s_tick;
         __syncthreads();
-        if (rl >= a.R) break;
+        if (rl >= Rlim) break;
         K2_PHASE(0);
+        // replicas sorted by the pre-sort pass: their sorted order is read back (post); the
+        // pre-sort pass itself writes it per replica
+        const bool post = A == 2 && a.mode == 2 && rl < a.pre_R;
+        uint16_t* ppos_r = ppos;
+        uint32_t* dsorted_r = dsorted;
+        if (A == 2 && (presort || post)) {
+            ppos_r = a.pp_pos + rl * npad;
+            dsorted_r = a.pp_ds + rl * npad;
+        }
         const int64_t r = a.r0 + rl;
         const float CP = a.cp[rl];
         float hdv[A];
@@ -1164,7 +1183,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         unsigned long long mn[A + 1], mx[A + 1];
 #pragma unroll
         for (int b = 0; b <= A; b++) { mn[b] = ~0ull; mx[b] = 0ull; }
-        const bool pre = A == 2 && geo && s_geo_ok;
+        const bool pre = A == 2 && geo && s_geo_ok && !post;
         if (pre) {   // restore the cached sub-bin geometry, zero the fine counters
             const uint16_t* g16 = reinterpret_cast<const uint16_t*>(geo);
             for (int32_t b = threadIdx.x; b < R3_NC; b += R2_THREADS) {
@@ -1175,7 +1194,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             if (threadIdx.x == 0) s_out = 0u;
             __syncthreads();
         }
-        if constexpr (A == 2) {
+        if constexpr (A == 2) if (!post) {
             // two archs: only the orderable d is needed to sort (crit is read for equal-gain runs).
             // 4 tasks per thread and trip (t, t+1 | t+2048, t+2049): both 16-byte base loads
             // are issued before the hashing
@@ -1359,10 +1378,10 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
         if constexpr (A == 2) {
             // one sort by (D, critc, t) -> P; then both queues in one pass (runs of equal gain fixed up)
             K2_PHASE(1);
-            {
+            if (!post) {
                 const uint64_t amin = s_min[A] & ~0xFFFFFFFFull, amax = s_max[A] & ~0xFFFFFFFFull;
                 const R3Keys K{dkey, nullptr, fbuf};
-                const R3PosOut O{ppos, dsorted};
+                const R3PosOut O{ppos_r, dsorted_r};
                 if (pre && !s_out) {
                     r3_sort<uint32_t>(K, O, a.n, gf.lo, gf.hi, S, s_geo_nfb);
                 } else if (geo && !pre && amin >= gf.lo && amax <= gf.hi && gf.lo < gf.hi) {
@@ -1379,6 +1398,10 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 }
             }
             K2_PHASE(7);
+            if (presort) {   // the pre-sort pass stops here (its order is in pp_pos / pp_ds)
+                __syncthreads();
+                continue;
+            }
             if (threadIdx.x == 0) { s_flag = 0; s_h0 = 0xffffffffu; s_h1 = 0xffffffffu; }
             __syncthreads();
             const int32_t cC = a.counts[rl * 2 + 0], cG = a.counts[rl * 2 + 1];
@@ -1398,11 +1421,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
             const int32_t nw = (a.n + 31) / 32;
             uint32_t* e0 = reinterpret_cast<uint32_t*>(Ps + ((a.n + 63) & ~63));
             uint32_t* e1 = e0 + nw;
-            {   // 16-byte copies (ppos and Ps are 32-byte aligned)
+            {   // 16-byte copies (ppos_r and Ps are 32-byte aligned)
                 const int32_t n8 = a.n >> 3;
                 for (int32_t i = threadIdx.x; i < n8; i += R2_THREADS)
-                    reinterpret_cast<uint4*>(Ps)[i] = __ldcg(reinterpret_cast<const uint4*>(ppos) + i);
-                for (int32_t i = (n8 << 3) + threadIdx.x; i < a.n; i += R2_THREADS) Ps[i] = ppos[i];
+                    reinterpret_cast<uint4*>(Ps)[i] = __ldcg(reinterpret_cast<const uint4*>(ppos_r) + i);
+                for (int32_t i = (n8 << 3) + threadIdx.x; i < a.n; i += R2_THREADS) Ps[i] = ppos_r[i];
             }
             {
                 K2_PHASE(8);
@@ -1428,13 +1451,13 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                     for (int h = 0; h < EQ_H; h++) {
                         const int32_t p4 = cb0 + h * STEP + lane * 4;
                         if (p4 + 4 <= a.n) {
-                            const uint4 v = __ldcg(reinterpret_cast<const uint4*>(dsorted + p4));
+                            const uint4 v = __ldcg(reinterpret_cast<const uint4*>(dsorted_r + p4));
                             Dv[h][0] = v.x; Dv[h][1] = v.y; Dv[h][2] = v.z; Dv[h][3] = v.w;
                         } else {
 #pragma unroll
-                            for (int j = 0; j < 4; j++) Dv[h][j] = p4 + j < a.n ? __ldcg(dsorted + p4 + j) : 0u;
+                            for (int j = 0; j < 4; j++) Dv[h][j] = p4 + j < a.n ? __ldcg(dsorted_r + p4 + j) : 0u;
                         }
-                        nx[h] = (lane == 31 && p4 + 4 < a.n) ? __ldcg(dsorted + p4 + 4) : 0u;
+                        nx[h] = (lane == 31 && p4 + 4 < a.n) ? __ldcg(dsorted_r + p4 + 4) : 0u;
                     }
 #pragma unroll
                     for (int h = 0; h < EQ_H; h++) {
@@ -1507,7 +1530,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 for (uint32_t i = threadIdx.x; i < nn; i += R2_THREADS) {
                     const uint32_t ent = nearl[i];
                     const int32_t p = (int32_t)(ent & 0x7FFFFFFFu);
-                    const uint32_t Da = __ldcg(dsorted + p), Db = __ldcg(dsorted + p + 1);   // no sentinels here
+                    const uint32_t Da = __ldcg(dsorted_r + p), Db = __ldcg(dsorted_r + p + 1);   // no sentinels here
                     const float da = u2f((Da & 0x80000000u) ? (Da & 0x7FFFFFFFu) : ~Da);
                     const float db = u2f((Db & 0x80000000u) ? (Db & 0x7FFFFFFFu) : ~Db);
                     const float d0 = (ent >> 31) ? __fsub_rn(0.0f, da) : da, d1 = (ent >> 31) ? __fsub_rn(0.0f, db) : db;
@@ -1722,6 +1745,27 @@ __global__ void __launch_bounds__(R2_THREADS, 1) k_rep2_sort(Rep2Args a) {
                 s_min[threadIdx.x] = ~0ull;
                 s_max[threadIdx.x] = 0ull;
             }
+            if (post) {   // sorted by the pre-sort pass: this CTA has no D(t) of the replica yet
+                for (int32_t t = threadIdx.x; t < a.n; t += R2_THREADS) {
+                    float x[2];
+                    uint32_t en = 0;
+                    bool dummy = false;
+                    const uint64_t c0 = ((uint64_t)r * (uint64_t)a.n + (uint64_t)t) * 2u + 1u;
+#pragma unroll
+                    for (int b = 0; b < 2; b++) {
+                        x[b] = canon_dur(perturb(__ldg(a.base + 2 * (int64_t)t + b), a.seed, a.sigma, c0 + b), dummy);
+                        if (((a.emask >> b) & 1u) && !is_inf(x[b])) en |= 1u << b;
+                    }
+                    uint32_t D;
+                    if (en == 3u) {
+                        const uint32_t db = f2u(__fsub_rn(x[1], x[0]));
+                        D = (db >> 31) ? ~db : (db | 0x80000000u);
+                    } else {
+                        D = en == 1u ? 0xFFFFFFFFu : 0u;
+                    }
+                    dkey[t] = D;
+                }
+            }
             __syncthreads();
             unsigned long long fmn[A], fmx[A];
 #pragma unroll
@@ -1796,45 +1840,9 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     const int32_t n = dag->n;
     const int64_t groups = (R + 31) / 32;
     const int grid2 = std::max(1, std::min<int>(R, dag->num_sms));
-    const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
-    size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
-                   align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 8) +
-                   align256((size_t)grid2 * ((n + 15) & ~15) * 4) + align256((size_t)grid2 * R3_GEO_BYTES);
-    MP_TRY(ensure_ws(dag, bytes, st));
-    Arena ar{dag->ws, dag->ws_cap};
-    Rep2Args a{};
-    a.n = n;
-    a.A = A;
-    a.L = dag->L;
-    a.R = R;
-    a.r0 = r0;
-    a.lvlq = dag->lvlq;
-    a.nodeq = dag->nodeq;
-    a.rowq = dag->rowq;
-    a.colq = dag->colq;
-    a.qof = dag->qof;
-    a.base = base;
-    a.emask = emask;
-    a.seed = seed;
-    a.sigma = sigma;
-    a.bl32 = ar.take<float>((size_t)groups * n * 32);
-    a.blT = ar.take<float>(blT_elems);
-    a.cp = cp;
-    a.hd = ar.take<uint32_t>((size_t)R * A);
-    a.counts = ar.take<int32_t>((size_t)R * A);
-    a.brw = ar.take<unsigned long long>((size_t)R * A * 2);
-    a.err = dag->err;
-    const size_t npad = (size_t)((n + 15) & ~15);
-    a.s_cold = ar.take<uint32_t>((size_t)grid2 * npad * (A + 1));
-    a.s_key = ar.take<uint32_t>((size_t)grid2 * npad * 2);   // hot scratch: s_key and s_pi adjacent
-    a.s_pi = ar.take<uint16_t>((size_t)grid2 * npad * 2);
-    a.s_geo = A == 2 ? ar.take<unsigned char>((size_t)grid2 * R3_GEO_BYTES) : nullptr;
-    a.qtask = qtask;
-    a.sum = sum;
-    a.ticket = dag->tickets + 56;
-    static std::atomic<uint64_t> attr{0};
     const int smem1 = 32 * 32 * 33 * 4;
     const int smem2 = (int)r3_smem_bytes();
+    static std::atomic<uint64_t> attr{0};
     if (first_on_device(attr)) {
         MP_CUDA(cudaFuncSetAttribute(k_rep2_bl<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem1));
         MP_CUDA(cudaFuncSetAttribute(k_rep2_bl<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem1));
@@ -1845,11 +1853,6 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         MP_CUDA(cudaFuncSetAttribute(k_rep2_sort<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2));
         MP_CUDA(cudaFuncSetAttribute(k_rep2_sort<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2));
     }
-    // statistics are merged with atomics: zero them (and CP) first
-    MP_CUDA(cudaMemsetAsync(cp, 0, (size_t)R * 4, st));
-    MP_CUDA(cudaMemsetAsync(a.hd, 0, (size_t)R * A * 4, st));
-    MP_CUDA(cudaMemsetAsync(a.counts, 0, (size_t)R * A * 4, st));
-    MP_CUDA(cudaMemsetAsync(a.brw, 0, (size_t)R * A * 16, st));
     // cluster size: enough CTAs per 32-replica group to cover the SMs (strong scaling keeps K1 short)
     // (8-CTA clusters and a cross-CTA dataflow mode -- bl lines as ready flags polled from L2 --
     // measured slower: R = 512 K1 0.98 ms (4-CTA, level barriers) vs 1.58 ms (8-CTA) and
@@ -1897,6 +1900,69 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         std::lock_guard<std::mutex> lk(cs_mu);
         cs_memo[{dag->device, groups * 8 + A}] = cs;
     }
+    // K2 pre-sort pass (two archs, one CTA per group): K1 leaves num_sms - groups SMs idle for
+    // its whole level walk; K2's hash + sort phases of the first pre_R replicas run there
+    // meanwhile (about 17 replicas per idle SM fit in K1's time: K1 walks n nodes x 32 replicas
+    // per SM, a pre-sort takes ~1/20 of that per replica); the main K2 pass then only finishes
+    // those replicas
+    const int idle = dag->num_sms - (int)(groups * cs);
+    // (clusters: fewer per SM -- the pre-sort CTAs then also delay some of K1's clusters; measured
+    // net: R = 512 1.53 -> 1.43 ms, 1024 2.09 -> 2.07, 2048 3.42 -> 3.40, 4096 6.01 -> 5.82)
+    const int per_idle = cs == 1 ? 17 : 6;
+    const int32_t pre_R = (A == 2 && idle > 0 && R >= 2 * 148) ? std::min<int32_t>(R / 4, idle * per_idle) : 0;
+    const size_t npad_b = (size_t)((n + 15) & ~15);
+    const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
+    size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
+                   align256((size_t)R * A * 16) + align256((size_t)grid2 * ((n + 15) & ~15) * 4 * (A + 1)) + align256((size_t)grid2 * ((n + 15) & ~15) * 8) +
+                   align256((size_t)grid2 * ((n + 15) & ~15) * 4) + align256((size_t)grid2 * R3_GEO_BYTES) +
+                   align256((size_t)pre_R * npad_b * 2) + align256((size_t)pre_R * npad_b * 4);
+    MP_TRY(ensure_ws(dag, bytes, st));
+    Arena ar{dag->ws, dag->ws_cap};
+    Rep2Args a{};
+    a.n = n;
+    a.A = A;
+    a.L = dag->L;
+    a.R = R;
+    a.r0 = r0;
+    a.lvlq = dag->lvlq;
+    a.nodeq = dag->nodeq;
+    a.rowq = dag->rowq;
+    a.colq = dag->colq;
+    a.qof = dag->qof;
+    a.base = base;
+    a.emask = emask;
+    a.seed = seed;
+    a.sigma = sigma;
+    a.bl32 = ar.take<float>((size_t)groups * n * 32);
+    a.blT = ar.take<float>(blT_elems);
+    a.cp = cp;
+    a.hd = ar.take<uint32_t>((size_t)R * A);
+    a.counts = ar.take<int32_t>((size_t)R * A);
+    a.brw = ar.take<unsigned long long>((size_t)R * A * 2);
+    a.err = dag->err;
+    const size_t npad = (size_t)((n + 15) & ~15);
+    a.s_cold = ar.take<uint32_t>((size_t)grid2 * npad * (A + 1));
+    a.s_key = ar.take<uint32_t>((size_t)grid2 * npad * 2);   // hot scratch: s_key and s_pi adjacent
+    a.s_pi = ar.take<uint16_t>((size_t)grid2 * npad * 2);
+    a.s_geo = A == 2 ? ar.take<unsigned char>((size_t)grid2 * R3_GEO_BYTES) : nullptr;
+    a.qtask = qtask;
+    a.sum = sum;
+    a.ticket = dag->tickets + 56;
+    a.mode = 0;
+    a.pre_R = pre_R;
+    a.pp_pos = pre_R > 0 ? ar.take<uint16_t>((size_t)pre_R * npad_b) : nullptr;
+    a.pp_ds = pre_R > 0 ? ar.take<uint32_t>((size_t)pre_R * npad_b) : nullptr;
+    a.ticket_pre = dag->tickets + 57;
+    // statistics are merged with atomics: zero them (and CP) first
+    MP_CUDA(cudaMemsetAsync(cp, 0, (size_t)R * 4, st));
+    MP_CUDA(cudaMemsetAsync(a.hd, 0, (size_t)R * A * 4, st));
+    MP_CUDA(cudaMemsetAsync(a.counts, 0, (size_t)R * A * 4, st));
+    MP_CUDA(cudaMemsetAsync(a.brw, 0, (size_t)R * A * 16, st));
+    if (pre_R > 0) {   // the pre-sort pass starts with K1, on a side stream
+        MP_TRY(ensure_side_stream(dag));
+        MP_CUDA(cudaEventRecord(dag->ev_a, st));
+        MP_CUDA(cudaStreamWaitEvent(dag->side, dag->ev_a, 0));
+    }
     for (;; cs = cs > 1 ? cs - 1 : 1) {
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3((unsigned)(groups * cs));
@@ -1919,6 +1985,23 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
         if (e == cudaSuccess) break;
         cudaGetLastError();
         if (cs == 1) return fail(MP_ERR_CUDA, "k_rep2_bl launch: %s", cudaGetErrorString(e));
+    }
+    if (pre_R > 0) {
+        MP_CUDA(cudaMemsetAsync(a.ticket_pre, 0, 4, dag->side));
+        Rep2Args ap = a;
+        ap.mode = 1;
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3((unsigned)idle);
+        cfg.blockDim = dim3(R2_THREADS);
+        cfg.dynamicSmemBytes = (size_t)smem2;
+        cfg.stream = dag->side;
+        {
+            mph::ProfScope ps("k_rep2_pre", dag->side);
+            MP_CUDA(cudaLaunchKernelEx(&cfg, k_rep2_sort<A>, ap));
+        }
+        MP_CUDA(cudaEventRecord(dag->ev_b, dag->side));
+        MP_CUDA(cudaStreamWaitEvent(st, dag->ev_b, 0));
+        a.mode = 2;
     }
     MP_CUDA(cudaMemsetAsync(a.ticket, 0, 4, st));
     {
