@@ -18,7 +18,7 @@ done
 timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > $O/bench_ref_c5.json 2> $O/bench_ref.err; echo "ref rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_c5.csv \
    python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-tlevel > $O/launches_c5.log 2>&1; echo "launches rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_rep2 -c 2 -o $O/full_c5 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_rep2 -c 3 -o $O/full_c5 \
    python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-tlevel > $O/full_c5.log 2>&1; echo "full c5 rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_bl_small|k_sort_pass|k_kahn" -c 3 -o $O/full_c2 \
    python bench.py --config c2 --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-probe --no-tlevel > $O/full_c2.log 2>&1; echo "full c2 rc=$?"
