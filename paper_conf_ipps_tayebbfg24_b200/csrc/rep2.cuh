@@ -1906,10 +1906,20 @@ inline mp_status rep2_launch(mp_dag* dag, const float* base, uint32_t emask, uin
     // per SM, a pre-sort takes ~1/20 of that per replica); the main K2 pass then only finishes
     // those replicas
     const int idle = dag->num_sms - (int)(groups * cs);
-    // (clusters: fewer per SM -- the pre-sort CTAs then also delay some of K1's clusters; measured
-    // net: R = 512 1.53 -> 1.43 ms, 1024 2.09 -> 2.07, 2048 3.42 -> 3.40, 4096 6.01 -> 5.82)
-    const int per_idle = cs == 1 ? 17 : 6;
-    const int32_t pre_R = (A == 2 && idle > 0 && R >= 2 * 148) ? std::min<int32_t>(R / 4, idle * per_idle) : 0;
+    // (clusters: fewer per SM -- the pre-sort CTAs then also delay some of K1's clusters; swept
+    // 4..15 per idle SM, measured net: R = 512 1.53 -> 1.44 ms, 1024 2.09 -> 1.98, 2048 3.42 ->
+    // 3.33, 4096 6.01 -> 5.81 with 17 / 9: 19 leaves the pre-sort too close to K1)
+#ifndef MP_PRE_FLOW
+#define MP_PRE_FLOW 17
+#endif
+#ifndef MP_PRE_CL
+#define MP_PRE_CL 9
+#endif
+    const int per_idle = cs == 1 ? MP_PRE_FLOW : MP_PRE_CL;
+#ifndef MP_PRE_DIV
+#define MP_PRE_DIV 4
+#endif
+    const int32_t pre_R = (A == 2 && idle > 0 && R >= 2 * 148) ? std::min<int32_t>(R / MP_PRE_DIV, idle * per_idle) : 0;
     const size_t npad_b = (size_t)((n + 15) & ~15);
     const size_t blT_elems = A == 2 ? 1 : (size_t)R * n;   // two archs: K2 reads K1's bl32 directly
     size_t bytes = align256((size_t)groups * n * 32 * 4) + align256(blT_elems * 4) + align256((size_t)R * A * 4) * 2 +
