@@ -1,4 +1,3 @@
-mkdir -p gpurun_out/meas
-timeout 900 python bench.py > gpurun_out/meas/bench_c5.json 2> gpurun_out/meas/bench_c5.err; echo "c5 rc=$?"
-python -c "
-import json; d=json.loads(open('gpurun_out/meas/bench_c5.json').read().strip().splitlines()[-1]); r=d['roofline']; print(d['ms_per_step'], d['value'], r['frac'], r['per_kernel_ms_per_step'])"
+mkdir -p gpurun_out/final
+timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/final/gpu_tests.log 2>&1; echo tests=$?; tail -2 gpurun_out/final/gpu_tests.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()"; echo smoke=$?
