@@ -228,6 +228,16 @@ __global__ void __launch_bounds__(1024) k_bl_small(int32_t L, const int32_t* __r
                 const int32_t e1 = srow[q + 1];
                 const int32_t v = snod[q];
                 float m = 0.0f;  // bl >= 0, and w + 0 = w: same as "bl = w without successors"
+                if constexpr (GBL) {   // bl in L2: a high out-degree node keeps 16 gathers in flight
+                    // (hier 0.61 -> 0.55 ms, lu64 0.35 -> 0.34; the shared-memory walk of c2 gains nothing)
+                    for (; e + 16 <= e1; e += 16) {
+                        float g[16];
+#pragma unroll
+                        for (int u = 0; u < 16; u++) g[u] = sbl[scol[e + u]];
+#pragma unroll
+                        for (int u = 0; u < 16; u++) m = fmaxf(m, g[u]);
+                    }
+                }
                 for (; e + 4 <= e1; e += 4)
                     m = fmaxf(m, fmaxf(fmaxf(sbl[scol[e]], sbl[scol[e + 1]]), fmaxf(sbl[scol[e + 2]], sbl[scol[e + 3]])));
                 for (; e < e1; e++) m = fmaxf(m, sbl[scol[e]]);

@@ -1,5 +1,3 @@
-mkdir -p gpurun_out/s33
-cp ab/libmp_lpt.so paper_conf_ipps_tayebbfg24_b200/libmp.so
-timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -m gpu -k "replica or c5" > gpurun_out/s33/rep_tests.log 2>&1; rc=$?; echo tests=$rc; tail -2 gpurun_out/s33/rep_tests.log
-if [ $rc -ne 0 ]; then exit 0; fi
-VARS="head lpt" RS="4096 2048 1024 512" bash tools/ab.sh
+mkdir -p gpurun_out/s35
+timeout 1500 python -m pytest tests -m gpu -q -x > gpurun_out/s35/gpu_tests.log 2>&1; echo tests=$?; tail -2 gpurun_out/s35/gpu_tests.log
+echo "== $(timeout 300 python tools/bl_time.py c2 lu64 hier 2>&1 | tail -3 | tr '\n' ' ' | cut -c1-250)"
