@@ -1,3 +1,4 @@
-mkdir -p gpurun_out/s35
-timeout 1500 python -m pytest tests -m gpu -q -x > gpurun_out/s35/gpu_tests.log 2>&1; echo tests=$?; tail -2 gpurun_out/s35/gpu_tests.log
-echo "== $(timeout 300 python tools/bl_time.py c2 lu64 hier 2>&1 | tail -3 | tr '\n' ' ' | cut -c1-250)"
+mkdir -p gpurun_out/meas
+for c in lu64 hier; do
+  timeout 600 python bench.py --config $c --steps 10 --warmup 3 --cpu-budget-s 8 > gpurun_out/meas/bench_$c.json 2> gpurun_out/meas/bench_$c.err; echo "$c rc=$?"
+done
